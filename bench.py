@@ -1,0 +1,360 @@
+#!/usr/bin/env python
+"""Benchmark: fused Stokes-FO residual + forward-AD Jacobian evaluation on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C4|C5|C1] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...   (N > 1: NCCL halo exchange)
+
+One step = one pass of the whole hot path over the
+configuration's mesh: R <- 0; stokesfo_jacobian (gather -> Ugrad -> Glen mu ->
+stress -> QP sum -> scatter-add R, plus the element Jacobians J_cell); at N > 1
+the NCCL halo sum of shared-node residuals.  Inputs are resident in HBM
+(C4: ~31 GB, far larger than the 126 MB L2, so no L2 flush is needed).
+Prints ONE JSON line on rank 0 (the driver's bench contract, DESIGN.md
+"Measurement").
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "Stokes-FO Jacobian+residual cells/s and achieved HBM GB/s at 1/2/4/8 B200"
+WORKLOADS = {
+    "C4": "C4 Antarctica-like 4 km footprint x 10 layers, hex8, 8 QPs, residual+Jacobian (BASELINE.json configs[3])",
+    "C5": "C5 Antarctica-like wedge6 (quads split), 10 layers, 6 QPs, residual+Jacobian (BASELINE.json configs[4])",
+    "C1": "C1/C2 tiny 16x16 footprint x 5 layers, hex8, residual+Jacobian (BASELINE.json configs[1])",
+}
+
+
+def bytes_per_launch(elem: str, cells: int, nodes: int) -> int:
+    """Algorithmic (compulsory) HBM bytes of one stokesfo_jacobian launch with
+    assembled R: per cell conn 4N +
+    GradBF 24NQ + wMeasure 8Q + k_c 8 + J_cell 8(2N)^2; per node U 16 + s 8 +
+    R read+write 32."""
+    N = 8 if elem == "hex8" else 6
+    Q = N
+    per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + 8 * (2 * N) ** 2
+    return cells * per_cell + nodes * (16 + 8 + 32)
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.file = None
+
+    def start(self):
+        try:
+            self.file = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=self.file, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.file.flush()
+        self.file.seek(0)
+        rows = [r.split(", ") for r in self.file.read().strip().splitlines() if r.strip()]
+        os.unlink(self.file.name)
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[1]))
+                mx = max(mx, float(r[2]))
+                for n, v in zip(names, r[5:9]):
+                    if v.strip().lower().startswith("active"):
+                        reasons.add(n)
+            except Exception:
+                continue
+        if not sm:
+            return None
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def build_mesh(cfg: str):
+    from paper_conf_sc_antepara0cw24_b200 import mesh_extrude, synth
+    fp, L, elem = synth.make_config(cfg)
+    conn, coords = mesh_extrude(fp.xy, fp.polys, fp.b, fp.H, L)
+    U = synth.velocity_balance(fp, L, seed=12)
+    s = synth.surface_nodal(fp, L)
+    kc = synth.flow_factor(fp, L)
+    return fp, L, elem, conn, coords, U, s, kc
+
+
+# ---------------------------------------------------------------------------
+# CPU oracle leg (cpu_baseline and --impl reference)
+# ---------------------------------------------------------------------------
+
+def oracle_sample_rate(elem, conn, coords, U, s, kc, target_s=12.0, start_cell=0):
+    """Time the oracle (as it stands) on a bounded contiguous sample of cells;
+    geometry precomputed untimed (the GPU contract).  Returns (cells/s, cells, s)."""
+    import numpy as np
+    import oracle as O
+    e = O.ELEM[elem]
+
+    def run(n):
+        cs = slice(start_cell, start_cell + n)
+        G, wm, _ = O.geometry(e, conn[cs], coords)
+        t0 = time.perf_counter()
+        O.evaluate(e, conn[cs], G, wm, U, surface=s, kc=kc[cs], mode="jac")
+        return time.perf_counter() - t0
+
+    n = 4096
+    dt = run(n)
+    n2 = int(min(conn.shape[0] - start_cell, max(n, n * target_s / max(dt, 1e-6))))
+    dt2 = run(n2)
+    return n2 / dt2, n2, dt2
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle timed on this host's cores (rank 0 only)."""
+    if rank != 0:
+        return 0
+    import oracle as O
+    cfg = args.config
+    fp, L, elem, conn, coords, U, s, kc = build_mesh(cfg)
+    import numpy as np
+    e = O.ELEM[elem]
+    # calibrate a per-step sample so that warmup + steps end within a few minutes
+    rate, _, _ = oracle_sample_rate(elem, conn, coords, U, s, kc, target_s=2.0)
+    per_step_s = min(8.0, 120.0 / max(1, args.steps + args.warmup))
+    n = int(max(1024, min(conn.shape[0], rate * per_step_s)))
+    G, wm, _ = O.geometry(e, conn[:n], coords)
+    for _ in range(args.warmup):
+        O.evaluate(e, conn[:n], G, wm, U, surface=s, kc=kc[:n], mode="jac")
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        O.evaluate(e, conn[:n], G, wm, U, surface=s, kc=kc[:n], mode="jac")
+    dt = (time.perf_counter() - t0) / args.steps
+    value = n / dt
+    sample = f"first {n} of {conn.shape[0]} cells per step (contiguous columns), geometry precomputed untimed"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "cells/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": WORKLOADS[cfg], "cells": int(conn.shape[0]), "sampled_cells_per_step": n},
+        "cpu_baseline": {"value": value, "unit": "cells/s", "cores": O.num_threads(), "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": value, "unit": "cells/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "gpu_launches": 0,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ---------------------------------------------------------------------------
+# GPU leg
+# ---------------------------------------------------------------------------
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO
+    from paper_conf_sc_antepara0cw24_b200.halo import Halo, LocalPart
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    fp, L, elem, conn_g, coords_g, U_g, s_g, kc_g = build_mesh(args.config)
+    part = LocalPart(conn_g, L, fp.nf, rank, world)
+    gids = part.gids
+    conn = torch.from_numpy(part.conn).to(dev)
+    coords = torch.from_numpy(np.ascontiguousarray(coords_g[gids])).to(dev)
+    surface = torch.from_numpy(np.ascontiguousarray(s_g[gids])).to(dev)
+    kc = torch.from_numpy(np.ascontiguousarray(kc_g[part.cell_lo:part.cell_hi])).to(dev)
+    U_host = torch.from_numpy(np.ascontiguousarray(U_g[gids])).pin_memory()
+    U = U_host.to(dev)
+    C, NN = conn.shape[0], coords.shape[0]
+    N = conn.shape[1]
+    stream = torch.cuda.current_stream(dev)
+    ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream)
+    J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device=dev)
+    R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
+    halo = None
+    if world > 1:
+        halo = Halo(part.neighbors, dev, pack=ctx.halo_pack, unpack_add=ctx.halo_unpack_add)
+    ctx.sync()
+    torch.cuda.synchronize(dev)
+
+    k0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    k1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+
+    def step(i=None):
+        R.zero_()
+        if i is not None:
+            k0[i].record(stream)
+        ctx.jacobian(U, J, R=R)
+        if i is not None:
+            k1[i].record(stream)
+        if halo is not None:
+            halo.exchange(R)
+
+    for _ in range(args.warmup):
+        step()
+    ctx.sync()
+
+    clocks = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    clocks.start()
+    time.sleep(0.3)
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for i in range(args.steps):
+        step(i)
+    t1.record(stream)
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms_total = t0.elapsed_time(t1)
+    kern_ms = sum(a.elapsed_time(b) for a, b in zip(k0, k1)) / args.steps
+    ctx.sync()
+
+    # ---- end-to-end through the public API with host buffers ----
+    e2e = None
+    if not args.no_e2e:
+        R_host = torch.empty((NN, 2), dtype=torch.float64).pin_memory()
+        for _ in range(2):
+            U.copy_(U_host, non_blocking=True)
+            step()
+            R_host.copy_(R, non_blocking=True)
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for i in range(args.steps):
+            U.copy_(U_host, non_blocking=True)
+            step()
+            R_host.copy_(R, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        e2e_ms = e0.elapsed_time(e1) / args.steps
+        e2e = [e2e_ms, U_host.numel() * 8, R_host.numel() * 8]
+
+    # ---- reduce over ranks (max time) ----
+    stats = torch.tensor([ms_total / args.steps, kern_ms, e2e[0] if e2e else 0.0], dtype=torch.float64, device=dev)
+    cells_all = torch.tensor([float(C)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(stats, op=dist.ReduceOp.MAX)
+        dist.all_reduce(cells_all, op=dist.ReduceOp.SUM)
+    ms_step, kern_ms_max, e2e_ms = stats.tolist()
+    total_cells = int(cells_all.item())
+
+    if rank == 0:
+        peak, peak_src = load_peaks()
+        bpl = bytes_per_launch(elem, C, NN)
+        achieved = bpl / (kern_ms_max * 1e-3) / 1e9
+        traffic = None
+        tpath = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tpath):
+            with open(tpath) as f:
+                tr = json.load(f)
+            key = f"{args.config}:{elem}:jacobian"
+            if key in tr and world == 1:
+                traffic = tr[key]["dram_bytes_per_launch"]
+        line = {
+            "metric": METRIC,
+            "value": total_cells / (ms_step * 1e-3),
+            "unit": "cells/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": ms_step,
+            "higher_is_better": True,
+            "scaling": "strong",
+            "vs_baseline": None,
+            "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": WORKLOADS[args.config], "cells": total_cells, "elem": elem, "layers": L,
+                       "cells_rank0": C, "nodes_rank0": NN, "parallelism": f"column-partition x{world}",
+                       "l2": "inputs exceed L2 (no flush needed)",
+                       "launch": ctx.launch_info()},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "eval_kernel<Hex8,true> (stokesfo_jacobian)" if elem == "hex8"
+                         else "eval_kernel<Wedge6,true> (stokesfo_jacobian)",
+                         "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src},
+            "achieved_hbm_gbs": achieved,
+            "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),
+            "clocks": clk,
+        }
+        if e2e:
+            line["e2e"] = {"value": total_cells / (e2e_ms * 1e-3), "unit": "cells/s",
+                           "h2d_bytes_per_step": e2e[1], "d2h_bytes_per_step": e2e[2],
+                           "note": "pinned U H2D + stokesfo_jacobian + R D2H per step; J_cell stays on device"}
+        if world == 1 and not args.no_cpu_baseline:
+            import oracle as O
+            rate, n, dt = oracle_sample_rate(elem, conn_g, coords_g, U_g, s_g, kc_g, target_s=12.0)
+            line["cpu_baseline"] = {"value": rate, "unit": "cells/s", "cores": O.num_threads(), "kind": "oracle",
+                                    "sample": f"first {n} cells of {args.config} (residual+AD Jacobian, "
+                                              f"geometry precomputed untimed), {dt:.1f} s"}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,187 @@
+/*
+ * stokesfo.h -- C ABI of libstokesfo.so: the B200 (sm_100a) Stokes-FO
+ * (Blatter-Pattyn) per-cell residual + forward-AD Jacobian evaluator.
+ *
+ * The problem the ABI follows is PAPER.md eq. (3):
+ *     F(U; {phi_i}, {grad phi_i}, H, ...) = 0,
+ * the finite-element discretisation of the first-order Stokes equations
+ * eq. (1) on a mesh extruded from a 2-D footprint,
+ * with the per-cell evaluation of Fig. 2 (StokesFOResid, optimized
+ * loop order) and its AD Jacobian (Sacado SFad, 16 derivative
+ * components per hex8 cell = 8 nodes x 2 velocity components).
+ *
+ * Conventions (all readings listed in DESIGN.md):
+ *   - dof = 2*node + comp (interleaved); local derivative index k = 2*n + a (Z9)
+ *   - hex8: Shards node order, 2x2x2 Gauss, q = i + 2j + 4k (Z8, Z9)
+ *   - wedge6: bottom triangle (0,0),(1,0),(0,1) then top; 3-point interior
+ *     triangle rule x 2-point Gauss, q = t + 3k (Z8)
+ *   - Glen's law (Z1-Z3): eps_e^2 = ux^2 + vy^2 + ux vy + 1/4 (uy+vx)^2
+ *     + 1/4 uz^2 + 1/4 vz^2;  mu = k_c (eps_e^2 + delta)^((1-n)/(2n)); n = 3.
+ *   - stresses exactly as Fig. 2; body force f = rho_g grad s_h
+ *     with sign + (eq. (1); Z6), or a caller-given force_qp.
+ *   - residual (Fig. 2):
+ *       R[n][a] = sum_q wM_q (sum_d sigma_(a,d) GradBF[n][q][d] + f_a BF[n][q])
+ *   - Jacobian J[(i,a),(j,b)] = dR_cell[i][a] / dU_cell[j][b] including
+ *     d mu / dU (full Newton, Z5); row-major [2N][2N], row = 2i+a, col = 2j+b.
+ *
+ * Memory and ownership:
+ *   - The caller owns ALL device memory (e.g. torch tensors via data_ptr()),
+ *     including the workspace.  The library never calls cudaMalloc.
+ *   - The ctx is a host object freed by stokesfo_destroy.  desc arrays (conn,
+ *     coords, surface, force_qp, flow_factor) must stay valid and unchanged
+ *     while the ctx lives (stokesfo_create snapshots geometry, conn and the
+ *     flow factor into the workspace; surface and force_qp are re-read at
+ *     every evaluation).
+ *   - Every device pointer must be 16-byte aligned (workspace: 256-byte),
+ *     otherwise EINVAL.
+ *
+ * Errors and execution:
+ *   - Functions return stokesfo_status_t codes; no exception crosses the ABI.
+ *   - Every call is asynchronous on desc.stream.  Device-side errors (det J <= 0,
+ *     conn out of range, CSR entry missing) set a sticky flag in the workspace
+ *     that stokesfo_sync reports as STOKESFO_EMESH.
+ *   - glen_n != 3 returns STOKESFO_EUNSUPPORTED (the CPU oracle supports any n).
+ *   - Element outputs (mu_qp, R_cell, J_cell, U_cell) are overwritten; global
+ *     outputs (R, csr_vals) are accumulated (+=): the caller zeroes them.
+ *   - A ctx is not thread-safe; distinct ctxs are independent.
+ */
+#ifndef STOKESFO_H
+#define STOKESFO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define STOKESFO_ABI_VERSION 1
+
+typedef struct stokesfo_ctx stokesfo_ctx; /* opaque host object */
+
+typedef enum { STOKESFO_HEX8 = 0, STOKESFO_WEDGE6 = 1 } stokesfo_elem_t;
+
+typedef enum {
+    STOKESFO_OK = 0,
+    STOKESFO_EINVAL = 1,       /* bad argument, size or alignment */
+    STOKESFO_EMESH = 2,        /* det J <= 0, conn out of range, CSR entry missing */
+    STOKESFO_ECUDA = 3,        /* a CUDA runtime error */
+    STOKESFO_ENOMEM = 4,       /* workspace too small */
+    STOKESFO_EUNSUPPORTED = 5  /* e.g. glen_n != 3 */
+} stokesfo_status_t;
+
+typedef struct {
+    uint32_t abi_version;        /* = STOKESFO_ABI_VERSION */
+    int32_t elem;                /* stokesfo_elem_t */
+    int64_t num_cells;           /* C, local to this device (may be 0) */
+    int64_t num_nodes;           /* local to this device */
+    const int32_t *conn;         /* dev [C][N] local node ids, N = 8 (hex8) / 6 (wedge6) */
+    const double *coords;        /* dev [num_nodes][3] (x, y, z) */
+    const double *surface;       /* dev [num_nodes] surface height s, or NULL */
+    const double *force_qp;      /* dev [C][Q][2] body force at QPs, or NULL; overrides surface */
+    const double *flow_factor;   /* dev [C] k_c = A_c^(-1/n)/2, or NULL (then scalar k) */
+    double k;                    /* Glen prefactor used when flow_factor == NULL */
+    double glen_n;               /* Glen exponent; must be 3 */
+    double delta;                /* regularisation of eps_e^2 (Z3), > 0 */
+    double rho_g;                /* rho * g multiplying grad s_h */
+    void *workspace;             /* dev, caller-owned, >= stokesfo_workspace_size() bytes */
+    size_t workspace_bytes;
+    void *stream;                /* cudaStream_t used by every call (NULL = legacy default) */
+} stokesfo_desc_t;
+
+/* Bytes of workspace needed for desc (only elem and num_cells are read). */
+int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes);
+
+/* Validate desc and run the basis/quadrature precompute:
+ * GradBF[c][n][q][:] = J_q^-T grad_xi phi_n(xi_q), wMeasure[c][q] = w_q det J_q
+ * into the workspace, plus a snapshot of conn and the flow factor.  Async on
+ * desc.stream; det J <= 0 or conn out of range is reported by stokesfo_sync. */
+int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out);
+
+/* Gather: U_cell[c][n][a] = U[2 conn[c][n] + a].
+ * U: dev [num_nodes][2]; U_cell: dev [C][N][2] (overwritten). */
+int stokesfo_gather(stokesfo_ctx *c, const double *U, double *U_cell);
+
+/* Residual evaluation, fused gather -> Ugrad -> mu -> stress -> QP sum ->
+ * scatter (Fig. 2).  U: dev [num_nodes][2].  Optional
+ * outputs (NULL to skip): mu_qp [C][Q] (overwritten), R_cell [C][N][2]
+ * (overwritten), R [num_nodes][2] (+=). */
+int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell,
+                             double *R);
+
+/* Residual + forward-AD Jacobian in one pass.
+ * J_cell: dev [C][2N][2N] row-major (required, overwritten); R_cell, R optional
+ * as above. */
+int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *R_cell, double *R);
+
+/* Assembly: R[2 conn[c][n] + a] += R_cell[c][n][a] (if R_cell and R are non-NULL)
+ * and csr_vals[pos(row, col)] += J_cell[c][k][l] (if J_cell and csr_vals are
+ * non-NULL; requires an earlier stokesfo_csr_pattern call with non-NULL rowptr
+ * and colidx, which must stay valid). */
+int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R,
+                              const double *J_cell, double *csr_vals);
+
+/* CSR pattern over dofs (rows = 2*num_nodes; columns of a row = sorted dofs of
+ * every node sharing a cell with the row's node).  Size query: pass rowptr =
+ * colidx = NULL to get *nnz.  Fill: rowptr dev [2*num_nodes+1] int64, colidx
+ * dev [nnz] int32.  Synchronises the stream (host-side construction). */
+int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t *colidx);
+
+/* Export the precomputed geometry in the canonical layout:
+ * grad_bf dev [C][N][Q][3], w_measure dev [C][Q] (either may be NULL). */
+int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure);
+
+/* Multi-GPU halo sum.  pack: buf[k][a] = R[2 send_nodes[k] + a];
+ * unpack_add: R[2 recv_nodes[k] + a] += buf[k][a].  Node lists are local ids,
+ * unique within a list; buf is dev [n][2]. */
+int stokesfo_halo_pack(stokesfo_ctx *c, const double *R, const int32_t *send_nodes, int64_t n,
+                       double *buf);
+int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *recv_nodes,
+                             int64_t n, double *R);
+
+/* Synchronise the ctx stream; returns ECUDA on a CUDA error, else EMESH if a
+ * device-side error flag was raised since create, else OK. */
+int stokesfo_sync(stokesfo_ctx *c);
+
+/* Static string for a status code. */
+const char *stokesfo_strerror(int status);
+
+void stokesfo_destroy(stokesfo_ctx *c);
+
+/* Launch/tiling facts for measurement (kernels launched per evaluation call,
+ * cells per tile, grid size).  Any pointer may be NULL. */
+int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid_resid,
+                         int32_t *grid_jac, int64_t *record_bytes_per_tile);
+
+/* ---------------- host-side mesh construction (no GPU needed) ------------- */
+
+/* Extrude a footprint by L uniform-sigma layers:
+ *   node(v,k) = v*(L+1)+k (k = 0 bed .. L surface); cell(f,k) = f*L+k;
+ *   conn[cell] = [poly verts at level k, same at level k+1];
+ *   coords[node] = (x_v, y_v, b_v + H_v * (k/L)).
+ * Host arrays: xy [nv][2], polys [nf][npoly] (npoly = 4 -> hex8, 3 -> wedge6),
+ * b, H [nv]; outputs conn [nf*L][2*npoly], coords [nv*(L+1)][3]. */
+int stokesfo_mesh_extrude(int32_t npoly, int64_t nv, const double *xy, int64_t nf,
+                          const int32_t *polys, const double *b, const double *H, int32_t L,
+                          int32_t *conn, double *coords);
+
+/* Column partition into nparts contiguous equal-count ranges:
+ * part r owns columns [ranges[r], ranges[r+1]), ranges[r] = floor(r*nf/nparts). */
+int stokesfo_mesh_partition_columns(int64_t nf, int32_t nparts, int64_t *ranges);
+
+/* Localise the cells of one part: local node ids are the ranks of the touched
+ * global ids in ascending order.  conn_global: host [ncells][npc].  Size query
+ * with gids == NULL (sets *num_local_nodes); fill gids [num_local_nodes] and
+ * conn_local [ncells][npc]. */
+int stokesfo_mesh_localize(int32_t npc, int64_t ncells, const int32_t *conn_global,
+                           int64_t *num_local_nodes, int64_t *gids, int32_t *conn_local);
+
+/* Halo list of "mine" w.r.t. "other": local ids (in mine) of the global ids the
+ * two sorted lists share, ordered by global id.  Size query with idx == NULL. */
+int stokesfo_mesh_halo_list(int64_t n_mine, const int64_t *gids_mine, int64_t n_other,
+                            const int64_t *gids_other, int64_t *n_shared, int32_t *idx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STOKESFO_H */

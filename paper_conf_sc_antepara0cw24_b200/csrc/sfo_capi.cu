@@ -1,0 +1,340 @@
+// sfo_capi.cu -- extern "C" entry points of libstokesfo.so (include/stokesfo.h).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "../../include/stokesfo.h"
+#include "sfo_kernels.cuh"
+
+using namespace sfo;
+
+struct stokesfo_ctx {
+    stokesfo_desc_t d;
+    cudaStream_t stream;
+    int N, Q, TC;
+    int64_t ntiles;
+    int *err;              // device flag in the workspace header
+    char *recs;            // device records
+    int grid_resid, grid_jac;
+    int rec_bytes;
+    const int64_t *rowptr = nullptr;  // CSR pattern (set by stokesfo_csr_pattern)
+    const int32_t *colidx = nullptr;
+    int64_t csr_rows = 0;
+};
+
+namespace {
+
+bool aligned(const void *p, size_t a) { return (reinterpret_cast<uintptr_t>(p) % a) == 0; }
+
+int cuda_status() {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        fprintf(stderr, "libstokesfo: CUDA error %s\n", cudaGetErrorString(e));
+        return STOKESFO_ECUDA;
+    }
+    return STOKESFO_OK;
+}
+
+template <class E>
+int64_t ws_bytes(int64_t ncells) {
+    const int64_t ntiles = (ncells + E::TC - 1) / E::TC;
+    return WS_HEADER + ntiles * (int64_t)Rec<E>::BYTES;
+}
+
+template <class E, bool JAC>
+int configure_eval(int *grid) {
+    using S = EvalSmem<E, JAC>;
+    auto fn = eval_kernel<E, JAC>;
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES) != cudaSuccess)
+        return cuda_status();
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, E::TC * E::N, S::BYTES) != cudaSuccess)
+        return cuda_status();
+    *grid = std::max(1, sms * std::max(1, per_sm));
+    return STOKESFO_OK;
+}
+
+template <class E>
+int create_impl(stokesfo_ctx *c) {
+    c->N = E::N;
+    c->Q = E::Q;
+    c->TC = E::TC;
+    c->rec_bytes = Rec<E>::BYTES;
+    c->ntiles = (c->d.num_cells + E::TC - 1) / E::TC;
+    int st = configure_eval<E, false>(&c->grid_resid);
+    if (st) return st;
+    st = configure_eval<E, true>(&c->grid_jac);
+    if (st) return st;
+    if (cudaMemsetAsync(c->err, 0, sizeof(int), c->stream) != cudaSuccess) return cuda_status();
+    if (c->ntiles > 0) {
+        const int64_t work = c->ntiles * E::TC * E::Q;
+        const int bs = 256;
+        geometry_kernel<E><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
+            c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.coords, c->d.flow_factor, c->d.k, c->recs, c->err);
+    }
+    return cuda_status();
+}
+
+template <class E, bool JAC>
+int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R, double *J_cell) {
+    if (c->ntiles == 0) return STOKESFO_OK;
+    EvalArgs a;
+    a.recs = c->recs;
+    a.ntiles = c->ntiles;
+    a.ncells = c->d.num_cells;
+    a.U = U;
+    a.surface = c->d.surface;
+    a.force_qp = c->d.force_qp;
+    a.rho_g = c->d.rho_g;
+    a.delta = c->d.delta;
+    a.mu_qp = mu_qp;
+    a.R_cell = R_cell;
+    a.R = R;
+    a.J_cell = J_cell;
+    const int grid = (int)std::min<int64_t>(JAC ? c->grid_jac : c->grid_resid, c->ntiles);
+    eval_kernel<E, JAC><<<grid, E::TC * E::N, EvalSmem<E, JAC>::BYTES, c->stream>>>(a);
+    return cuda_status();
+}
+
+#define DISPATCH(ctx, CALL)                                   \
+    ((ctx)->d.elem == STOKESFO_HEX8 ? CALL(Hex8) : CALL(Wedge6))
+
+}  // namespace
+
+extern "C" {
+
+const char *stokesfo_strerror(int s) {
+    switch (s) {
+        case STOKESFO_OK: return "ok";
+        case STOKESFO_EINVAL: return "invalid argument (size, pointer or alignment)";
+        case STOKESFO_EMESH: return "mesh error (det J <= 0, conn out of range or CSR entry missing)";
+        case STOKESFO_ECUDA: return "CUDA runtime error";
+        case STOKESFO_ENOMEM: return "workspace too small";
+        case STOKESFO_EUNSUPPORTED: return "unsupported configuration (glen_n must be 3)";
+        default: return "unknown status";
+    }
+}
+
+int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes) {
+    if (!d || !bytes || d->num_cells < 0) return STOKESFO_EINVAL;
+    if (d->elem == STOKESFO_HEX8) *bytes = (size_t)ws_bytes<Hex8>(d->num_cells);
+    else if (d->elem == STOKESFO_WEDGE6) *bytes = (size_t)ws_bytes<Wedge6>(d->num_cells);
+    else return STOKESFO_EINVAL;
+    return STOKESFO_OK;
+}
+
+int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
+    if (!d || !out) return STOKESFO_EINVAL;
+    *out = nullptr;
+    if (d->abi_version != STOKESFO_ABI_VERSION) return STOKESFO_EINVAL;
+    if (d->elem != STOKESFO_HEX8 && d->elem != STOKESFO_WEDGE6) return STOKESFO_EINVAL;
+    if (d->num_cells < 0 || d->num_nodes < 0 || d->num_nodes > INT32_MAX) return STOKESFO_EINVAL;
+    if (d->num_cells > 0 && (!d->conn || !d->coords || d->num_nodes == 0)) return STOKESFO_EINVAL;
+    if (!(d->delta > 0.0)) return STOKESFO_EINVAL;
+    if (d->glen_n != 3.0) return STOKESFO_EUNSUPPORTED;
+    const void *ptrs[] = {d->conn, d->coords, d->surface, d->force_qp, d->flow_factor};
+    for (const void *p : ptrs)
+        if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
+    if (!d->workspace || !aligned(d->workspace, 256)) return STOKESFO_EINVAL;
+    size_t need = 0;
+    stokesfo_workspace_size(d, &need);
+    if (d->workspace_bytes < need) return STOKESFO_ENOMEM;
+    stokesfo_ctx *c = new (std::nothrow) stokesfo_ctx();
+    if (!c) return STOKESFO_ENOMEM;
+    c->d = *d;
+    c->stream = reinterpret_cast<cudaStream_t>(d->stream);
+    c->err = reinterpret_cast<int *>(d->workspace);
+    c->recs = reinterpret_cast<char *>(d->workspace) + WS_HEADER;
+    int st = (d->elem == STOKESFO_HEX8) ? create_impl<Hex8>(c) : create_impl<Wedge6>(c);
+    if (st) {
+        delete c;
+        return st;
+    }
+    *out = c;
+    return STOKESFO_OK;
+}
+
+void stokesfo_destroy(stokesfo_ctx *c) { delete c; }
+
+int stokesfo_gather(stokesfo_ctx *c, const double *U, double *U_cell) {
+    if (!c || !U || !U_cell || !aligned(U, 16) || !aligned(U_cell, 16)) return STOKESFO_EINVAL;
+    const int64_t work = c->d.num_cells * c->N;
+    if (work == 0) return STOKESFO_OK;
+    const int bs = 256;
+    const unsigned g = (unsigned)((work + bs - 1) / bs);
+    auto U2 = reinterpret_cast<const double2 *>(U);
+    auto Uc = reinterpret_cast<double2 *>(U_cell);
+    if (c->N == 8) gather_kernel<8><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.conn, U2, Uc);
+    else gather_kernel<6><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.conn, U2, Uc);
+    return cuda_status();
+}
+
+int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R) {
+    if (!c || !U || !aligned(U, 16)) return STOKESFO_EINVAL;
+    const void *ps[] = {mu_qp, R_cell, R};
+    for (const void *p : ps)
+        if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
+#define CALL(E) eval_impl<E, false>(c, U, mu_qp, R_cell, R, nullptr)
+    return DISPATCH(c, CALL);
+#undef CALL
+}
+
+int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *R_cell, double *R) {
+    if (!c || !U || !J_cell || !aligned(U, 16) || !aligned(J_cell, 16)) return STOKESFO_EINVAL;
+    const void *ps[] = {R_cell, R};
+    for (const void *p : ps)
+        if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
+#define CALL(E) eval_impl<E, true>(c, U, nullptr, R_cell, R, J_cell)
+    return DISPATCH(c, CALL);
+#undef CALL
+}
+
+int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, const double *J_cell,
+                              double *csr_vals) {
+    if (!c) return STOKESFO_EINVAL;
+    const void *ps[] = {R_cell, R, J_cell, csr_vals};
+    for (const void *p : ps)
+        if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
+    const int64_t C = c->d.num_cells;
+    const int bs = 256;
+    if (R_cell && R && C > 0) {
+        const int64_t work = C * c->N;
+        const unsigned g = (unsigned)((work + bs - 1) / bs);
+        auto Rc = reinterpret_cast<const double2 *>(R_cell);
+        if (c->N == 8) scatter_r_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, Rc, R);
+        else scatter_r_kernel<6><<<g, bs, 0, c->stream>>>(C, c->d.conn, Rc, R);
+    }
+    if (J_cell && csr_vals && C > 0) {
+        if (!c->rowptr || !c->colidx) return STOKESFO_EINVAL;
+        const int64_t work = C * 2 * c->N;
+        const unsigned g = (unsigned)((work + bs - 1) / bs);
+        if (c->N == 8)
+            scatter_csr_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->colidx, csr_vals, c->err);
+        else
+            scatter_csr_kernel<6><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->colidx, csr_vals, c->err);
+    }
+    return cuda_status();
+}
+
+int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure) {
+    if (!c) return STOKESFO_EINVAL;
+    if ((grad_bf && !aligned(grad_bf, 16)) || (w_measure && !aligned(w_measure, 16))) return STOKESFO_EINVAL;
+    const int64_t work = c->d.num_cells * c->Q;
+    if (work == 0) return STOKESFO_OK;
+    const int bs = 256;
+    const unsigned g = (unsigned)((work + bs - 1) / bs);
+    if (c->N == 8) geometry_export_kernel<Hex8><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
+    else geometry_export_kernel<Wedge6><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
+    return cuda_status();
+}
+
+int stokesfo_halo_pack(stokesfo_ctx *c, const double *R, const int32_t *send_nodes, int64_t n, double *buf) {
+    if (!c || n < 0) return STOKESFO_EINVAL;
+    if (n == 0) return STOKESFO_OK;
+    if (!R || !send_nodes || !buf || !aligned(R, 16) || !aligned(buf, 16)) return STOKESFO_EINVAL;
+    const int bs = 256;
+    halo_pack_kernel<<<(unsigned)((n + bs - 1) / bs), bs, 0, c->stream>>>(
+        n, send_nodes, reinterpret_cast<const double2 *>(R), reinterpret_cast<double2 *>(buf));
+    return cuda_status();
+}
+
+int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *recv_nodes, int64_t n, double *R) {
+    if (!c || n < 0) return STOKESFO_EINVAL;
+    if (n == 0) return STOKESFO_OK;
+    if (!R || !recv_nodes || !buf || !aligned(R, 16) || !aligned(buf, 16)) return STOKESFO_EINVAL;
+    const int bs = 256;
+    halo_unpack_add_kernel<<<(unsigned)((n + bs - 1) / bs), bs, 0, c->stream>>>(
+        n, recv_nodes, reinterpret_cast<const double2 *>(buf), reinterpret_cast<double2 *>(R));
+    return cuda_status();
+}
+
+int stokesfo_sync(stokesfo_ctx *c) {
+    if (!c) return STOKESFO_EINVAL;
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_status();
+    int h = 0;
+    if (cudaMemcpy(&h, c->err, sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess) return cuda_status();
+    return h ? STOKESFO_EMESH : STOKESFO_OK;
+}
+
+int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid_resid, int32_t *grid_jac,
+                         int64_t *record_bytes_per_tile) {
+    if (!c) return STOKESFO_EINVAL;
+    if (cells_per_tile) *cells_per_tile = c->TC;
+    if (grid_resid) *grid_resid = (int32_t)std::min<int64_t>(c->grid_resid, std::max<int64_t>(c->ntiles, 1));
+    if (grid_jac) *grid_jac = (int32_t)std::min<int64_t>(c->grid_jac, std::max<int64_t>(c->ntiles, 1));
+    if (record_bytes_per_tile) *record_bytes_per_tile = c->rec_bytes;
+    return STOKESFO_OK;
+}
+
+// CSR pattern: host-side construction from a device->host copy of conn.
+int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t *colidx) {
+    if (!c || !nnz) return STOKESFO_EINVAL;
+    const int64_t C = c->d.num_cells, NN = c->d.num_nodes;
+    const int N = c->N;
+    std::vector<int32_t> conn((size_t)(C * N));
+    if (C > 0 &&
+        cudaMemcpyAsync(conn.data(), c->d.conn, conn.size() * 4, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess)
+        return cuda_status();
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_status();
+    // node -> cells (CSR)
+    std::vector<int64_t> nc(NN + 1, 0);
+    for (int64_t i = 0; i < C * N; ++i) nc[conn[i] + 1]++;
+    for (int64_t v = 0; v < NN; ++v) nc[v + 1] += nc[v];
+    std::vector<int32_t> ncell(C * N);
+    {
+        std::vector<int64_t> pos(nc.begin(), nc.end() - 1);
+        for (int64_t i = 0; i < C * N; ++i) ncell[pos[conn[i]]++] = (int32_t)(i / N);
+    }
+    // node -> sorted unique neighbour nodes
+    std::vector<int64_t> rp(2 * NN + 1, 0);
+    std::vector<int32_t> nb;
+    std::vector<int32_t> all;
+    std::vector<int64_t> nstart(NN + 1, 0);
+    for (int64_t v = 0; v < NN; ++v) {
+        nb.clear();
+        for (int64_t k = nc[v]; k < nc[v + 1]; ++k) {
+            const int64_t cell = ncell[k];
+            for (int n = 0; n < N; ++n) nb.push_back(conn[cell * N + n]);
+        }
+        std::sort(nb.begin(), nb.end());
+        nb.erase(std::unique(nb.begin(), nb.end()), nb.end());
+        all.insert(all.end(), nb.begin(), nb.end());
+        nstart[v + 1] = (int64_t)all.size();
+    }
+    for (int64_t v = 0; v < NN; ++v) {
+        const int64_t deg = 2 * (nstart[v + 1] - nstart[v]);
+        rp[2 * v + 1] = rp[2 * v] + deg;
+        rp[2 * v + 2] = rp[2 * v + 1] + deg;
+    }
+    *nnz = rp[2 * NN];
+    if (!rowptr || !colidx) return STOKESFO_OK;
+    if (!aligned(rowptr, 8) || !aligned(colidx, 4)) return STOKESFO_EINVAL;
+    std::vector<int32_t> ci((size_t)*nnz);
+    for (int64_t v = 0; v < NN; ++v)
+        for (int a = 0; a < 2; ++a) {
+            int64_t o = rp[2 * v + a];
+            for (int64_t k = nstart[v]; k < nstart[v + 1]; ++k) {
+                ci[o++] = 2 * all[k];
+                ci[o++] = 2 * all[k] + 1;
+            }
+        }
+    if (cudaMemcpyAsync(rowptr, rp.data(), rp.size() * 8, cudaMemcpyHostToDevice, c->stream) != cudaSuccess)
+        return cuda_status();
+    if (!ci.empty() &&
+        cudaMemcpyAsync(colidx, ci.data(), ci.size() * 4, cudaMemcpyHostToDevice, c->stream) != cudaSuccess)
+        return cuda_status();
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_status();
+    c->rowptr = rowptr;
+    c->colidx = colidx;
+    c->csr_rows = 2 * NN;
+    return STOKESFO_OK;
+}
+
+}  // extern "C"

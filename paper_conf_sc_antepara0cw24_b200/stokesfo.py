@@ -1,0 +1,284 @@
+"""Thin ctypes binding of libstokesfo.so (include/stokesfo.h).
+
+Argument marshalling only: every step of the evaluation runs in the library's
+CUDA kernels.  PyTorch supplies device memory (tensors -> data_ptr()) and the
+stream; nothing here computes the method.  There is no CPU fallback: if the
+library cannot be loaded, every call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from . import build as _build
+
+HEX8, WEDGE6 = 0, 1
+ELEM = {"hex8": HEX8, "wedge6": WEDGE6}
+NODES = {HEX8: 8, WEDGE6: 6}
+QPS = {HEX8: 8, WEDGE6: 6}
+ABI_VERSION = 1
+
+STATUS = {0: "OK", 1: "EINVAL", 2: "EMESH", 3: "ECUDA", 4: "ENOMEM", 5: "EUNSUPPORTED"}
+
+
+class StokesFOError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        msg = _lib().stokesfo_strerror(status).decode() if _LIB is not None else STATUS.get(status, "?")
+        super().__init__(f"{where}: {STATUS.get(status, status)} ({msg})")
+
+
+class Desc(ctypes.Structure):
+    _fields_ = [
+        ("abi_version", ctypes.c_uint32), ("elem", ctypes.c_int32),
+        ("num_cells", ctypes.c_int64), ("num_nodes", ctypes.c_int64),
+        ("conn", ctypes.c_void_p), ("coords", ctypes.c_void_p), ("surface", ctypes.c_void_p),
+        ("force_qp", ctypes.c_void_p), ("flow_factor", ctypes.c_void_p),
+        ("k", ctypes.c_double), ("glen_n", ctypes.c_double), ("delta", ctypes.c_double),
+        ("rho_g", ctypes.c_double),
+        ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_size_t),
+        ("stream", ctypes.c_void_p),
+    ]
+
+
+_LIB = None
+EXPORTS = [
+    "stokesfo_workspace_size", "stokesfo_create", "stokesfo_gather", "stokesfo_viscosity_resid",
+    "stokesfo_jacobian", "stokesfo_scatter_assemble", "stokesfo_csr_pattern", "stokesfo_geometry",
+    "stokesfo_halo_pack", "stokesfo_halo_unpack_add", "stokesfo_sync", "stokesfo_strerror",
+    "stokesfo_destroy", "stokesfo_launch_info", "stokesfo_mesh_extrude",
+    "stokesfo_mesh_partition_columns", "stokesfo_mesh_localize", "stokesfo_mesh_halo_list",
+]
+
+
+def lib_path() -> str:
+    return _build.LIB
+
+
+def _lib():
+    """Load libstokesfo.so (building it in-tree with nvcc if absent)."""
+    global _LIB
+    if _LIB is None:
+        path = _build.LIB
+        if not os.path.exists(path):
+            _build.build()
+        L = ctypes.CDLL(path)
+        P, I64, I32, D = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_double
+        L.stokesfo_workspace_size.argtypes = [ctypes.POINTER(Desc), ctypes.POINTER(ctypes.c_size_t)]
+        L.stokesfo_create.argtypes = [ctypes.POINTER(Desc), ctypes.POINTER(ctypes.c_void_p)]
+        L.stokesfo_gather.argtypes = [P, P, P]
+        L.stokesfo_viscosity_resid.argtypes = [P, P, P, P, P]
+        L.stokesfo_jacobian.argtypes = [P, P, P, P, P]
+        L.stokesfo_scatter_assemble.argtypes = [P, P, P, P, P]
+        L.stokesfo_csr_pattern.argtypes = [P, ctypes.POINTER(I64), P, P]
+        L.stokesfo_geometry.argtypes = [P, P, P]
+        L.stokesfo_halo_pack.argtypes = [P, P, P, I64, P]
+        L.stokesfo_halo_unpack_add.argtypes = [P, P, P, I64, P]
+        L.stokesfo_sync.argtypes = [P]
+        L.stokesfo_strerror.argtypes = [ctypes.c_int]
+        L.stokesfo_strerror.restype = ctypes.c_char_p
+        L.stokesfo_destroy.argtypes = [P]
+        L.stokesfo_destroy.restype = None
+        L.stokesfo_launch_info.argtypes = [P, ctypes.POINTER(I32), ctypes.POINTER(I32), ctypes.POINTER(I32),
+                                           ctypes.POINTER(I64)]
+        L.stokesfo_mesh_extrude.argtypes = [I32, I64, P, I64, P, P, P, I32, P, P]
+        L.stokesfo_mesh_partition_columns.argtypes = [I64, I32, P]
+        L.stokesfo_mesh_localize.argtypes = [I32, I64, P, ctypes.POINTER(I64), P, P]
+        L.stokesfo_mesh_halo_list.argtypes = [I64, P, I64, P, ctypes.POINTER(I64), P]
+        _LIB = L
+    return _LIB
+
+
+def _check(st: int, where: str):
+    if st != 0:
+        raise StokesFOError(st, where)
+
+
+def _ptr(t):
+    """Device (or host numpy) pointer of a tensor/array, or None."""
+    if t is None:
+        return None
+    if isinstance(t, np.ndarray):
+        return t.ctypes.data_as(ctypes.c_void_p)
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _dev(t, dtype, shape=None, name="array"):
+    import torch
+    if t is None:
+        return None
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    if shape is not None and tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name} must have shape {tuple(shape)}, got {tuple(t.shape)}")
+    return t
+
+
+class StokesFO:
+    """One evaluation context (stokesfo_ctx) over a local mesh on one GPU."""
+
+    def __init__(self, elem, conn, coords, surface=None, force_qp=None, flow_factor=None, k=10.77,
+                 glen_n=3.0, delta=1e-10, rho_g=8.927, stream=None):
+        import torch
+        self.elem = ELEM[elem] if isinstance(elem, str) else int(elem)
+        self.N, self.Q = NODES[self.elem], QPS[self.elem]
+        C = int(conn.shape[0])
+        nn = int(coords.shape[0])
+        self.num_cells, self.num_nodes = C, nn
+        self.conn = _dev(conn, torch.int32, (C, self.N), "conn")
+        self.coords = _dev(coords, torch.float64, (nn, 3), "coords")
+        self.surface = _dev(surface, torch.float64, (nn,), "surface")
+        self.force_qp = _dev(force_qp, torch.float64, (C, self.Q, 2), "force_qp")
+        self.flow_factor = _dev(flow_factor, torch.float64, (C,), "flow_factor")
+        self.device = self.coords.device
+        self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+        d = Desc()
+        d.abi_version = ABI_VERSION
+        d.elem = self.elem
+        d.num_cells, d.num_nodes = C, nn
+        d.conn, d.coords = _ptr(self.conn), _ptr(self.coords)
+        d.surface, d.force_qp, d.flow_factor = _ptr(self.surface), _ptr(self.force_qp), _ptr(self.flow_factor)
+        d.k, d.glen_n, d.delta, d.rho_g = k, glen_n, delta, rho_g
+        d.stream = ctypes.c_void_p(self.stream.cuda_stream)
+        nbytes = ctypes.c_size_t(0)
+        _check(_lib().stokesfo_workspace_size(ctypes.byref(d), ctypes.byref(nbytes)), "workspace_size")
+        self.workspace = torch.empty(max(int(nbytes.value), 256), dtype=torch.uint8, device=self.device)
+        d.workspace, d.workspace_bytes = _ptr(self.workspace), self.workspace.numel()
+        self._desc = d
+        h = ctypes.c_void_p()
+        _check(_lib().stokesfo_create(ctypes.byref(d), ctypes.byref(h)), "create")
+        self._h = h
+        self.rowptr = None
+        self.colidx = None
+
+    # -- lifetime -------------------------------------------------------------
+    def destroy(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            _lib().stokesfo_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+    # -- calls (same names as the C ABI) --------------------------------------
+    def gather(self, U, U_cell=None):
+        import torch
+        _dev(U, torch.float64, (self.num_nodes, 2), "U")
+        if U_cell is None:
+            U_cell = torch.empty((self.num_cells, self.N, 2), dtype=torch.float64, device=self.device)
+        _check(_lib().stokesfo_gather(self._h, _ptr(U), _ptr(U_cell)), "gather")
+        return U_cell
+
+    def viscosity_resid(self, U, mu_qp=None, R_cell=None, R=None):
+        import torch
+        _dev(U, torch.float64, (self.num_nodes, 2), "U")
+        _dev(mu_qp, torch.float64, (self.num_cells, self.Q), "mu_qp")
+        _dev(R_cell, torch.float64, (self.num_cells, self.N, 2), "R_cell")
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_viscosity_resid(self._h, _ptr(U), _ptr(mu_qp), _ptr(R_cell), _ptr(R)),
+               "viscosity_resid")
+
+    def jacobian(self, U, J_cell, R_cell=None, R=None):
+        import torch
+        _dev(U, torch.float64, (self.num_nodes, 2), "U")
+        _dev(J_cell, torch.float64, (self.num_cells, 2 * self.N, 2 * self.N), "J_cell")
+        _dev(R_cell, torch.float64, (self.num_cells, self.N, 2), "R_cell")
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_jacobian(self._h, _ptr(U), _ptr(J_cell), _ptr(R_cell), _ptr(R)), "jacobian")
+
+    def csr_pattern(self):
+        import torch
+        nnz = ctypes.c_int64(0)
+        _check(_lib().stokesfo_csr_pattern(self._h, ctypes.byref(nnz), None, None), "csr_pattern(size)")
+        self.rowptr = torch.empty(2 * self.num_nodes + 1, dtype=torch.int64, device=self.device)
+        self.colidx = torch.empty(max(int(nnz.value), 1), dtype=torch.int32, device=self.device)
+        _check(_lib().stokesfo_csr_pattern(self._h, ctypes.byref(nnz), _ptr(self.rowptr), _ptr(self.colidx)),
+               "csr_pattern")
+        self.colidx = self.colidx[:int(nnz.value)]
+        return self.rowptr, self.colidx
+
+    def scatter_assemble(self, R_cell=None, R=None, J_cell=None, csr_vals=None):
+        _check(_lib().stokesfo_scatter_assemble(self._h, _ptr(R_cell), _ptr(R), _ptr(J_cell), _ptr(csr_vals)),
+               "scatter_assemble")
+
+    def geometry(self):
+        import torch
+        G = torch.empty((self.num_cells, self.N, self.Q, 3), dtype=torch.float64, device=self.device)
+        wm = torch.empty((self.num_cells, self.Q), dtype=torch.float64, device=self.device)
+        _check(_lib().stokesfo_geometry(self._h, _ptr(G), _ptr(wm)), "geometry")
+        return G, wm
+
+    def halo_pack(self, R, send_nodes, buf):
+        _check(_lib().stokesfo_halo_pack(self._h, _ptr(R), _ptr(send_nodes), int(send_nodes.numel()), _ptr(buf)),
+               "halo_pack")
+
+    def halo_unpack_add(self, buf, recv_nodes, R):
+        _check(_lib().stokesfo_halo_unpack_add(self._h, _ptr(buf), _ptr(recv_nodes), int(recv_nodes.numel()),
+                                               _ptr(R)), "halo_unpack_add")
+
+    def sync(self):
+        _check(_lib().stokesfo_sync(self._h), "sync")
+
+    def launch_info(self):
+        tc, gr, gj = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+        rb = ctypes.c_int64()
+        _check(_lib().stokesfo_launch_info(self._h, ctypes.byref(tc), ctypes.byref(gr), ctypes.byref(gj),
+                                           ctypes.byref(rb)), "launch_info")
+        return {"cells_per_tile": tc.value, "grid_resid": gr.value, "grid_jac": gj.value,
+                "record_bytes_per_tile": rb.value}
+
+
+# ---------------------------------------------------------------------------
+# Host-side mesh construction (numpy in, numpy out)
+# ---------------------------------------------------------------------------
+
+def mesh_extrude(xy, polys, b, H, L: int):
+    xy = np.ascontiguousarray(xy, dtype=np.float64)
+    polys = np.ascontiguousarray(polys, dtype=np.int32)
+    b = np.ascontiguousarray(b, dtype=np.float64)
+    H = np.ascontiguousarray(H, dtype=np.float64)
+    nv, nf, npoly = xy.shape[0], polys.shape[0], polys.shape[1]
+    conn = np.empty((nf * L, 2 * npoly), dtype=np.int32)
+    coords = np.empty((nv * (L + 1), 3), dtype=np.float64)
+    _check(_lib().stokesfo_mesh_extrude(npoly, nv, _ptr(xy), nf, _ptr(polys), _ptr(b), _ptr(H), L,
+                                        _ptr(conn), _ptr(coords)), "mesh_extrude")
+    return conn, coords
+
+
+def mesh_partition_columns(nf: int, nparts: int):
+    r = np.empty(nparts + 1, dtype=np.int64)
+    _check(_lib().stokesfo_mesh_partition_columns(nf, nparts, _ptr(r)), "mesh_partition_columns")
+    return r
+
+
+def mesh_localize(conn_part):
+    conn_part = np.ascontiguousarray(conn_part, dtype=np.int32)
+    nc, npc = conn_part.shape
+    n = ctypes.c_int64(0)
+    _check(_lib().stokesfo_mesh_localize(npc, nc, _ptr(conn_part), ctypes.byref(n), None, None), "mesh_localize")
+    gids = np.empty(n.value, dtype=np.int64)
+    lconn = np.empty_like(conn_part)
+    _check(_lib().stokesfo_mesh_localize(npc, nc, _ptr(conn_part), ctypes.byref(n), _ptr(gids), _ptr(lconn)),
+           "mesh_localize")
+    return lconn, gids
+
+
+def mesh_halo_list(gids_mine, gids_other):
+    gids_mine = np.ascontiguousarray(gids_mine, dtype=np.int64)
+    gids_other = np.ascontiguousarray(gids_other, dtype=np.int64)
+    n = ctypes.c_int64(0)
+    _check(_lib().stokesfo_mesh_halo_list(gids_mine.size, _ptr(gids_mine), gids_other.size, _ptr(gids_other),
+                                          ctypes.byref(n), None), "mesh_halo_list")
+    idx = np.empty(n.value, dtype=np.int32)
+    _check(_lib().stokesfo_mesh_halo_list(gids_mine.size, _ptr(gids_mine), gids_other.size, _ptr(gids_other),
+                                          ctypes.byref(n), _ptr(idx)), "mesh_halo_list")
+    return idx

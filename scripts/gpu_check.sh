@@ -1,0 +1,18 @@
+#!/bin/bash
+# One gpurun pass: GPU tests, smoke, bench, ncu launch list + full capture.
+# Usage (under gpurun): bash scripts/gpu_check.sh [tag] [config]
+TAG=${1:-r01}
+CFG=${2:-C4}
+OUT=gpurun_out
+mkdir -p $OUT
+nvidia-smi -L > $OUT/gpu_$TAG.txt 2>&1
+nvidia-smi --query-gpu=clocks.sm,clocks.max.sm,clocks.mem,power.limit --format=csv >> $OUT/gpu_$TAG.txt 2>&1
+python -c "import __graft_entry__ as g; g.build()" > $OUT/build_$TAG.log 2>&1
+timeout 900 python -m pytest tests -m gpu -x -q -p no:cacheprovider > $OUT/pytest_gpu_$TAG.log 2>&1; echo "pytest exit $?" >> $OUT/pytest_gpu_$TAG.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke_$TAG.log 2>&1; echo "smoke exit $?" >> $OUT/smoke_$TAG.log
+timeout 600 python bench.py --config $CFG --steps 20 --warmup 5 > $OUT/bench_$TAG.json 2> $OUT/bench_$TAG.err; echo "bench exit $?" >> $OUT/bench_$TAG.err
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_$TAG.csv \
+   python bench.py --config $CFG --steps 3 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launch_$TAG.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:eval_kernel -s 3 -c 1 \
+   -o $OUT/prof_$TAG python bench.py --config $CFG --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_full_$TAG.log 2>&1
+echo done

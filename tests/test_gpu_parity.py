@@ -1,0 +1,266 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by
+element on the same seeded inputs.  Tolerances (SURVEY 8(c) 'Tolerances';
+BASELINE.json north_star '1e-12 relative'):
+  element outputs  per cell ||X_gpu - X_orc||_max <= 1e-12 ||X_orc||_max
+  assembled R      per entry |dR| <= 1e-12 sum|contributions|
+  geometry         per (c,q) ||dGradBF|| <= 1e-12 sum_n ||GradBF||
+  gather, integer structures, valence probe: bit-exact."""
+import numpy as np
+import pytest
+
+import oracle as O
+from tests import _meshes as M
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-12
+
+
+@pytest.fixture(scope="module")
+def torch():
+    import torch as _t
+    if not _t.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return _t
+
+
+def _t(torch, a, dtype=None):
+    a = np.ascontiguousarray(a)
+    return torch.from_numpy(a).to("cuda") if dtype is None else torch.from_numpy(a).to("cuda", dtype)
+
+
+def _setup(torch, elem="hex8", n=16, L=5, drop=0, kind="random", scalar_k=False, surface=True):
+    fp, conn, coords = M.tiny(elem, n=n, L=L)
+    if drop:
+        conn = conn[:conn.shape[0] - drop]
+    U, s, kc = M.fields(fp, L, kind=kind)
+    kc = kc[:conn.shape[0]]
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO
+    ctx = StokesFO(elem, _t(torch, conn), _t(torch, coords), surface=_t(torch, s) if surface else None,
+                   flow_factor=None if scalar_k else _t(torch, kc), k=10.77)
+    e = O.ELEM[elem]
+    G, wm, bad = O.geometry(e, conn, coords)
+    assert bad == 0
+    orc = dict(G=G, wm=wm, conn=conn, coords=coords, U=U, s=s if surface else None,
+               kc=None if scalar_k else kc, e=e)
+    return ctx, orc
+
+
+def _cell_rel(a, b):
+    a = a.reshape(a.shape[0], -1)
+    b = b.reshape(b.shape[0], -1)
+    sc = np.maximum(np.abs(b).max(1), 1e-300)
+    return float((np.abs(a - b).max(1) / sc).max())
+
+
+def _assembled_check(R_gpu, orc, R_cell_orc):
+    e = orc["e"]
+    Rref = O.scatter(e, orc["conn"], R_cell_orc, orc["coords"].shape[0])
+    absR = O.scatter(e, orc["conn"], np.abs(R_cell_orc), orc["coords"].shape[0])
+    err = np.abs(R_gpu - Rref)
+    assert (err <= TOL * absR + 1e-300).all(), float((err / np.maximum(absR, 1e-300)).max())
+
+
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_geometry_parity(torch, elem):
+    ctx, orc = _setup(torch, elem)
+    G, wm = ctx.geometry()
+    ctx.sync()
+    G = G.cpu().numpy()
+    wm = wm.cpu().numpy()
+    scale = np.abs(orc["G"]).sum(axis=(1, 3))  # [C][Q]: sum over n, d
+    err = np.abs(G - orc["G"]).max(axis=(1, 3))
+    assert (err <= TOL * scale).all()
+    assert (np.abs(wm - orc["wm"]) <= TOL * np.abs(orc["wm"])).all()
+
+
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_gather_bit_exact(torch, elem):
+    ctx, orc = _setup(torch, elem)
+    Uc = ctx.gather(_t(torch, orc["U"]))
+    ctx.sync()
+    assert np.array_equal(Uc.cpu().numpy(), O.gather(orc["e"], orc["conn"], orc["U"]))
+
+
+@pytest.mark.parametrize("elem,drop,kind", [("hex8", 0, "random"), ("hex8", 5, "balance"),
+                                            ("wedge6", 0, "random"), ("wedge6", 7, "balance")])
+def test_viscosity_resid_parity(torch, elem, drop, kind):
+    ctx, orc = _setup(torch, elem, drop=drop, kind=kind)
+    C, N, Q = ctx.num_cells, ctx.N, ctx.Q
+    mu = torch.empty((C, Q), dtype=torch.float64, device="cuda")
+    Rc = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
+    R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+    ctx.viscosity_resid(_t(torch, orc["U"]), mu_qp=mu, R_cell=Rc, R=R)
+    ctx.sync()
+    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"])
+    assert np.abs(mu.cpu().numpy() / ref["mu_qp"] - 1).max() <= TOL
+    assert _cell_rel(Rc.cpu().numpy(), ref["R_cell"]) <= TOL
+    _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
+
+
+@pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 0), ("wedge6", 11)])
+def test_jacobian_parity(torch, elem, drop):
+    ctx, orc = _setup(torch, elem, drop=drop)
+    C, N = ctx.num_cells, ctx.N
+    J = torch.full((C, 2 * N, 2 * N), float("nan"), dtype=torch.float64, device="cuda")
+    Rc = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
+    R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+    ctx.jacobian(_t(torch, orc["U"]), J, R_cell=Rc, R=R)
+    ctx.sync()
+    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
+                     mode="jac")
+    Jg = J.cpu().numpy()
+    assert np.isfinite(Jg).all()
+    assert _cell_rel(Jg, ref["J_cell"]) <= TOL
+    assert _cell_rel(Rc.cpu().numpy(), ref["R_cell"]) <= TOL
+    _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
+
+
+def test_jacobian_residual_equals_viscosity_resid(torch):
+    ctx, orc = _setup(torch, "hex8")
+    C, N = ctx.num_cells, ctx.N
+    J = torch.empty((C, 16, 16), dtype=torch.float64, device="cuda")
+    R1 = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
+    R2 = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
+    U = _t(torch, orc["U"])
+    ctx.jacobian(U, J, R_cell=R1)
+    ctx.viscosity_resid(U, R_cell=R2)
+    ctx.sync()
+    assert torch.equal(R1, R2)
+
+
+@pytest.mark.parametrize("scalar_k,surface", [(True, True), (False, False), (True, False)])
+def test_optional_inputs(torch, scalar_k, surface):
+    ctx, orc = _setup(torch, "hex8", n=6, L=3, scalar_k=scalar_k, surface=surface)
+    C = ctx.num_cells
+    J = torch.empty((C, 16, 16), dtype=torch.float64, device="cuda")
+    Rc = torch.empty((C, 8, 2), dtype=torch.float64, device="cuda")
+    ctx.jacobian(_t(torch, orc["U"]), J, R_cell=Rc)
+    ctx.sync()
+    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
+                     k=10.77, mode="jac")
+    assert _cell_rel(J.cpu().numpy(), ref["J_cell"]) <= TOL
+    assert _cell_rel(Rc.cpu().numpy(), ref["R_cell"]) <= TOL
+
+
+def test_force_qp_input(torch):
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO
+    fp, conn, coords = M.tiny("hex8", n=6, L=3)
+    U, s, kc = M.fields(fp, 3)
+    f = np.random.default_rng(9).normal(0, 1, (conn.shape[0], 8, 2))
+    ctx = StokesFO("hex8", _t(torch, conn), _t(torch, coords), surface=_t(torch, s), force_qp=_t(torch, f),
+                   flow_factor=_t(torch, kc))
+    Rc = torch.empty((conn.shape[0], 8, 2), dtype=torch.float64, device="cuda")
+    ctx.viscosity_resid(_t(torch, U), R_cell=Rc)
+    ctx.sync()
+    G, wm, _ = O.geometry(0, conn, coords)
+    ref = O.evaluate(0, conn, G, wm, U, force_qp=f, kc=kc)
+    assert _cell_rel(Rc.cpu().numpy(), ref["R_cell"]) <= TOL
+
+
+@pytest.mark.parametrize("name", ["B", "W"])
+def test_golden_cells_gpu(torch, golden, name):
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO
+    g = golden[name]
+    N = 8 if g["elem"] == "hex8" else 6
+    conn = np.arange(N, dtype=np.int32)[None]
+    ctx = StokesFO(g["elem"], _t(torch, conn), _t(torch, np.array(g["coords"], float)),
+                   surface=_t(torch, np.array(g["s"], float)), k=g["k"], delta=g["delta"], rho_g=g["rho_g"])
+    J = torch.empty((1, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
+    Rc = torch.empty((1, N, 2), dtype=torch.float64, device="cuda")
+    mu = torch.empty((1, N), dtype=torch.float64, device="cuda")
+    U = _t(torch, np.array(g["U"], float))
+    ctx.jacobian(U, J, R_cell=Rc)
+    ctx.viscosity_resid(U, mu_qp=mu)
+    ctx.sync()
+    tol = golden["tolerance_gpu"]
+    J = J.cpu().numpy()[0]
+    assert np.abs(mu.cpu().numpy()[0] - g["mu_q"]).max() <= tol * max(g["mu_q"])
+    assert np.abs(Rc.cpu().numpy()[0] - np.array(g["R_cell"])).max() <= tol * np.abs(g["R_cell"]).max()
+    assert np.abs(J[0] - g["J_row0"]).max() <= tol * np.abs(J).max()
+    assert np.abs(np.diag(J) - g["J_diag"]).max() <= tol * np.abs(J).max()
+
+
+def test_valence_probe_bit_exact(torch):
+    ctx, orc = _setup(torch, "hex8")
+    ones = torch.ones((ctx.num_cells, 8, 2), dtype=torch.float64, device="cuda")
+    R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+    ctx.scatter_assemble(R_cell=ones, R=R)
+    ctx.sync()
+    val = np.bincount(orc["conn"].reshape(-1), minlength=ctx.num_nodes).astype(float)
+    Rh = R.cpu().numpy()
+    assert np.array_equal(Rh[:, 0], val) and np.array_equal(Rh[:, 1], val)
+
+
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_csr_pattern_and_assembly(torch, elem):
+    ctx, orc = _setup(torch, elem, n=5, L=3)
+    rowptr, colidx = ctx.csr_pattern()
+    rp2, ci2 = O.csr_pattern(orc["conn"], ctx.num_nodes)
+    assert np.array_equal(rowptr.cpu().numpy(), rp2) and np.array_equal(colidx.cpu().numpy(), ci2)
+    C, N = ctx.num_cells, ctx.N
+    J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
+    ctx.jacobian(_t(torch, orc["U"]), J)
+    vals = torch.zeros(colidx.numel(), dtype=torch.float64, device="cuda")
+    ctx.scatter_assemble(J_cell=J, csr_vals=vals)
+    ctx.sync()
+    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
+                     mode="jac")["J_cell"]
+    v2, miss = O.scatter_csr(orc["e"], orc["conn"], ref, rp2, ci2)
+    a2, _ = O.scatter_csr(orc["e"], orc["conn"], np.abs(ref), rp2, ci2)
+    assert miss == 0
+    assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2 + 1e-300).all()
+
+
+def test_halo_pack_unpack(torch):
+    ctx, orc = _setup(torch, "hex8", n=4, L=2)
+    R = torch.from_numpy(np.random.default_rng(3).normal(size=(ctx.num_nodes, 2))).cuda()
+    nodes = torch.tensor([5, 0, 17, 3], dtype=torch.int32, device="cuda")
+    buf = torch.empty((4, 2), dtype=torch.float64, device="cuda")
+    ctx.halo_pack(R, nodes, buf)
+    R2 = R.clone()
+    ctx.halo_unpack_add(buf, nodes, R2)
+    ctx.sync()
+    assert torch.equal(buf, R[nodes.long()])
+    assert torch.equal(R2[nodes.long()], R[nodes.long()] * 2)
+
+
+def test_edge_cases_and_errors(torch):
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO, StokesFOError
+    fp, conn, coords = M.tiny("hex8", n=2, L=1)
+    # empty mesh: every call is a no-op
+    ctx0 = StokesFO("hex8", _t(torch, conn[:0]), _t(torch, coords))
+    J0 = torch.empty((0, 16, 16), dtype=torch.float64, device="cuda")
+    ctx0.jacobian(torch.zeros((coords.shape[0], 2), dtype=torch.float64, device="cuda"), J0)
+    ctx0.sync()
+    # one cell
+    ctx1 = StokesFO("hex8", _t(torch, conn[:1]), _t(torch, coords))
+    J1 = torch.empty((1, 16, 16), dtype=torch.float64, device="cuda")
+    U = np.random.default_rng(0).normal(0, 50, (coords.shape[0], 2))
+    ctx1.jacobian(_t(torch, U), J1)
+    ctx1.sync()
+    G, wm, _ = O.geometry(0, conn[:1], coords)
+    ref = O.evaluate(0, conn[:1], G, wm, U, k=10.77, mode="jac")
+    assert _cell_rel(J1.cpu().numpy(), ref["J_cell"]) <= TOL
+    # glen_n != 3
+    with pytest.raises(StokesFOError, match="EUNSUPPORTED"):
+        StokesFO("hex8", _t(torch, conn), _t(torch, coords), glen_n=2.0)
+    # inverted cell -> EMESH at sync
+    bad = conn.copy()
+    bad[0] = bad[0][[4, 5, 6, 7, 0, 1, 2, 3]]
+    ctxb = StokesFO("hex8", _t(torch, bad), _t(torch, coords))
+    with pytest.raises(StokesFOError, match="EMESH"):
+        ctxb.sync()
+    # conn out of range -> EMESH
+    bad2 = conn.copy()
+    bad2[1, 3] = coords.shape[0] + 5
+    ctxc = StokesFO("hex8", _t(torch, bad2), _t(torch, coords))
+    with pytest.raises(StokesFOError, match="EMESH"):
+        ctxc.sync()
+    # misaligned output pointer -> EINVAL
+    big = torch.empty(2 * 16 * 16 + 1, dtype=torch.float64, device="cuda")
+    lib = __import__("paper_conf_sc_antepara0cw24_b200.stokesfo", fromlist=["_lib"])._lib()
+    import ctypes
+    st = lib.stokesfo_jacobian(ctx1._h, ctypes.c_void_p(_t(torch, U).data_ptr()),
+                               ctypes.c_void_p(big.data_ptr() + 8), None, None)
+    assert st == 1
