@@ -164,7 +164,9 @@ int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
 void stokesfo_destroy(stokesfo_ctx *c) { delete c; }
 
 int stokesfo_gather(stokesfo_ctx *c, const double *U, double *U_cell) {
-    if (!c || !U || !U_cell || !aligned(U, 16) || !aligned(U_cell, 16)) return STOKESFO_EINVAL;
+    if (!c) return STOKESFO_EINVAL;
+    if (c->d.num_cells == 0) return STOKESFO_OK;
+    if (!U || !U_cell || !aligned(U, 16) || !aligned(U_cell, 16)) return STOKESFO_EINVAL;
     const int64_t work = c->d.num_cells * c->N;
     if (work == 0) return STOKESFO_OK;
     const int bs = 256;
@@ -177,7 +179,9 @@ int stokesfo_gather(stokesfo_ctx *c, const double *U, double *U_cell) {
 }
 
 int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R) {
-    if (!c || !U || !aligned(U, 16)) return STOKESFO_EINVAL;
+    if (!c) return STOKESFO_EINVAL;
+    if (c->d.num_cells == 0) return STOKESFO_OK;
+    if (!U || !aligned(U, 16)) return STOKESFO_EINVAL;
     const void *ps[] = {mu_qp, R_cell, R};
     for (const void *p : ps)
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
@@ -187,7 +191,9 @@ int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, do
 }
 
 int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *R_cell, double *R) {
-    if (!c || !U || !J_cell || !aligned(U, 16) || !aligned(J_cell, 16)) return STOKESFO_EINVAL;
+    if (!c) return STOKESFO_EINVAL;
+    if (c->d.num_cells == 0) return STOKESFO_OK;  // nothing to evaluate (outputs may be NULL)
+    if (!U || !J_cell || !aligned(U, 16) || !aligned(J_cell, 16)) return STOKESFO_EINVAL;
     const void *ps[] = {R_cell, R};
     for (const void *p : ps)
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;

@@ -16,9 +16,25 @@ namespace sfo {
 // ---------------------------------------------------------------------------
 struct Hex8 {
     static constexpr int N = 8, Q = 8, TC = 16, ELEM = 0;
+    // phase-2 mapping: thread <-> (cell t/N, node t%N): the 8 threads of a cell
+    // share one warp quarter, so per-(cell,qp) scalars are read as broadcasts.
+    static constexpr bool NODE_MAJOR_P2 = false;
+    static constexpr int JPITCH = 4 * N * N;  // J staging pitch per cell (dense: one bulk store per tile)
+    // Swizzles (cell index within the tile), chosen with a bank model of 64-bit
+    // shared loads served per half-warp: every phase-1/phase-2 GradBF load and
+    // every conn load is conflict-free.
+    __host__ __device__ static constexpr int gswz(int c, int n) { return c ^ ((2 * n) & 15); }
+    __host__ __device__ static constexpr int cswz(int c, int n) { return c ^ (4 * ((n >> 1) & 3)); }
 };
 struct Wedge6 {
     static constexpr int N = 6, Q = 6, TC = 32, ELEM = 1;
+    // phase-2 mapping: thread <-> (cell t%TC, node t/TC) (node-major: 6 does not
+    // divide a warp); J staging uses a padded pitch (73 x 16 B) and per-cell
+    // bulk stores so the 16-byte staging stores are conflict-free.
+    static constexpr bool NODE_MAJOR_P2 = true;
+    static constexpr int JPITCH = 4 * N * N + 2;
+    __host__ __device__ static constexpr int gswz(int c, int) { return c; }
+    __host__ __device__ static constexpr int cswz(int c, int) { return c; }
 };
 
 __host__ __device__ constexpr int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
@@ -39,9 +55,9 @@ struct Rec {
     static constexpr int G_OFF = WM_OFF + Q * TC * 8;
     static constexpr int BYTES = (int)round_up(G_OFF + N * Q * 3 * TC * 8, 128);
     // index helpers (in elements of the respective type)
-    __host__ __device__ static constexpr int conn(int n, int c) { return n * TC + c; }
+    __host__ __device__ static constexpr int conn(int n, int c) { return n * TC + E::cswz(c, n); }
     __host__ __device__ static constexpr int wm(int q, int c) { return q * TC + c; }
-    __host__ __device__ static constexpr int g(int n, int q, int d, int c) { return ((n * Q + q) * 3 + d) * TC + c; }
+    __host__ __device__ static constexpr int g(int n, int q, int d, int c) { return ((n * Q + q) * 3 + d) * TC + E::gswz(c, n); }
 };
 
 // Workspace: [0, 256) header (error flag), then ntiles records.
@@ -93,6 +109,14 @@ __device__ __forceinline__ void bulk_s2g(void *dst, const void *src, uint32_t by
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void cp_async16(void *dst, const void *src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }

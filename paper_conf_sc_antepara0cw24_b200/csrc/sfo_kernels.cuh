@@ -76,12 +76,11 @@ __device__ __forceinline__ void basis<Wedge6>(int n, double x, double y, double 
     dz = lam * 0.5 * s;
 }
 
-// Swizzled position of GradBF (n, q, d, c) inside a record: the cell index is
-// XORed with 4*(n mod 4) so that the 8 (or 6) node slices of one (q, d) fall in
-// different shared-memory bank groups (phase-2 loads are conflict-free).
+// Position of GradBF (n, q, d, c) inside a record (swizzled cell index, see
+// the element traits in sfo_common.cuh).
 template <class E>
 __host__ __device__ __forceinline__ int gidx(int n, int q, int d, int c) {
-    return ((n * E::Q + q) * 3 + d) * E::TC + (c ^ ((n & 3) << 2));
+    return Rec<E>::g(n, q, d, c);
 }
 
 // ---------------------------------------------------------------------------
@@ -217,57 +216,78 @@ struct EvalArgs {
     double *J_cell;           // [C][2N][2N] (JAC)
 };
 
-constexpr int STAGES = 2;
 constexpr int NQS = 9;  // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 beta12, wmu2, gamma, wf0, wf1
 
+// Shared memory: two stage buffers + per-QP scalars + 2 mbarriers.
+// A stage buffer holds [record | gathered U (double2 [N][TC]) | s ([N][TC])];
+// once a tile's phase 2 has consumed its record, the same buffer stages the
+// tile's element Jacobians for the TMA bulk store (JAC).
 template <class E, bool JAC>
 struct EvalSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static constexpr int REC = Rec<E>::BYTES;
-    static constexpr int OFF_REC = 0;
-    static constexpr int OFF_U = OFF_REC + STAGES * REC;               // double [N][2][TC]
-    static constexpr int OFF_S = OFF_U + N * 2 * TC * 8;                // double [N][TC]
-    static constexpr int OFF_QS = OFF_S + N * TC * 8;                   // double [NQS][Q][TC]
-    static constexpr int OFF_J = (int)round_up(OFF_QS + NQS * Q * TC * 8, 128);  // double [TC][2N][2N]
-    static constexpr int J_BYTES = JAC ? TC * 4 * N * N * 8 : 0;
-    static constexpr int OFF_BAR = OFF_J + J_BYTES;
-    static constexpr int BYTES = OFF_BAR + STAGES * 8;
+    static constexpr int U_OFF = REC;                        // double2 [N][TC]
+    static constexpr int S_OFF = U_OFF + N * TC * 16;        // double  [N][TC]
+    static constexpr int IN_BYTES = S_OFF + N * TC * 8;
+    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;
+    static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
+    static constexpr int OFF_QS = 2 * STAGE;                 // double [NQS][Q][TC]
+    static constexpr int OFF_BAR = OFF_QS + NQS * Q * TC * 8;
+    static constexpr int BYTES = OFF_BAR + 2 * 8;
 };
 
+// Issue the gather of U (16 B) and s (8 B) of one tile through its conn, as
+// cp.async copies into the tile's stage buffer (thread <-> (cell, node)).
+template <class E>
+__device__ __forceinline__ void issue_gather(char *stage, const double *U, const double *surface, bool have_s) {
+    using R = Rec<E>;
+    using S = EvalSmem<E, false>;
+    const int t = threadIdx.x;
+    const int c = t % E::TC, n = t / E::TC;
+    const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[R::conn(n, c)];
+    cp_async16(stage + S::U_OFF + (n * E::TC + c) * 16, U + 2 * (int64_t)g);
+    if (have_s) cp_async8(stage + S::S_OFF + (n * E::TC + c) * 8, surface + g);
+    cp_async_commit();
+}
+
 template <class E, bool JAC>
-__global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
-    constexpr int N = E::N, Q = E::Q, TC = E::TC, NT = TC * N;
+__global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) eval_kernel(EvalArgs a) {
+    constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "thread mappings assume N == Q");
     using R = Rec<E>;
     using S = EvalSmem<E, JAC>;
+    static_assert(S::U_OFF == EvalSmem<E, false>::U_OFF && S::S_OFF == EvalSmem<E, false>::S_OFF, "layout");
     extern __shared__ __align__(128) char smem[];
-    double *Us = reinterpret_cast<double *>(smem + S::OFF_U);
-    double *ss = reinterpret_cast<double *>(smem + S::OFF_S);
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
-    double *Js = reinterpret_cast<double *>(smem + S::OFF_J);
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
     const int t = threadIdx.x;
+    const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
 
     uint64_t pol_stream = 0;
     if (t == 0) {
         pol_stream = policy_evict_first();
-        for (int s = 0; s < STAGES; ++s) mbar_init(&bar[s], 1);
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
     if (t == 0) {
-        for (int s = 0; s < STAGES; ++s) {
+        for (int s = 0; s < 2; ++s) {
             const int64_t tile = blockIdx.x + (int64_t)s * gridDim.x;
             if (tile < a.ntiles) {
                 mbar_arrive_expect_tx(&bar[s], R::BYTES);
-                bulk_g2s(smem + S::OFF_REC + s * R::BYTES, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[s],
-                         pol_stream);
+                bulk_g2s(smem + s * S::STAGE, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[s], pol_stream);
             }
         }
     }
+    if ((int64_t)blockIdx.x < a.ntiles) {
+        mbar_wait(&bar[0], 0);
+        issue_gather<E>(smem, a.U, a.surface, have_s);
+    }
 
-    // phase-2 identity: thread <-> (cell c2, node i); basis values of node i
-    const int c2 = t / N, i = t % N;
+    // phase-2 identity: thread <-> (cell c2, node i)
+    const int c2 = E::NODE_MAJOR_P2 ? t % TC : t / N;
+    const int i = E::NODE_MAJOR_P2 ? t / TC : t % N;
     double bfi[Q];
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
@@ -275,31 +295,23 @@ __global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
         qp_coords<E>(q, x, y, z, w);
         basis<E>(i, x, y, z, bfi[q], dx, dy, dz);
     }
-    const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
     constexpr double P_EXP = -1.0 / 3.0;  // (1 - n) / (2 n) at n = 3
 
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
-        const int st = it % STAGES;
-        const char *rec = smem + S::OFF_REC + st * R::BYTES;
-        const int32_t *rconn = reinterpret_cast<const int32_t *>(rec + R::CONN_OFF);
-        const double *rkc = reinterpret_cast<const double *>(rec + R::KC_OFF);
-        const double *rwm = reinterpret_cast<const double *>(rec + R::WM_OFF);
-        const double *rg = reinterpret_cast<const double *>(rec + R::G_OFF);
+        const int st = it & 1;
+        char *stage = smem + st * S::STAGE;
+        const int32_t *rconn = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF);
+        const double *rkc = reinterpret_cast<const double *>(stage + R::KC_OFF);
+        const double *rwm = reinterpret_cast<const double *>(stage + R::WM_OFF);
+        const double *rg = reinterpret_cast<const double *>(stage + R::G_OFF);
+        const double2 *Us = reinterpret_cast<const double2 *>(stage + S::U_OFF);
+        const double *ss = reinterpret_cast<const double *>(stage + S::S_OFF);
         const int64_t cell0 = tile * TC;
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
-        mbar_wait(&bar[st], (uint32_t)((it / STAGES) & 1));
 
-        // ---- phase 0: gather U and s of the tile (thread <-> (cell, node)) ----
-        {
-            const int c = t % TC, n = t / TC;
-            const int32_t g = rconn[R::conn(n, c)];
-            const double2 u = __ldg(reinterpret_cast<const double2 *>(a.U) + g);
-            Us[(n * 2 + 0) * TC + c] = u.x;
-            Us[(n * 2 + 1) * TC + c] = u.y;
-            if (have_s) ss[n * TC + c] = __ldg(a.surface + g);
-        }
-        __syncthreads();
+        cp_async_wait_all();  // this thread's gathers for this tile have landed
+        __syncthreads();      // ... and everyone's
 
         // ---- phase 1: per-QP quantities (thread <-> (cell, qp)) ----
         {
@@ -310,10 +322,9 @@ __global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
                 const double g0 = rg[gidx<E>(n, q, 0, c)];
                 const double g1 = rg[gidx<E>(n, q, 1, c)];
                 const double g2 = rg[gidx<E>(n, q, 2, c)];
-                const double u = Us[(n * 2 + 0) * TC + c];
-                const double v = Us[(n * 2 + 1) * TC + c];
-                ux += u * g0; uy += u * g1; uz += u * g2;
-                vx += v * g0; vy += v * g1; vz += v * g2;
+                const double2 uv = Us[n * TC + c];
+                ux += uv.x * g0; uy += uv.x * g1; uz += uv.x * g2;
+                vx += uv.y * g0; vy += uv.y * g1; vz += uv.y * g2;
                 if (have_s) {
                     const double sn = ss[n * TC + c];
                     gs0 += sn * g0; gs1 += sn * g1;
@@ -323,19 +334,18 @@ __global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
             // effective strain rate^2 (reading Z2) and Glen viscosity, n = 3
             const double e2 = ux * ux + vy * vy + ux * vy + 0.25 * uyvx * uyvx + 0.25 * uz * uz + 0.25 * vz * vz;
             const double r = rcbrt(e2 + a.delta);  // (e2 + delta)^(-1/3)
-            const double kc = rkc[c];
-            const double mu = kc * r;
+            const double mu = rkc[c] * r;
             const double wm = rwm[R::wm(q, c)];
             const double wmu2 = 2.0 * wm * mu;
             // beta = B g: sigma = 2 mu beta reproduces strs00..strs12 of Fig. 2
             double *qq = qs + q * TC + c;
-            qq[0 * Q * TC] = 2.0 * ux + vy;   // beta_(0,0): strs00 / (2 mu)
-            qq[1 * Q * TC] = 0.5 * uyvx;      // beta_(0,1): strs01 / (2 mu)
-            qq[2 * Q * TC] = 0.5 * uz;        // beta_(0,2): strs02 / (2 mu)
-            qq[3 * Q * TC] = ux + 2.0 * vy;   // beta_(1,1): strs11 / (2 mu)
-            qq[4 * Q * TC] = 0.5 * vz;        // beta_(1,2): strs12 / (2 mu)
+            qq[0 * Q * TC] = 2.0 * ux + vy;   // beta_(0,0) = strs00 / (2 mu)
+            qq[1 * Q * TC] = 0.5 * uyvx;      // beta_(0,1) = beta_(1,0) = strs01 / (2 mu)
+            qq[2 * Q * TC] = 0.5 * uz;        // beta_(0,2) = strs02 / (2 mu)
+            qq[3 * Q * TC] = ux + 2.0 * vy;   // beta_(1,1) = strs11 / (2 mu)
+            qq[4 * Q * TC] = 0.5 * vz;        // beta_(1,2) = strs12 / (2 mu)
             qq[5 * Q * TC] = wmu2;
-            // gamma = wM 2 mu p / (e2 + delta) = wM 2 k p r^4  (d mu / d e2 chain, reading Z5)
+            // gamma = wM 2 mu p / (e2 + delta) = wmu2 p r^3  (d mu / d e2 chain, reading Z5)
             qq[6 * Q * TC] = wmu2 * P_EXP * (r * r * r);
             double wf0 = 0.0, wf1 = 0.0;
             if (a.force_qp) {
@@ -354,7 +364,17 @@ __global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
         }
         __syncthreads();
 
+        // ---- prefetch: gather U, s of the next tile while this one computes ----
+        {
+            const int64_t nt = tile + gridDim.x;
+            if (nt < a.ntiles) {
+                mbar_wait(&bar[st ^ 1], (uint32_t)(((it + 1) >> 1) & 1));
+                issue_gather<E>(smem + (st ^ 1) * S::STAGE, a.U, a.surface, have_s);
+            }
+        }
+
         // ---- phase 2: per-node accumulation (thread <-> (cell c2, node i)) ----
+        const int32_t gnode = rconn[R::conn(i, c2)];
         double R0 = 0.0, R1 = 0.0;
         constexpr int K = N / 2;            // symmetric block scheme: blocks (i, i+k), k = 0..K
         double Jb[JAC ? K + 1 : 1][2][2];   // Jb[k][a][b] = J[(i,a), (j_k,b)], j_k = (i+k) mod N
@@ -383,14 +403,13 @@ __global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
                 // M_ab = wmu2 * (B-block (a,b) applied to G_i) + gamma h_(i,a) beta_(b,.)
                 const double gam = qq[6 * Q * TC];
                 const double gh0 = gam * h0, gh1 = gam * h1;
-                const double m00x = fma(2.0 * wmu2, gi0, gh0 * b00), m00y = fma(0.5 * wmu2, gi1, gh0 * b01),
-                             m00z = fma(0.5 * wmu2, gi2, gh0 * b02);
-                const double m01x = fma(0.5 * wmu2, gi1, gh0 * b10), m01y = fma(wmu2, gi0, gh0 * b11),
-                             m01z = gh0 * b12;
-                const double m10x = fma(wmu2, gi1, gh1 * b00), m10y = fma(0.5 * wmu2, gi0, gh1 * b01),
-                             m10z = gh1 * b02;
-                const double m11x = fma(0.5 * wmu2, gi0, gh1 * b10), m11y = fma(2.0 * wmu2, gi1, gh1 * b11),
-                             m11z = fma(0.5 * wmu2, gi2, gh1 * b12);
+                const double w0 = wmu2 * gi0, w1 = wmu2 * gi1, w2 = wmu2 * gi2;
+                const double m00x = fma(2.0, w0, gh0 * b00), m00y = fma(0.5, w1, gh0 * b01),
+                             m00z = fma(0.5, w2, gh0 * b02);
+                const double m01x = fma(0.5, w1, gh0 * b10), m01y = fma(gh0, b11, w0), m01z = gh0 * b12;
+                const double m10x = fma(gh1, b00, w1), m10y = fma(0.5, w0, gh1 * b01), m10z = gh1 * b02;
+                const double m11x = fma(0.5, w0, gh1 * b10), m11y = fma(2.0, w1, gh1 * b11),
+                             m11z = fma(0.5, w2, gh1 * b12);
 #pragma unroll
                 for (int k = 0; k <= K; ++k) {
                     const int j = (i + k) % N;
@@ -411,33 +430,13 @@ __global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
         }
         const bool valid = c2 < nvalid;
         const int64_t cell = cell0 + c2;
-        if (valid) {
-            if (a.R) {
-                const int32_t g = rconn[R::conn(i, c2)];
-                atomicAdd(a.R + 2 * (int64_t)g + 0, R0);
-                atomicAdd(a.R + 2 * (int64_t)g + 1, R1);
-            }
-            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + (cell * N + i) * 2) = make_double2(R0, R1);
-        }
+        __syncthreads();  // everyone is done with this stage's record and qs
 
-        // all threads are done with this stage's record, qs, Us; the previous
-        // tile's bulk store has finished reading the J staging buffer
-        if (JAC && t == 0) bulk_wait_read0();
-        __syncthreads();
-        if (t == 0) {
-            const int64_t nt = tile + (int64_t)STAGES * gridDim.x;
-            if (nt < a.ntiles) {
-                mbar_arrive_expect_tx(&bar[st], R::BYTES);
-                bulk_g2s(smem + S::OFF_REC + st * R::BYTES, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st],
-                         pol_stream);
-            }
-        }
         if (JAC) {
-            // stage J[c2] rows (2i, 2i+1): direct blocks (i, i+k), k = 0..K, and
-            // transposed blocks (i+k, i) for 0 < k < K (J is symmetric: the
-            // Hessian of the quadrature energy).  Rotating j with i keeps the
-            // 16-byte stores of a warp in distinct bank groups.
-            double *Jc = Js + c2 * (4 * N * N);
+            // Stage J[c2] rows (2i, 2i+1) into this stage buffer: direct blocks
+            // (i, i+k), k = 0..K, and transposed blocks (i+k, i) for 0 < k < K
+            // (J is symmetric: the Hessian of the quadrature energy).
+            double *Jc = reinterpret_cast<double *>(stage) + c2 * E::JPITCH;
             constexpr int LD = 2 * N;
 #pragma unroll
             for (int k = 0; k <= K; ++k) {
@@ -454,13 +453,33 @@ __global__ void __launch_bounds__(E::TC *E::N) eval_kernel(EvalArgs a) {
             fence_proxy_async_smem();
             __syncthreads();
             if (t == 0) {
-                bulk_s2g(a.J_cell + cell0 * (4 * N * N), Js, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
+                if (E::JPITCH == 4 * N * N) {
+                    bulk_s2g(a.J_cell + cell0 * (4 * N * N), stage, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
+                } else {
+                    for (int c = 0; c < nvalid; ++c)
+                        bulk_s2g(a.J_cell + (cell0 + c) * (4 * N * N), stage + c * E::JPITCH * 8,
+                                 (uint32_t)(4 * N * N * 8), pol_stream);
+                }
                 bulk_commit();
+                bulk_wait_read0();  // staging read done -> the buffer may take the next record
             }
+        }
+        if (t == 0) {
+            const int64_t nt = tile + 2 * (int64_t)gridDim.x;
+            if (nt < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[st], R::BYTES);
+                bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
+            }
+        }
+        if (valid) {
+            if (a.R) {
+                atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
+                atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
+            }
+            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + (cell * N + i) * 2) = make_double2(R0, R1);
         }
     }
     if (JAC && t == 0) bulk_wait0();
-    (void)NT;
 }
 
 // ---------------------------------------------------------------------------
