@@ -4,6 +4,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -22,6 +23,7 @@ struct stokesfo_ctx {
     char *recs;            // device records
     int grid_resid, grid_jac;
     int rec_bytes;
+    int nstage_resid, nstage_jac;  // TMA record ring depth of the eval kernels
     const int64_t *rowptr = nullptr;  // CSR pattern (set by stokesfo_csr_pattern)
     const int32_t *colidx = nullptr;
     int64_t csr_rows = 0;
@@ -40,16 +42,21 @@ int cuda_status() {
     return STOKESFO_OK;
 }
 
+template <class E, bool JAC>
+constexpr int default_stages() {
+    return 2;
+}
+
 template <class E>
 int64_t ws_bytes(int64_t ncells) {
     const int64_t ntiles = (ncells + E::TC - 1) / E::TC;
     return WS_HEADER + ntiles * (int64_t)Rec<E>::BYTES;
 }
 
-template <class E, bool JAC>
+template <class E, bool JAC, int NS>
 int configure_eval(int *grid) {
-    using S = EvalSmem<E, JAC>;
-    auto fn = eval_kernel<E, JAC>;
+    using S = EvalSmem<E, JAC, NS>;
+    auto fn = eval_kernel<E, JAC, NS>;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES) != cudaSuccess)
         return cuda_status();
     int dev = 0, sms = 0, per_sm = 0;
@@ -68,9 +75,15 @@ int create_impl(stokesfo_ctx *c) {
     c->TC = E::TC;
     c->rec_bytes = Rec<E>::BYTES;
     c->ntiles = (c->d.num_cells + E::TC - 1) / E::TC;
-    int st = configure_eval<E, false>(&c->grid_resid);
+    // ring depth: default per element, STOKESFO_STAGES_{RESID,JAC} override (2 or 3)
+    c->nstage_resid = default_stages<E, false>();
+    c->nstage_jac = default_stages<E, true>();
+    if (const char *e = getenv("STOKESFO_STAGES_RESID")) c->nstage_resid = atoi(e) == 3 ? 3 : 2;
+    if (const char *e = getenv("STOKESFO_STAGES_JAC")) c->nstage_jac = atoi(e) == 3 ? 3 : 2;
+    int st = c->nstage_resid == 3 ? configure_eval<E, false, 3>(&c->grid_resid)
+                                  : configure_eval<E, false, 2>(&c->grid_resid);
     if (st) return st;
-    st = configure_eval<E, true>(&c->grid_jac);
+    st = c->nstage_jac == 3 ? configure_eval<E, true, 3>(&c->grid_jac) : configure_eval<E, true, 2>(&c->grid_jac);
     if (st) return st;
     if (cudaMemsetAsync(c->err, 0, sizeof(int), c->stream) != cudaSuccess) return cuda_status();
     if (c->ntiles > 0) {
@@ -99,7 +112,10 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.R = R;
     a.J_cell = J_cell;
     const int grid = (int)std::min<int64_t>(JAC ? c->grid_jac : c->grid_resid, c->ntiles);
-    eval_kernel<E, JAC><<<grid, E::TC * E::N, EvalSmem<E, JAC>::BYTES, c->stream>>>(a);
+    if ((JAC ? c->nstage_jac : c->nstage_resid) == 3)
+        eval_kernel<E, JAC, 3><<<grid, E::TC * E::N, EvalSmem<E, JAC, 3>::BYTES, c->stream>>>(a);
+    else
+        eval_kernel<E, JAC, 2><<<grid, E::TC * E::N, EvalSmem<E, JAC, 2>::BYTES, c->stream>>>(a);
     return cuda_status();
 }
 

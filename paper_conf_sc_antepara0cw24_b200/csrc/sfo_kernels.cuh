@@ -222,7 +222,7 @@ constexpr int NQS = 9;  // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 b
 // A stage buffer holds [record | gathered U (double2 [N][TC]) | s ([N][TC])];
 // once a tile's phase 2 has consumed its record, the same buffer stages the
 // tile's element Jacobians for the TMA bulk store (JAC).
-template <class E, bool JAC>
+template <class E, bool JAC, int NSTAGE = 2>
 struct EvalSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static constexpr int REC = Rec<E>::BYTES;
@@ -231,9 +231,9 @@ struct EvalSmem {
     static constexpr int IN_BYTES = S_OFF + N * TC * 8;
     static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
-    static constexpr int OFF_QS = 2 * STAGE;                 // double [NQS][Q][TC]
+    static constexpr int OFF_QS = NSTAGE * STAGE;            // double [NQS][Q][TC]
     static constexpr int OFF_BAR = OFF_QS + NQS * Q * TC * 8;
-    static constexpr int BYTES = OFF_BAR + 2 * 8;
+    static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
 };
 
 // Issue the gather of U (16 B) and s (8 B) of one tile through its conn, as
@@ -250,12 +250,19 @@ __device__ __forceinline__ void issue_gather(char *stage, const double *U, const
     cp_async_commit();
 }
 
-template <class E, bool JAC>
-__global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) eval_kernel(EvalArgs a) {
+// Resident CTAs per SM the register budget is tuned for (shared memory permits
+// this many for hex8 at the given stage count).
+template <class E, bool JAC, int NSTAGE>
+constexpr int min_blocks() {
+    return E::N == 8 ? (NSTAGE == 2 ? 3 : 2) : 2;
+}
+
+template <class E, bool JAC, int NSTAGE>
+__global__ void __launch_bounds__(E::TC *E::N, (min_blocks<E, JAC, NSTAGE>())) eval_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "thread mappings assume N == Q");
     using R = Rec<E>;
-    using S = EvalSmem<E, JAC>;
+    using S = EvalSmem<E, JAC, NSTAGE>;
     static_assert(S::U_OFF == EvalSmem<E, false>::U_OFF && S::S_OFF == EvalSmem<E, false>::S_OFF, "layout");
     extern __shared__ __align__(128) char smem[];
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
@@ -266,13 +273,12 @@ __global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) ev
     uint64_t pol_stream = 0;
     if (t == 0) {
         pol_stream = policy_evict_first();
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
+        for (int s = 0; s < NSTAGE; ++s) mbar_init(&bar[s], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
     if (t == 0) {
-        for (int s = 0; s < 2; ++s) {
+        for (int s = 0; s < NSTAGE; ++s) {
             const int64_t tile = blockIdx.x + (int64_t)s * gridDim.x;
             if (tile < a.ntiles) {
                 mbar_arrive_expect_tx(&bar[s], R::BYTES);
@@ -299,7 +305,7 @@ __global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) ev
 
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
-        const int st = it & 1;
+        const int st = it % NSTAGE;
         char *stage = smem + st * S::STAGE;
         const int32_t *rconn = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF);
         const double *rkc = reinterpret_cast<const double *>(stage + R::KC_OFF);
@@ -364,15 +370,6 @@ __global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) ev
         }
         __syncthreads();
 
-        // ---- prefetch: gather U, s of the next tile while this one computes ----
-        {
-            const int64_t nt = tile + gridDim.x;
-            if (nt < a.ntiles) {
-                mbar_wait(&bar[st ^ 1], (uint32_t)(((it + 1) >> 1) & 1));
-                issue_gather<E>(smem + (st ^ 1) * S::STAGE, a.U, a.surface, have_s);
-            }
-        }
-
         // ---- phase 2: per-node accumulation (thread <-> (cell c2, node i)) ----
         const int32_t gnode = rconn[R::conn(i, c2)];
         double R0 = 0.0, R1 = 0.0;
@@ -384,6 +381,16 @@ __global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) ev
         }
 #pragma unroll
         for (int q = 0; q < Q; ++q) {
+            if (q == Q / 2) {
+                // prefetch: gather U, s of the next tile (its record was issued
+                // NSTAGE-1 tiles ago) while the rest of this tile computes
+                const int64_t nt = tile + gridDim.x;
+                if (nt < a.ntiles) {
+                    const int ns = (it + 1) % NSTAGE;
+                    mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NSTAGE) & 1));
+                    issue_gather<E>(smem + ns * S::STAGE, a.U, a.surface, have_s);
+                }
+            }
             const double *qq = qs + q * TC + c2;
             const double b00 = qq[0 * Q * TC], b01 = qq[1 * Q * TC], b02 = qq[2 * Q * TC];
             const double b11 = qq[3 * Q * TC], b12 = qq[4 * Q * TC];
@@ -394,10 +401,10 @@ __global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) ev
             const double gi1 = rg[gidx<E>(i, q, 1, c2)];
             const double gi2 = rg[gidx<E>(i, q, 2, c2)];
             // h_(i,a) = sum_d G_i[d] beta_(a,d);  residual row (i,a) = wmu2 h + wf_a BF_i
-            const double h0 = gi0 * b00 + gi1 * b01 + gi2 * b02;
-            const double h1 = gi0 * b10 + gi1 * b11 + gi2 * b12;
-            R0 += wmu2 * h0 + wf0 * bfi[q];
-            R1 += wmu2 * h1 + wf1 * bfi[q];
+            const double h0 = fma(gi2, b02, fma(gi1, b01, gi0 * b00));
+            const double h1 = fma(gi2, b12, fma(gi1, b11, gi0 * b10));
+            R0 = fma(wf0, bfi[q], fma(wmu2, h0, R0));
+            R1 = fma(wf1, bfi[q], fma(wmu2, h1, R1));
             if (JAC) {
                 // J_q[(i,a),(j,b)] = sum_e M_ab[e] G_j[e] with
                 // M_ab = wmu2 * (B-block (a,b) applied to G_i) + gamma h_(i,a) beta_(b,.)
@@ -421,10 +428,11 @@ __global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) ev
                         gj1 = rg[gidx<E>(j, q, 1, c2)];
                         gj2 = rg[gidx<E>(j, q, 2, c2)];
                     }
-                    Jb[k][0][0] += m00x * gj0 + m00y * gj1 + m00z * gj2;
-                    Jb[k][0][1] += m01x * gj0 + m01y * gj1 + m01z * gj2;
-                    Jb[k][1][0] += m10x * gj0 + m10y * gj1 + m10z * gj2;
-                    Jb[k][1][1] += m11x * gj0 + m11y * gj1 + m11z * gj2;
+                    // explicit 3-deep DFMA chains into the accumulators (no DMUL/DADD)
+                    Jb[k][0][0] = fma(m00z, gj2, fma(m00y, gj1, fma(m00x, gj0, Jb[k][0][0])));
+                    Jb[k][0][1] = fma(m01z, gj2, fma(m01y, gj1, fma(m01x, gj0, Jb[k][0][1])));
+                    Jb[k][1][0] = fma(m10z, gj2, fma(m10y, gj1, fma(m10x, gj0, Jb[k][1][0])));
+                    Jb[k][1][1] = fma(m11z, gj2, fma(m11y, gj1, fma(m11x, gj0, Jb[k][1][1])));
                 }
             }
         }
@@ -465,7 +473,7 @@ __global__ void __launch_bounds__(E::TC *E::N, JAC ? (E::N == 8 ? 3 : 2) : 3) ev
             }
         }
         if (t == 0) {
-            const int64_t nt = tile + 2 * (int64_t)gridDim.x;
+            const int64_t nt = tile + (int64_t)NSTAGE * gridDim.x;
             if (nt < a.ntiles) {
                 mbar_arrive_expect_tx(&bar[st], R::BYTES);
                 bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
