@@ -30,17 +30,23 @@ WORKLOADS = {
     "C4": "C4 Antarctica-like 4 km footprint x 10 layers, hex8, 8 QPs, residual+Jacobian (BASELINE.json configs[3])",
     "C5": "C5 Antarctica-like wedge6 (quads split), 10 layers, 6 QPs, residual+Jacobian (BASELINE.json configs[4])",
     "C1": "C1/C2 tiny 16x16 footprint x 5 layers, hex8, residual+Jacobian (BASELINE.json configs[1])",
+    "C3": "C3 Greenland-like 1-10 km NVB footprint x 10 layers, hex8, residual+Jacobian (BASELINE.json configs[2])",
 }
 
 
-def bytes_per_launch(elem: str, cells: int, nodes: int) -> int:
+def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored") -> int:
     """Algorithmic (compulsory) HBM bytes of one stokesfo_jacobian launch with
-    assembled R: per cell conn 4N +
-    GradBF 24NQ + wMeasure 8Q + k_c 8 + J_cell 8(2N)^2; per node U 16 + s 8 +
-    R read+write 32."""
+    assembled R.
+    stored:     per cell conn 4N + GradBF 24NQ + wMeasure 8Q + k_c 8 + J_cell 8(2N)^2;
+                per node U 16 + s 8 + R read+write 32.
+    on_the_fly: per cell conn 4N + k_c 8 + J_cell 8(2N)^2;
+                per node U 16 + s 8 + R 32 + coordinates 32 (x, y, z, pad)."""
     N = 8 if elem == "hex8" else 6
     Q = N
-    per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + 8 * (2 * N) ** 2
+    J = 8 * (2 * N) ** 2
+    if geometry == "on_the_fly":
+        return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32)
+    per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + J
     return cells * per_cell + nodes * (16 + 8 + 32)
 
 
@@ -114,7 +120,7 @@ def build_mesh(cfg: str):
     from paper_conf_sc_antepara0cw24_b200 import mesh_extrude, synth
     fp, L, elem = synth.make_config(cfg)
     conn, coords = mesh_extrude(fp.xy, fp.polys, fp.b, fp.H, L)
-    U = synth.velocity_balance(fp, L, seed=12)
+    U = synth.velocity_balance(fp, L, seed=11 if cfg == "C3" else 12)
     s = synth.surface_nodal(fp, L)
     kc = synth.flow_factor(fp, L)
     return fp, L, elem, conn, coords, U, s, kc
@@ -192,6 +198,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
@@ -223,7 +230,7 @@ def main():
     C, NN = conn.shape[0], coords.shape[0]
     N = conn.shape[1]
     stream = torch.cuda.current_stream(dev)
-    ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream)
+    ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream, geometry=args.geometry)
     J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device=dev)
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     halo = None
@@ -303,14 +310,14 @@ def main():
 
     if rank == 0:
         peak, peak_src = load_peaks()
-        bpl = bytes_per_launch(elem, C, NN)
+        bpl = bytes_per_launch(elem, C, NN, args.geometry)
         achieved = bpl / (kern_ms_max * 1e-3) / 1e9
         traffic = None
         tpath = os.path.join(ROOT, "profiles", "traffic.json")
         if os.path.exists(tpath):
             with open(tpath) as f:
                 tr = json.load(f)
-            key = f"{args.config}:{elem}:jacobian"
+            key = f"{args.config}:{elem}:jacobian:{args.geometry}"
             if key in tr and world == 1:
                 traffic = tr[key]["dram_bytes_per_launch"]
         line = {
@@ -327,13 +334,14 @@ def main():
             "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": WORKLOADS[args.config], "cells": total_cells, "elem": elem, "layers": L,
+                       "geometry": args.geometry,
                        "cells_rank0": C, "nodes_rank0": NN, "parallelism": f"column-partition x{world}",
                        "l2": "inputs exceed L2 (no flush needed)",
                        "launch": ctx.launch_info()},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "eval_kernel<Hex8,true> (stokesfo_jacobian)" if elem == "hex8"
-                         else "eval_kernel<Wedge6,true> (stokesfo_jacobian)",
+                         "kernel": ("eval_otf_kernel" if args.geometry == "on_the_fly" else "eval_kernel")
+                         + ("<Hex8,true>" if elem == "hex8" else "<Wedge6,true>") + " (stokesfo_jacobian)",
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src},
             "achieved_hbm_gbs": achieved,
             "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),

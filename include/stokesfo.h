@@ -61,6 +61,16 @@ typedef struct stokesfo_ctx stokesfo_ctx; /* opaque host object */
 
 typedef enum { STOKESFO_HEX8 = 0, STOKESFO_WEDGE6 = 1 } stokesfo_elem_t;
 
+/* Where GradBF = J^-T grad_xi phi and wMeasure = w det J (eq. (3) inputs
+ * {phi_i}, {grad phi_i}) come from during an evaluation:
+ *   STORED:     precomputed once by stokesfo_create and streamed
+ *               from the workspace at every evaluation (1,640 B/cell hex8);
+ *   ON_THE_FLY: recomputed per tile from the gathered node coordinates inside
+ *               the evaluation kernels (40 streamed B/cell hex8; det J <= 0 is
+ *               re-checked at every evaluation).
+ * Both give the same results up to rounding (parity-tested at 1e-12). */
+typedef enum { STOKESFO_GEOMETRY_STORED = 0, STOKESFO_GEOMETRY_ON_THE_FLY = 1 } stokesfo_geometry_mode_t;
+
 typedef enum {
     STOKESFO_OK = 0,
     STOKESFO_EINVAL = 1,       /* bad argument, size or alignment */
@@ -87,15 +97,20 @@ typedef struct {
     void *workspace;             /* dev, caller-owned, >= stokesfo_workspace_size() bytes */
     size_t workspace_bytes;
     void *stream;                /* cudaStream_t used by every call (NULL = legacy default) */
+    int32_t geometry_mode;       /* stokesfo_geometry_mode_t */
+    int32_t reserved0;
 } stokesfo_desc_t;
 
-/* Bytes of workspace needed for desc (only elem and num_cells are read). */
+/* Bytes of workspace needed for desc (reads elem, num_cells, num_nodes and
+ * geometry_mode). */
 int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes);
 
 /* Validate desc and run the basis/quadrature precompute:
  * GradBF[c][n][q][:] = J_q^-T grad_xi phi_n(xi_q), wMeasure[c][q] = w_q det J_q
- * into the workspace, plus a snapshot of conn and the flow factor.  Async on
- * desc.stream; det J <= 0 or conn out of range is reported by stokesfo_sync. */
+ * into the workspace (STORED mode; ON_THE_FLY mode stores node coordinates
+ * instead and checks det J), plus a snapshot of conn and the flow factor.
+ * Async on desc.stream; det J <= 0 or conn out of range is reported by
+ * stokesfo_sync. */
 int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out);
 
 /* Gather: U_cell[c][n][a] = U[2 conn[c][n] + a].

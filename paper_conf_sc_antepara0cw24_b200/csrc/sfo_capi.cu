@@ -20,7 +20,9 @@ struct stokesfo_ctx {
     int N, Q, TC;
     int64_t ntiles;
     int *err;              // device flag in the workspace header
-    char *recs;            // device records
+    char *recs;            // device records (full or light)
+    double4 *xyz4;         // node coordinates (on-the-fly geometry mode)
+    int mode;              // stokesfo_geometry_mode_t
     int grid_resid, grid_jac;
     int rec_bytes;
     int nstage_resid, nstage_jac;  // TMA record ring depth of the eval kernels
@@ -48,9 +50,31 @@ constexpr int default_stages() {
 }
 
 template <class E>
-int64_t ws_bytes(int64_t ncells) {
+int64_t xyz4_bytes(int64_t nnodes) {
+    return round_up(nnodes * 32, 256);
+}
+
+template <class E>
+int64_t ws_bytes(int64_t ncells, int64_t nnodes, int mode) {
     const int64_t ntiles = (ncells + E::TC - 1) / E::TC;
+    if (mode == STOKESFO_GEOMETRY_ON_THE_FLY)
+        return WS_HEADER + xyz4_bytes<E>(nnodes) + ntiles * (int64_t)Rec<E>::LIGHT_BYTES;
     return WS_HEADER + ntiles * (int64_t)Rec<E>::BYTES;
+}
+
+template <class E, bool JAC>
+int configure_otf(int *grid) {
+    using S = OtfSmem<E, JAC>;
+    auto fn = eval_otf_kernel<E, JAC>;
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES) != cudaSuccess)
+        return cuda_status();
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, E::TC * E::N, S::BYTES) != cudaSuccess)
+        return cuda_status();
+    *grid = std::max(1, sms * std::max(1, per_sm));
+    return STOKESFO_OK;
 }
 
 template <class E, bool JAC, int NS>
@@ -73,24 +97,46 @@ int create_impl(stokesfo_ctx *c) {
     c->N = E::N;
     c->Q = E::Q;
     c->TC = E::TC;
-    c->rec_bytes = Rec<E>::BYTES;
     c->ntiles = (c->d.num_cells + E::TC - 1) / E::TC;
-    // ring depth: default per element, STOKESFO_STAGES_{RESID,JAC} override (2 or 3)
-    c->nstage_resid = default_stages<E, false>();
-    c->nstage_jac = default_stages<E, true>();
-    if (const char *e = getenv("STOKESFO_STAGES_RESID")) c->nstage_resid = atoi(e) == 3 ? 3 : 2;
-    if (const char *e = getenv("STOKESFO_STAGES_JAC")) c->nstage_jac = atoi(e) == 3 ? 3 : 2;
-    int st = c->nstage_resid == 3 ? configure_eval<E, false, 3>(&c->grid_resid)
+    const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
+    c->rec_bytes = otf ? Rec<E>::LIGHT_BYTES : Rec<E>::BYTES;
+    int st;
+    if (otf) {
+        c->nstage_resid = c->nstage_jac = NLIGHT;
+        st = configure_otf<E, false>(&c->grid_resid);
+        if (st) return st;
+        st = configure_otf<E, true>(&c->grid_jac);
+        if (st) return st;
+    } else {
+        // ring depth: default per element, STOKESFO_STAGES_{RESID,JAC} override (2 or 3)
+        c->nstage_resid = default_stages<E, false>();
+        c->nstage_jac = default_stages<E, true>();
+        if (const char *e = getenv("STOKESFO_STAGES_RESID")) c->nstage_resid = atoi(e) == 3 ? 3 : 2;
+        if (const char *e = getenv("STOKESFO_STAGES_JAC")) c->nstage_jac = atoi(e) == 3 ? 3 : 2;
+        st = c->nstage_resid == 3 ? configure_eval<E, false, 3>(&c->grid_resid)
                                   : configure_eval<E, false, 2>(&c->grid_resid);
-    if (st) return st;
-    st = c->nstage_jac == 3 ? configure_eval<E, true, 3>(&c->grid_jac) : configure_eval<E, true, 2>(&c->grid_jac);
-    if (st) return st;
+        if (st) return st;
+        st = c->nstage_jac == 3 ? configure_eval<E, true, 3>(&c->grid_jac) : configure_eval<E, true, 2>(&c->grid_jac);
+        if (st) return st;
+    }
     if (cudaMemsetAsync(c->err, 0, sizeof(int), c->stream) != cudaSuccess) return cuda_status();
     if (c->ntiles > 0) {
-        const int64_t work = c->ntiles * E::TC * E::Q;
         const int bs = 256;
-        geometry_kernel<E><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
-            c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.coords, c->d.flow_factor, c->d.k, c->recs, c->err);
+        if (otf) {
+            xyz4_kernel<<<(unsigned)((c->d.num_nodes + bs - 1) / bs), bs, 0, c->stream>>>(c->d.num_nodes, c->d.coords,
+                                                                                          c->xyz4);
+            light_record_kernel<E><<<(unsigned)((c->ntiles * E::TC + bs - 1) / bs), bs, 0, c->stream>>>(
+                c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.flow_factor, c->d.k, c->recs, c->err);
+            const int64_t work = c->d.num_cells * E::Q;
+            geometry_kernel<E, GEO_CHECK><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
+                c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.coords, nullptr, 0.0, nullptr, nullptr, nullptr,
+                c->err);
+        } else {
+            const int64_t work = c->ntiles * E::TC * E::Q;
+            geometry_kernel<E, GEO_RECORDS><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
+                c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.coords, c->d.flow_factor, c->d.k, c->recs, nullptr,
+                nullptr, c->err);
+        }
     }
     return cuda_status();
 }
@@ -100,6 +146,8 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     if (c->ntiles == 0) return STOKESFO_OK;
     EvalArgs a;
     a.recs = c->recs;
+    a.xyz4 = c->xyz4;
+    a.err = c->err;
     a.ntiles = c->ntiles;
     a.ncells = c->d.num_cells;
     a.U = U;
@@ -112,7 +160,9 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.R = R;
     a.J_cell = J_cell;
     const int grid = (int)std::min<int64_t>(JAC ? c->grid_jac : c->grid_resid, c->ntiles);
-    if ((JAC ? c->nstage_jac : c->nstage_resid) == 3)
+    if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY)
+        eval_otf_kernel<E, JAC><<<grid, E::TC * E::N, OtfSmem<E, JAC>::BYTES, c->stream>>>(a);
+    else if ((JAC ? c->nstage_jac : c->nstage_resid) == 3)
         eval_kernel<E, JAC, 3><<<grid, E::TC * E::N, EvalSmem<E, JAC, 3>::BYTES, c->stream>>>(a);
     else
         eval_kernel<E, JAC, 2><<<grid, E::TC * E::N, EvalSmem<E, JAC, 2>::BYTES, c->stream>>>(a);
@@ -140,8 +190,10 @@ const char *stokesfo_strerror(int s) {
 
 int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes) {
     if (!d || !bytes || d->num_cells < 0) return STOKESFO_EINVAL;
-    if (d->elem == STOKESFO_HEX8) *bytes = (size_t)ws_bytes<Hex8>(d->num_cells);
-    else if (d->elem == STOKESFO_WEDGE6) *bytes = (size_t)ws_bytes<Wedge6>(d->num_cells);
+    if (d->geometry_mode != STOKESFO_GEOMETRY_STORED && d->geometry_mode != STOKESFO_GEOMETRY_ON_THE_FLY)
+        return STOKESFO_EINVAL;
+    if (d->elem == STOKESFO_HEX8) *bytes = (size_t)ws_bytes<Hex8>(d->num_cells, d->num_nodes, d->geometry_mode);
+    else if (d->elem == STOKESFO_WEDGE6) *bytes = (size_t)ws_bytes<Wedge6>(d->num_cells, d->num_nodes, d->geometry_mode);
     else return STOKESFO_EINVAL;
     return STOKESFO_OK;
 }
@@ -160,14 +212,22 @@ int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
     if (!d->workspace || !aligned(d->workspace, 256)) return STOKESFO_EINVAL;
     size_t need = 0;
-    stokesfo_workspace_size(d, &need);
+    if (stokesfo_workspace_size(d, &need) != STOKESFO_OK) return STOKESFO_EINVAL;
     if (d->workspace_bytes < need) return STOKESFO_ENOMEM;
     stokesfo_ctx *c = new (std::nothrow) stokesfo_ctx();
     if (!c) return STOKESFO_ENOMEM;
     c->d = *d;
     c->stream = reinterpret_cast<cudaStream_t>(d->stream);
     c->err = reinterpret_cast<int *>(d->workspace);
-    c->recs = reinterpret_cast<char *>(d->workspace) + WS_HEADER;
+    c->mode = d->geometry_mode;
+    char *ws = reinterpret_cast<char *>(d->workspace);
+    if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY) {
+        c->xyz4 = reinterpret_cast<double4 *>(ws + WS_HEADER);
+        c->recs = ws + WS_HEADER + (d->elem == STOKESFO_HEX8 ? xyz4_bytes<Hex8>(d->num_nodes) : xyz4_bytes<Wedge6>(d->num_nodes));
+    } else {
+        c->xyz4 = nullptr;
+        c->recs = ws + WS_HEADER;
+    }
     int st = (d->elem == STOKESFO_HEX8) ? create_impl<Hex8>(c) : create_impl<Wedge6>(c);
     if (st) {
         delete c;
@@ -252,8 +312,20 @@ int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure) {
     if (work == 0) return STOKESFO_OK;
     const int bs = 256;
     const unsigned g = (unsigned)((work + bs - 1) / bs);
-    if (c->N == 8) geometry_export_kernel<Hex8><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
-    else geometry_export_kernel<Wedge6><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
+    if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY) {  // recompute with the same device code, canonical layout
+        if (c->N == 8)
+            geometry_kernel<Hex8, GEO_CANON><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.num_nodes, c->d.conn,
+                                                                      c->d.coords, nullptr, 0.0, nullptr, grad_bf,
+                                                                      w_measure, c->err);
+        else
+            geometry_kernel<Wedge6, GEO_CANON><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.num_nodes, c->d.conn,
+                                                                        c->d.coords, nullptr, 0.0, nullptr, grad_bf,
+                                                                        w_measure, c->err);
+    } else if (c->N == 8) {
+        geometry_export_kernel<Hex8><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
+    } else {
+        geometry_export_kernel<Wedge6><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
+    }
     return cuda_status();
 }
 

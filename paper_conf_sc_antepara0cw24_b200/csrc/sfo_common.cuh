@@ -54,6 +54,8 @@ struct Rec {
     static constexpr int WM_OFF = KC_OFF + TC * 8;
     static constexpr int G_OFF = WM_OFF + Q * TC * 8;
     static constexpr int BYTES = (int)round_up(G_OFF + N * Q * 3 * TC * 8, 128);
+    // light record (on-the-fly geometry mode): conn + k_c only
+    static constexpr int LIGHT_BYTES = (int)round_up(KC_OFF + TC * 8, 128);
     // index helpers (in elements of the respective type)
     __host__ __device__ static constexpr int conn(int n, int c) { return n * TC + E::cswz(c, n); }
     __host__ __device__ static constexpr int wm(int q, int c) { return q * TC + c; }

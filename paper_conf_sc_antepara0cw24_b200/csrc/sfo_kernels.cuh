@@ -85,33 +85,42 @@ __host__ __device__ __forceinline__ int gidx(int n, int q, int d, int c) {
 
 // ---------------------------------------------------------------------------
 // G1: geometry precompute.  Thread <-> (cell, qp).
+//   OUT = GEO_RECORDS: full per-tile records (stored-geometry mode, at create)
+//   OUT = GEO_CANON:   canonical grad_bf [C][N][Q][3], w_measure [C][Q] (export)
+//   OUT = GEO_CHECK:   only the det J > 0 / conn range checks
 // ---------------------------------------------------------------------------
-template <class E>
+enum { GEO_RECORDS = 0, GEO_CANON = 1, GEO_CHECK = 2 };
+
+template <class E, int OUT>
 __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *__restrict__ conn,
                                 const double *__restrict__ coords, const double *__restrict__ kc_in, double kscal,
-                                char *__restrict__ recs, int *__restrict__ err) {
+                                char *__restrict__ recs, double *__restrict__ grad_bf, double *__restrict__ w_measure,
+                                int *__restrict__ err) {
     using R = Rec<E>;
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     const int64_t ntiles = (ncells + TC - 1) / TC;
     const int64_t gid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (gid >= ntiles * TC * Q) return;
+    const int64_t nwork = (OUT == GEO_RECORDS ? ntiles * TC : ncells) * Q;
+    if (gid >= nwork) return;
     const int q = (int)(gid % Q);
     const int64_t cell = gid / Q;
     const int64_t tile = cell / TC;
     const int c = (int)(cell % TC);
-    char *rec = recs + tile * (int64_t)R::BYTES;
+    char *rec = OUT == GEO_RECORDS ? recs + tile * (int64_t)R::BYTES : nullptr;
     int32_t *rconn = reinterpret_cast<int32_t *>(rec + R::CONN_OFF);
     double *rkc = reinterpret_cast<double *>(rec + R::KC_OFF);
     double *rwm = reinterpret_cast<double *>(rec + R::WM_OFF);
     double *rg = reinterpret_cast<double *>(rec + R::G_OFF);
     if (cell >= ncells) {  // padding cells of the ragged last tile: zero record
-        if (q == 0) {
-            for (int n = 0; n < N; ++n) rconn[R::conn(n, c)] = 0;
-            rkc[c] = 0.0;
+        if (OUT == GEO_RECORDS) {
+            if (q == 0) {
+                for (int n = 0; n < N; ++n) rconn[R::conn(n, c)] = 0;
+                rkc[c] = 0.0;
+            }
+            rwm[R::wm(q, c)] = 0.0;
+            for (int n = 0; n < N; ++n)
+                for (int d = 0; d < 3; ++d) rg[gidx<E>(n, q, d, c)] = 0.0;
         }
-        rwm[R::wm(q, c)] = 0.0;
-        for (int n = 0; n < N; ++n)
-            for (int d = 0; d < 3; ++d) rg[gidx<E>(n, q, d, c)] = 0.0;
         return;
     }
     int32_t nid[N];
@@ -124,7 +133,7 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
         }
     }
     if (bad_conn) atomicOr(err, ERR_CONN);
-    if (q == 0) {
+    if (OUT == GEO_RECORDS && q == 0) {
         for (int n = 0; n < N; ++n) rconn[R::conn(n, c)] = nid[n];
         rkc[c] = kc_in ? kc_in[cell] : kscal;
     }
@@ -159,14 +168,18 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
     cof[2][2] = J[0][0] * J[1][1] - J[0][1] * J[1][0];
     const double det = J[0][0] * cof[0][0] + J[0][1] * cof[0][1] + J[0][2] * cof[0][2];
     if (!(det > 0.0)) atomicOr(err, ERR_DETJ);
+    if (OUT == GEO_CHECK) return;
     const double idet = 1.0 / det;
 #pragma unroll
     for (int n = 0; n < N; ++n)
 #pragma unroll
-        for (int r = 0; r < 3; ++r)
-            rg[gidx<E>(n, q, r, c)] =
-                (cof[r][0] * dphi[n][0] + cof[r][1] * dphi[n][1] + cof[r][2] * dphi[n][2]) * idet;
-    rwm[R::wm(q, c)] = wq * det;
+        for (int r = 0; r < 3; ++r) {
+            const double g = (cof[r][0] * dphi[n][0] + cof[r][1] * dphi[n][1] + cof[r][2] * dphi[n][2]) * idet;
+            if (OUT == GEO_RECORDS) rg[gidx<E>(n, q, r, c)] = g;
+            else if (grad_bf) grad_bf[((cell * N + n) * Q + q) * 3 + r] = g;
+        }
+    if (OUT == GEO_RECORDS) rwm[R::wm(q, c)] = wq * det;
+    else if (w_measure) w_measure[cell * Q + q] = wq * det;
 }
 
 // Export records -> canonical grad_bf [C][N][Q][3], w_measure [C][Q].
@@ -204,7 +217,9 @@ __global__ void gather_kernel(int64_t ncells, const int32_t *__restrict__ conn, 
 // G3/G4: fused evaluation.
 // ---------------------------------------------------------------------------
 struct EvalArgs {
-    const char *recs;
+    const char *recs;         // per-tile records (full: stored geometry; light: conn + k_c)
+    const double4 *xyz4;      // on-the-fly geometry: node coordinates (x, y, z, 0)
+    int *err;                 // sticky device error flag
     int64_t ntiles, ncells;
     const double *U;          // [nodes][2]
     const double *surface;    // [nodes] or null
@@ -218,7 +233,159 @@ struct EvalArgs {
 
 constexpr int NQS = 9;  // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 beta12, wmu2, gamma, wf0, wf1
 
-// Shared memory: two stage buffers + per-QP scalars + 2 mbarriers.
+// ---- shared device pieces ---------------------------------------------------
+
+// Per-QP tail of phase 1: given Ugrad and grad s_h at (cell c, qp q), evaluate
+// the effective strain rate (Z2), Glen viscosity at n = 3 (Z1, Z3) and the
+// per-QP scalars phase 2 needs.  beta = B g so that sigma = 2 mu beta gives
+// strs00..strs12 of Fig. 2.
+template <class E>
+__device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, int q, int nvalid, int64_t cell0,
+                                        bool have_s, double kc, double wm, double ux, double uy, double uz, double vx,
+                                        double vy, double vz, double gs0, double gs1) {
+    constexpr int Q = E::Q, TC = E::TC;
+    constexpr double P_EXP = -1.0 / 3.0;  // (1 - n) / (2 n) at n = 3
+    const double uyvx = uy + vx;
+    const double e2 = ux * ux + vy * vy + ux * vy + 0.25 * uyvx * uyvx + 0.25 * uz * uz + 0.25 * vz * vz;
+    const double r = rcbrt(e2 + a.delta);  // (e2 + delta)^(-1/3)
+    const double mu = kc * r;
+    const double wmu2 = 2.0 * wm * mu;
+    double *qq = qs + q * TC + c;
+    qq[0 * Q * TC] = 2.0 * ux + vy;   // beta_(0,0) = strs00 / (2 mu)
+    qq[1 * Q * TC] = 0.5 * uyvx;      // beta_(0,1) = beta_(1,0) = strs01 / (2 mu)
+    qq[2 * Q * TC] = 0.5 * uz;        // beta_(0,2) = strs02 / (2 mu)
+    qq[3 * Q * TC] = ux + 2.0 * vy;   // beta_(1,1) = strs11 / (2 mu)
+    qq[4 * Q * TC] = 0.5 * vz;        // beta_(1,2) = strs12 / (2 mu)
+    qq[5 * Q * TC] = wmu2;
+    // gamma = wM 2 mu p / (e2 + delta) = wmu2 p r^3  (d mu / d e2, reading Z5)
+    qq[6 * Q * TC] = wmu2 * P_EXP * (r * r * r);
+    double wf0 = 0.0, wf1 = 0.0;
+    if (a.force_qp) {
+        if (c < nvalid) {
+            const double2 f = *reinterpret_cast<const double2 *>(a.force_qp + ((cell0 + c) * Q + q) * 2);
+            wf0 = wm * f.x;
+            wf1 = wm * f.y;
+        }
+    } else if (have_s) {
+        wf0 = wm * a.rho_g * gs0;
+        wf1 = wm * a.rho_g * gs1;
+    }
+    qq[7 * Q * TC] = wf0;
+    qq[8 * Q * TC] = wf1;
+    if (a.mu_qp && c < nvalid) a.mu_qp[(cell0 + c) * Q + q] = mu;
+}
+
+// Phase 2, thread <-> (cell c2, node i): residual rows (i,0), (i,1) and, for
+// JAC, the 2x2 tangent blocks J[(i,.),(j_k,.)], j_k = (i+k) mod N, k = 0..N/2,
+// accumulated over QPs in registers (the paper's local accumulation).
+// J_q[(i,a),(j,b)] = sum_e M_ab[e] G_j[e],
+// M_ab = wM 2 mu (B-block (a,b) applied to G_i) + gamma h_(i,a) beta_(b,.)
+// is the exact forward derivative of the chain (seed-sparse Sacado lanes).
+// pf() is called once at q = Q/2 (prefetch hook).
+template <class E, bool JAC, class PF>
+__device__ __forceinline__ void node_accumulate(const double *rg, const double *qs, int c2, int i, const double *bfi,
+                                                double &R0, double &R1, double (&Jb)[E::N / 2 + 1][2][2], PF pf) {
+    constexpr int N = E::N, Q = E::Q, TC = E::TC, K = N / 2;
+    R0 = 0.0;
+    R1 = 0.0;
+    if (JAC) {
+#pragma unroll
+        for (int k = 0; k <= K; ++k) Jb[k][0][0] = Jb[k][0][1] = Jb[k][1][0] = Jb[k][1][1] = 0.0;
+    }
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+        if (q == Q / 2) pf();
+        const double *qq = qs + q * TC + c2;
+        const double b00 = qq[0 * Q * TC], b01 = qq[1 * Q * TC], b02 = qq[2 * Q * TC];
+        const double b11 = qq[3 * Q * TC], b12 = qq[4 * Q * TC];
+        const double b10 = b01;
+        const double wmu2 = qq[5 * Q * TC];
+        const double wf0 = qq[7 * Q * TC], wf1 = qq[8 * Q * TC];
+        const double gi0 = rg[gidx<E>(i, q, 0, c2)];
+        const double gi1 = rg[gidx<E>(i, q, 1, c2)];
+        const double gi2 = rg[gidx<E>(i, q, 2, c2)];
+        // h_(i,a) = sum_d G_i[d] beta_(a,d);  residual row (i,a) += wmu2 h + wf_a BF_i
+        const double h0 = fma(gi2, b02, fma(gi1, b01, gi0 * b00));
+        const double h1 = fma(gi2, b12, fma(gi1, b11, gi0 * b10));
+        R0 = fma(wf0, bfi[q], fma(wmu2, h0, R0));
+        R1 = fma(wf1, bfi[q], fma(wmu2, h1, R1));
+        if (JAC) {
+            const double gam = qq[6 * Q * TC];
+            const double gh0 = gam * h0, gh1 = gam * h1;
+            const double w0 = wmu2 * gi0, w1 = wmu2 * gi1, w2 = wmu2 * gi2;
+            const double m00x = fma(2.0, w0, gh0 * b00), m00y = fma(0.5, w1, gh0 * b01),
+                         m00z = fma(0.5, w2, gh0 * b02);
+            const double m01x = fma(0.5, w1, gh0 * b10), m01y = fma(gh0, b11, w0), m01z = gh0 * b12;
+            const double m10x = fma(gh1, b00, w1), m10y = fma(0.5, w0, gh1 * b01), m10z = gh1 * b02;
+            const double m11x = fma(0.5, w0, gh1 * b10), m11y = fma(2.0, w1, gh1 * b11),
+                         m11z = fma(0.5, w2, gh1 * b12);
+#pragma unroll
+            for (int k = 0; k <= K; ++k) {
+                const int j = (i + k) % N;
+                double gj0, gj1, gj2;
+                if (k == 0) {
+                    gj0 = gi0; gj1 = gi1; gj2 = gi2;
+                } else {
+                    gj0 = rg[gidx<E>(j, q, 0, c2)];
+                    gj1 = rg[gidx<E>(j, q, 1, c2)];
+                    gj2 = rg[gidx<E>(j, q, 2, c2)];
+                }
+                // explicit 3-deep DFMA chains into the accumulators (no DMUL/DADD)
+                Jb[k][0][0] = fma(m00z, gj2, fma(m00y, gj1, fma(m00x, gj0, Jb[k][0][0])));
+                Jb[k][0][1] = fma(m01z, gj2, fma(m01y, gj1, fma(m01x, gj0, Jb[k][0][1])));
+                Jb[k][1][0] = fma(m10z, gj2, fma(m10y, gj1, fma(m10x, gj0, Jb[k][1][0])));
+                Jb[k][1][1] = fma(m11z, gj2, fma(m11y, gj1, fma(m11x, gj0, Jb[k][1][1])));
+            }
+        }
+    }
+}
+
+// Write J[c2] rows (2i, 2i+1) into a staging image of the global layout:
+// direct blocks (i, i+k), k = 0..K, and transposed blocks (i+k, i) for
+// 0 < k < K (J is symmetric: the Hessian of the quadrature energy).  Rotating
+// j with i keeps the 16-byte stores of a quarter-warp in distinct bank groups.
+template <class E>
+__device__ __forceinline__ void stage_J(double *base, int c2, int i, const double (&Jb)[E::N / 2 + 1][2][2]) {
+    constexpr int N = E::N, K = N / 2, LD = 2 * N;
+    double *Jc = base + c2 * E::JPITCH;
+#pragma unroll
+    for (int k = 0; k <= K; ++k) {
+        const int j = (i + k) % N;
+        *reinterpret_cast<double2 *>(Jc + (2 * i + 0) * LD + 2 * j) = make_double2(Jb[k][0][0], Jb[k][0][1]);
+        *reinterpret_cast<double2 *>(Jc + (2 * i + 1) * LD + 2 * j) = make_double2(Jb[k][1][0], Jb[k][1][1]);
+        if (k > 0 && k < K) {
+            *reinterpret_cast<double2 *>(Jc + (2 * j + 0) * LD + 2 * i) = make_double2(Jb[k][0][0], Jb[k][1][0]);
+            *reinterpret_cast<double2 *>(Jc + (2 * j + 1) * LD + 2 * i) = make_double2(Jb[k][0][1], Jb[k][1][1]);
+        }
+    }
+}
+
+// One thread issues the TMA bulk store(s) of the staged J image of a tile.
+template <class E>
+__device__ __forceinline__ void store_J(double *J_cell, int64_t cell0, int nvalid, const char *stage, uint64_t pol) {
+    constexpr int NN = 4 * E::N * E::N;
+    if (E::JPITCH == NN) {
+        bulk_s2g(J_cell + cell0 * NN, stage, (uint32_t)(nvalid * NN * 8), pol);
+    } else {
+        for (int c = 0; c < nvalid; ++c)
+            bulk_s2g(J_cell + (cell0 + c) * NN, stage + c * E::JPITCH * 8, (uint32_t)(NN * 8), pol);
+    }
+    bulk_commit();
+}
+
+template <class E>
+__device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
+#pragma unroll
+    for (int q = 0; q < E::Q; ++q) {
+        double x, y, z, w, dx, dy, dz;
+        qp_coords<E>(q, x, y, z, w);
+        basis<E>(i, x, y, z, bfi[q], dx, dy, dz);
+    }
+}
+
+// ---- G3/G4 with stored geometry (the §8(a2) precompute streamed per tile) ----
+
+// Shared memory: NSTAGE stage buffers + per-QP scalars + mbarriers.
 // A stage buffer holds [record | gathered U (double2 [N][TC]) | s ([N][TC])];
 // once a tile's phase 2 has consumed its record, the same buffer stages the
 // tile's element Jacobians for the TMA bulk store (JAC).
@@ -291,17 +458,10 @@ __global__ void __launch_bounds__(E::TC *E::N, (min_blocks<E, JAC, NSTAGE>())) e
         issue_gather<E>(smem, a.U, a.surface, have_s);
     }
 
-    // phase-2 identity: thread <-> (cell c2, node i)
     const int c2 = E::NODE_MAJOR_P2 ? t % TC : t / N;
     const int i = E::NODE_MAJOR_P2 ? t / TC : t % N;
     double bfi[Q];
-#pragma unroll
-    for (int q = 0; q < Q; ++q) {
-        double x, y, z, w, dx, dy, dz;
-        qp_coords<E>(q, x, y, z, w);
-        basis<E>(i, x, y, z, bfi[q], dx, dy, dz);
-    }
-    constexpr double P_EXP = -1.0 / 3.0;  // (1 - n) / (2 n) at n = 3
+    basis_row<E>(i, bfi);
 
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
@@ -329,146 +489,38 @@ __global__ void __launch_bounds__(E::TC *E::N, (min_blocks<E, JAC, NSTAGE>())) e
                 const double g1 = rg[gidx<E>(n, q, 1, c)];
                 const double g2 = rg[gidx<E>(n, q, 2, c)];
                 const double2 uv = Us[n * TC + c];
-                ux += uv.x * g0; uy += uv.x * g1; uz += uv.x * g2;
-                vx += uv.y * g0; vy += uv.y * g1; vz += uv.y * g2;
+                ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
+                vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
                 if (have_s) {
                     const double sn = ss[n * TC + c];
-                    gs0 += sn * g0; gs1 += sn * g1;
+                    gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
             }
-            const double uyvx = uy + vx;
-            // effective strain rate^2 (reading Z2) and Glen viscosity, n = 3
-            const double e2 = ux * ux + vy * vy + ux * vy + 0.25 * uyvx * uyvx + 0.25 * uz * uz + 0.25 * vz * vz;
-            const double r = rcbrt(e2 + a.delta);  // (e2 + delta)^(-1/3)
-            const double mu = rkc[c] * r;
-            const double wm = rwm[R::wm(q, c)];
-            const double wmu2 = 2.0 * wm * mu;
-            // beta = B g: sigma = 2 mu beta reproduces strs00..strs12 of Fig. 2
-            double *qq = qs + q * TC + c;
-            qq[0 * Q * TC] = 2.0 * ux + vy;   // beta_(0,0) = strs00 / (2 mu)
-            qq[1 * Q * TC] = 0.5 * uyvx;      // beta_(0,1) = beta_(1,0) = strs01 / (2 mu)
-            qq[2 * Q * TC] = 0.5 * uz;        // beta_(0,2) = strs02 / (2 mu)
-            qq[3 * Q * TC] = ux + 2.0 * vy;   // beta_(1,1) = strs11 / (2 mu)
-            qq[4 * Q * TC] = 0.5 * vz;        // beta_(1,2) = strs12 / (2 mu)
-            qq[5 * Q * TC] = wmu2;
-            // gamma = wM 2 mu p / (e2 + delta) = wmu2 p r^3  (d mu / d e2 chain, reading Z5)
-            qq[6 * Q * TC] = wmu2 * P_EXP * (r * r * r);
-            double wf0 = 0.0, wf1 = 0.0;
-            if (a.force_qp) {
-                if (c < nvalid) {
-                    const double2 f = *reinterpret_cast<const double2 *>(a.force_qp + ((cell0 + c) * Q + q) * 2);
-                    wf0 = wm * f.x;
-                    wf1 = wm * f.y;
-                }
-            } else if (have_s) {
-                wf0 = wm * a.rho_g * gs0;
-                wf1 = wm * a.rho_g * gs1;
-            }
-            qq[7 * Q * TC] = wf0;
-            qq[8 * Q * TC] = wf1;
-            if (a.mu_qp && c < nvalid) a.mu_qp[(cell0 + c) * Q + q] = mu;
+            qp_tail<E>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy, vz, gs0,
+                       gs1);
         }
         __syncthreads();
 
-        // ---- phase 2: per-node accumulation (thread <-> (cell c2, node i)) ----
+        // ---- phase 2 (+ prefetch of the next tile's gather at q = Q/2) ----
         const int32_t gnode = rconn[R::conn(i, c2)];
-        double R0 = 0.0, R1 = 0.0;
-        constexpr int K = N / 2;            // symmetric block scheme: blocks (i, i+k), k = 0..K
-        double Jb[JAC ? K + 1 : 1][2][2];   // Jb[k][a][b] = J[(i,a), (j_k,b)], j_k = (i+k) mod N
-        if (JAC) {
-#pragma unroll
-            for (int k = 0; k <= K; ++k) Jb[k][0][0] = Jb[k][0][1] = Jb[k][1][0] = Jb[k][1][1] = 0.0;
-        }
-#pragma unroll
-        for (int q = 0; q < Q; ++q) {
-            if (q == Q / 2) {
-                // prefetch: gather U, s of the next tile (its record was issued
-                // NSTAGE-1 tiles ago) while the rest of this tile computes
-                const int64_t nt = tile + gridDim.x;
-                if (nt < a.ntiles) {
-                    const int ns = (it + 1) % NSTAGE;
-                    mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NSTAGE) & 1));
-                    issue_gather<E>(smem + ns * S::STAGE, a.U, a.surface, have_s);
-                }
+        double R0, R1;
+        double Jb[N / 2 + 1][2][2];
+        node_accumulate<E, JAC>(rg, qs, c2, i, bfi, R0, R1, Jb, [&]() {
+            const int64_t nt = tile + gridDim.x;
+            if (nt < a.ntiles) {
+                const int ns = (it + 1) % NSTAGE;
+                mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NSTAGE) & 1));
+                issue_gather<E>(smem + ns * S::STAGE, a.U, a.surface, have_s);
             }
-            const double *qq = qs + q * TC + c2;
-            const double b00 = qq[0 * Q * TC], b01 = qq[1 * Q * TC], b02 = qq[2 * Q * TC];
-            const double b11 = qq[3 * Q * TC], b12 = qq[4 * Q * TC];
-            const double b10 = b01;
-            const double wmu2 = qq[5 * Q * TC];
-            const double wf0 = qq[7 * Q * TC], wf1 = qq[8 * Q * TC];
-            const double gi0 = rg[gidx<E>(i, q, 0, c2)];
-            const double gi1 = rg[gidx<E>(i, q, 1, c2)];
-            const double gi2 = rg[gidx<E>(i, q, 2, c2)];
-            // h_(i,a) = sum_d G_i[d] beta_(a,d);  residual row (i,a) = wmu2 h + wf_a BF_i
-            const double h0 = fma(gi2, b02, fma(gi1, b01, gi0 * b00));
-            const double h1 = fma(gi2, b12, fma(gi1, b11, gi0 * b10));
-            R0 = fma(wf0, bfi[q], fma(wmu2, h0, R0));
-            R1 = fma(wf1, bfi[q], fma(wmu2, h1, R1));
-            if (JAC) {
-                // J_q[(i,a),(j,b)] = sum_e M_ab[e] G_j[e] with
-                // M_ab = wmu2 * (B-block (a,b) applied to G_i) + gamma h_(i,a) beta_(b,.)
-                const double gam = qq[6 * Q * TC];
-                const double gh0 = gam * h0, gh1 = gam * h1;
-                const double w0 = wmu2 * gi0, w1 = wmu2 * gi1, w2 = wmu2 * gi2;
-                const double m00x = fma(2.0, w0, gh0 * b00), m00y = fma(0.5, w1, gh0 * b01),
-                             m00z = fma(0.5, w2, gh0 * b02);
-                const double m01x = fma(0.5, w1, gh0 * b10), m01y = fma(gh0, b11, w0), m01z = gh0 * b12;
-                const double m10x = fma(gh1, b00, w1), m10y = fma(0.5, w0, gh1 * b01), m10z = gh1 * b02;
-                const double m11x = fma(0.5, w0, gh1 * b10), m11y = fma(2.0, w1, gh1 * b11),
-                             m11z = fma(0.5, w2, gh1 * b12);
-#pragma unroll
-                for (int k = 0; k <= K; ++k) {
-                    const int j = (i + k) % N;
-                    double gj0, gj1, gj2;
-                    if (k == 0) {
-                        gj0 = gi0; gj1 = gi1; gj2 = gi2;
-                    } else {
-                        gj0 = rg[gidx<E>(j, q, 0, c2)];
-                        gj1 = rg[gidx<E>(j, q, 1, c2)];
-                        gj2 = rg[gidx<E>(j, q, 2, c2)];
-                    }
-                    // explicit 3-deep DFMA chains into the accumulators (no DMUL/DADD)
-                    Jb[k][0][0] = fma(m00z, gj2, fma(m00y, gj1, fma(m00x, gj0, Jb[k][0][0])));
-                    Jb[k][0][1] = fma(m01z, gj2, fma(m01y, gj1, fma(m01x, gj0, Jb[k][0][1])));
-                    Jb[k][1][0] = fma(m10z, gj2, fma(m10y, gj1, fma(m10x, gj0, Jb[k][1][0])));
-                    Jb[k][1][1] = fma(m11z, gj2, fma(m11y, gj1, fma(m11x, gj0, Jb[k][1][1])));
-                }
-            }
-        }
-        const bool valid = c2 < nvalid;
-        const int64_t cell = cell0 + c2;
+        });
         __syncthreads();  // everyone is done with this stage's record and qs
 
         if (JAC) {
-            // Stage J[c2] rows (2i, 2i+1) into this stage buffer: direct blocks
-            // (i, i+k), k = 0..K, and transposed blocks (i+k, i) for 0 < k < K
-            // (J is symmetric: the Hessian of the quadrature energy).
-            double *Jc = reinterpret_cast<double *>(stage) + c2 * E::JPITCH;
-            constexpr int LD = 2 * N;
-#pragma unroll
-            for (int k = 0; k <= K; ++k) {
-                const int j = (i + k) % N;
-                *reinterpret_cast<double2 *>(Jc + (2 * i + 0) * LD + 2 * j) = make_double2(Jb[k][0][0], Jb[k][0][1]);
-                *reinterpret_cast<double2 *>(Jc + (2 * i + 1) * LD + 2 * j) = make_double2(Jb[k][1][0], Jb[k][1][1]);
-                if (k > 0 && k < K) {
-                    *reinterpret_cast<double2 *>(Jc + (2 * j + 0) * LD + 2 * i) =
-                        make_double2(Jb[k][0][0], Jb[k][1][0]);
-                    *reinterpret_cast<double2 *>(Jc + (2 * j + 1) * LD + 2 * i) =
-                        make_double2(Jb[k][0][1], Jb[k][1][1]);
-                }
-            }
+            stage_J<E>(reinterpret_cast<double *>(stage), c2, i, Jb);
             fence_proxy_async_smem();
             __syncthreads();
             if (t == 0) {
-                if (E::JPITCH == 4 * N * N) {
-                    bulk_s2g(a.J_cell + cell0 * (4 * N * N), stage, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
-                } else {
-                    for (int c = 0; c < nvalid; ++c)
-                        bulk_s2g(a.J_cell + (cell0 + c) * (4 * N * N), stage + c * E::JPITCH * 8,
-                                 (uint32_t)(4 * N * N * 8), pol_stream);
-                }
-                bulk_commit();
+                store_J<E>(a.J_cell, cell0, nvalid, stage, pol_stream);
                 bulk_wait_read0();  // staging read done -> the buffer may take the next record
             }
         }
@@ -479,15 +531,247 @@ __global__ void __launch_bounds__(E::TC *E::N, (min_blocks<E, JAC, NSTAGE>())) e
                 bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
             }
         }
-        if (valid) {
+        if (c2 < nvalid) {
             if (a.R) {
                 atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
                 atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
             }
-            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + (cell * N + i) * 2) = make_double2(R0, R1);
+            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c2) * N + i) * 2) = make_double2(R0, R1);
         }
     }
     if (JAC && t == 0) bulk_wait0();
+}
+
+// ---- G3/G4 with on-the-fly geometry ------------------------------------------
+// Same evaluation, but GradBF and wM are recomputed per tile from the gathered
+// node coordinates instead of being streamed (1,640 -> 40 streamed B/cell for
+// hex8): B200's FP64 rate per HBM byte makes recomputation cheaper than
+// streaming.  Light records (conn + k_c, 640 B per hex8 tile) ride a 4-deep TMA
+// ring; U, s and the coordinates are gathered with cp.async one tile ahead.
+
+constexpr int NLIGHT = 4;
+
+template <class E, bool JAC>
+struct OtfSmem {
+    static constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    static constexpr int LREC = Rec<E>::LIGHT_BYTES;
+    static constexpr int OFF_L = 0;                                         // NLIGHT light records
+    static constexpr int OFF_IN = OFF_L + NLIGHT * LREC;                    // 2 gathered-input buffers
+    static constexpr int IN_U = 0, IN_XY = N * TC * 16, IN_ZW = 2 * N * TC * 16, IN_S = 3 * N * TC * 16;
+    static constexpr int IN_BYTES = (int)round_up(IN_S + N * TC * 8, 128);
+    static constexpr int OFF_DPHI = OFF_IN + 2 * IN_BYTES;                  // double [Q][N][3]
+    static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * N * 3 * 8, 128);  // GradBF [N][Q][3][TC] (swizzled)
+    static constexpr int OFF_QS = OFF_G + N * Q * 3 * TC * 8;               // double [NQS][Q][TC]
+    static constexpr int G_QS_BYTES = OFF_QS + NQS * Q * TC * 8 - OFF_G;
+    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;            // J staging overlays G + qs
+    static_assert(J_BYTES <= G_QS_BYTES, "J staging must fit over G + qs");
+    static constexpr int OFF_BAR = OFF_QS + NQS * Q * TC * 8;
+    static constexpr int BYTES = OFF_BAR + NLIGHT * 8;
+};
+
+template <class E>
+__device__ __forceinline__ void issue_gather_otf(char *in, const int32_t *lconn, const double *U,
+                                                 const double4 *xyz4, const double *surface, bool have_s) {
+    using S = OtfSmem<E, false>;
+    const int t = threadIdx.x;
+    const int c = t % E::TC, n = t / E::TC;
+    const int32_t g = lconn[Rec<E>::conn(n, c)];
+    const int o = (n * E::TC + c) * 16;
+    cp_async16(in + S::IN_U + o, U + 2 * (int64_t)g);
+    cp_async16(in + S::IN_XY + o, reinterpret_cast<const double *>(xyz4 + g));
+    cp_async16(in + S::IN_ZW + o, reinterpret_cast<const double *>(xyz4 + g) + 2);
+    if (have_s) cp_async8(in + S::IN_S + (n * E::TC + c) * 8, surface + g);
+    cp_async_commit();
+}
+
+template <class E, bool JAC>
+__global__ void __launch_bounds__(E::TC *E::N, (E::N == 8 ? 3 : 2)) eval_otf_kernel(EvalArgs a) {
+    constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    static_assert(N == Q, "thread mappings assume N == Q");
+    using R = Rec<E>;
+    using S = OtfSmem<E, JAC>;
+    static_assert(S::OFF_IN == OtfSmem<E, false>::OFF_IN && S::IN_BYTES == OtfSmem<E, false>::IN_BYTES, "layout");
+    extern __shared__ __align__(128) char smem[];
+    double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
+    double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
+    double *dphi = reinterpret_cast<double *>(smem + S::OFF_DPHI);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
+    const int t = threadIdx.x;
+    const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
+
+    // reference gradients d phi_n / d xi at every QP (shared table)
+    for (int e = t; e < Q * N; e += blockDim.x) {
+        const int q = e / N, n = e % N;
+        double x, y, z, w, phi;
+        qp_coords<E>(q, x, y, z, w);
+        basis<E>(n, x, y, z, phi, dphi[e * 3 + 0], dphi[e * 3 + 1], dphi[e * 3 + 2]);
+    }
+    uint64_t pol_stream = 0;
+    if (t == 0) {
+        pol_stream = policy_evict_first();
+        for (int s = 0; s < NLIGHT; ++s) mbar_init(&bar[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (t == 0) {
+        for (int s = 0; s < NLIGHT; ++s) {
+            const int64_t tile = blockIdx.x + (int64_t)s * gridDim.x;
+            if (tile < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[s], S::LREC);
+                bulk_g2s(smem + S::OFF_L + s * S::LREC, a.recs + tile * (int64_t)S::LREC, S::LREC, &bar[s],
+                         pol_stream);
+            }
+        }
+    }
+    if ((int64_t)blockIdx.x < a.ntiles) {
+        mbar_wait(&bar[0], 0);
+        issue_gather_otf<E>(smem + S::OFF_IN, reinterpret_cast<const int32_t *>(smem + S::OFF_L), a.U, a.xyz4,
+                            a.surface, have_s);
+    }
+    double wq;
+    {
+        double x, y, z;
+        qp_coords<E>(t / TC, x, y, z, wq);
+    }
+
+    const int c2 = E::NODE_MAJOR_P2 ? t % TC : t / N;
+    const int i = E::NODE_MAJOR_P2 ? t / TC : t % N;
+    double bfi[Q];
+    basis_row<E>(i, bfi);
+
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+        const int sl = it % NLIGHT;
+        const char *lrec = smem + S::OFF_L + sl * S::LREC;
+        const int32_t *lconn = reinterpret_cast<const int32_t *>(lrec + R::CONN_OFF);
+        const double *lkc = reinterpret_cast<const double *>(lrec + R::KC_OFF);
+        const char *in = smem + S::OFF_IN + (it & 1) * S::IN_BYTES;
+        const double2 *Us = reinterpret_cast<const double2 *>(in + S::IN_U);
+        const double2 *XY = reinterpret_cast<const double2 *>(in + S::IN_XY);
+        const double2 *ZW = reinterpret_cast<const double2 *>(in + S::IN_ZW);
+        const double *ss = reinterpret_cast<const double *>(in + S::IN_S);
+        const int64_t cell0 = tile * TC;
+        const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
+
+        cp_async_wait_all();
+        if (JAC && t == 0) bulk_wait_read0();  // previous tile's J staging (over G + qs) has been read
+        __syncthreads();
+
+        // ---- phase 1 (thread <-> (cell, qp)): geometry, GradBF -> smem, then Ugrad etc. ----
+        {
+            const int c = t % TC, q = t / TC;
+            const double *dq = dphi + q * N * 3;
+            double J00 = 0, J01 = 0, J02 = 0, J10 = 0, J11 = 0, J12 = 0, J20 = 0, J21 = 0, J22 = 0;
+#pragma unroll
+            for (int n = 0; n < N; ++n) {
+                const double2 xy = XY[n * TC + c];
+                const double z = ZW[n * TC + c].x;
+                const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
+                J00 = fma(xy.x, d0, J00); J01 = fma(xy.x, d1, J01); J02 = fma(xy.x, d2, J02);
+                J10 = fma(xy.y, d0, J10); J11 = fma(xy.y, d1, J11); J12 = fma(xy.y, d2, J12);
+                J20 = fma(z, d0, J20); J21 = fma(z, d1, J21); J22 = fma(z, d2, J22);
+            }
+            // cofactors: (J^-T)[r][s] = cof[r][s] / det
+            const double c00 = J11 * J22 - J12 * J21, c01 = J12 * J20 - J10 * J22, c02 = J10 * J21 - J11 * J20;
+            const double c10 = J02 * J21 - J01 * J22, c11 = J00 * J22 - J02 * J20, c12 = J01 * J20 - J00 * J21;
+            const double c20 = J01 * J12 - J02 * J11, c21 = J02 * J10 - J00 * J12, c22 = J00 * J11 - J01 * J10;
+            const double det = J00 * c00 + J01 * c01 + J02 * c02;
+            if (!(det > 0.0) && c < nvalid) atomicOr(a.err, ERR_DETJ);
+            const double id = 1.0 / det;
+            double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+#pragma unroll
+            for (int n = 0; n < N; ++n) {
+                const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
+                const double g0 = fma(c00, d0, fma(c01, d1, c02 * d2)) * id;
+                const double g1 = fma(c10, d0, fma(c11, d1, c12 * d2)) * id;
+                const double g2 = fma(c20, d0, fma(c21, d1, c22 * d2)) * id;
+                rg[gidx<E>(n, q, 0, c)] = g0;
+                rg[gidx<E>(n, q, 1, c)] = g1;
+                rg[gidx<E>(n, q, 2, c)] = g2;
+                const double2 uv = Us[n * TC + c];
+                ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
+                vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
+                if (have_s) {
+                    const double sn = ss[n * TC + c];
+                    gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
+                }
+            }
+            qp_tail<E>(a, qs, c, q, nvalid, cell0, have_s, lkc[c], wq * det, ux, uy, uz, vx, vy, vz, gs0, gs1);
+        }
+        __syncthreads();
+
+        // ---- phase 2 (+ prefetch of the next tile's gather at q = Q/2) ----
+        const int32_t gnode = lconn[R::conn(i, c2)];
+        double R0, R1;
+        double Jb[N / 2 + 1][2][2];
+        node_accumulate<E, JAC>(rg, qs, c2, i, bfi, R0, R1, Jb, [&]() {
+            const int64_t nt = tile + gridDim.x;
+            if (nt < a.ntiles) {
+                const int ns = (it + 1) % NLIGHT;
+                mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NLIGHT) & 1));
+                issue_gather_otf<E>(smem + S::OFF_IN + ((it + 1) & 1) * S::IN_BYTES,
+                                    reinterpret_cast<const int32_t *>(smem + S::OFF_L + ns * S::LREC), a.U, a.xyz4,
+                                    a.surface, have_s);
+            }
+        });
+        __syncthreads();  // G, qs and this light record are consumed
+
+        if (t == 0) {  // refill this light-record slot NLIGHT tiles ahead
+            const int64_t nt = tile + (int64_t)NLIGHT * gridDim.x;
+            if (nt < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[sl], S::LREC);
+                bulk_g2s(smem + S::OFF_L + sl * S::LREC, a.recs + nt * (int64_t)S::LREC, S::LREC, &bar[sl],
+                         pol_stream);
+            }
+        }
+        if (JAC) {
+            stage_J<E>(rg, c2, i, Jb);
+            fence_proxy_async_smem();
+            __syncthreads();
+            if (t == 0) store_J<E>(a.J_cell, cell0, nvalid, smem + S::OFF_G, pol_stream);
+        }
+        if (c2 < nvalid) {
+            if (a.R) {
+                atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
+                atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
+            }
+            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c2) * N + i) * 2) = make_double2(R0, R1);
+        }
+    }
+    if (JAC && t == 0) bulk_wait0();
+}
+
+// Setup for the on-the-fly mode: node coordinates as double4, light records
+// (conn + k_c); conn range is checked here, det J at every evaluation.
+__global__ void xyz4_kernel(int64_t nnodes, const double *__restrict__ coords, double4 *__restrict__ xyz4) {
+    const int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (v < nnodes) xyz4[v] = make_double4(coords[3 * v], coords[3 * v + 1], coords[3 * v + 2], 0.0);
+}
+
+template <class E>
+__global__ void light_record_kernel(int64_t ncells, int64_t nnodes, const int32_t *__restrict__ conn,
+                                    const double *__restrict__ kc_in, double kscal, char *__restrict__ recs,
+                                    int *__restrict__ err) {
+    using R = Rec<E>;
+    constexpr int N = E::N, TC = E::TC;
+    const int64_t cell = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t ntiles = (ncells + TC - 1) / TC;
+    if (cell >= ntiles * TC) return;
+    char *rec = recs + (cell / TC) * (int64_t)R::LIGHT_BYTES;
+    const int c = (int)(cell % TC);
+    int32_t *rconn = reinterpret_cast<int32_t *>(rec + R::CONN_OFF);
+    double *rkc = reinterpret_cast<double *>(rec + R::KC_OFF);
+    bool bad = false;
+    for (int n = 0; n < N; ++n) {
+        int32_t g = cell < ncells ? conn[cell * N + n] : 0;
+        if (g < 0 || g >= nnodes) {
+            bad = true;
+            g = 0;
+        }
+        rconn[R::conn(n, c)] = g;
+    }
+    if (bad) atomicOr(err, ERR_CONN);
+    rkc[c] = cell < ncells ? (kc_in ? kc_in[cell] : kscal) : 0.0;
 }
 
 // ---------------------------------------------------------------------------

@@ -20,6 +20,7 @@ NODES = {HEX8: 8, WEDGE6: 6}
 QPS = {HEX8: 8, WEDGE6: 6}
 ABI_VERSION = 1
 
+GEOMETRY = {"stored": 0, "on_the_fly": 1}
 STATUS = {0: "OK", 1: "EINVAL", 2: "EMESH", 3: "ECUDA", 4: "ENOMEM", 5: "EUNSUPPORTED"}
 
 
@@ -40,6 +41,7 @@ class Desc(ctypes.Structure):
         ("rho_g", ctypes.c_double),
         ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_size_t),
         ("stream", ctypes.c_void_p),
+        ("geometry_mode", ctypes.c_int32), ("reserved0", ctypes.c_int32),
     ]
 
 
@@ -124,7 +126,7 @@ class StokesFO:
     """One evaluation context (stokesfo_ctx) over a local mesh on one GPU."""
 
     def __init__(self, elem, conn, coords, surface=None, force_qp=None, flow_factor=None, k=10.77,
-                 glen_n=3.0, delta=1e-10, rho_g=8.927, stream=None):
+                 glen_n=3.0, delta=1e-10, rho_g=8.927, stream=None, geometry="stored"):
         import torch
         self.elem = ELEM[elem] if isinstance(elem, str) else int(elem)
         self.N, self.Q = NODES[self.elem], QPS[self.elem]
@@ -146,6 +148,8 @@ class StokesFO:
         d.surface, d.force_qp, d.flow_factor = _ptr(self.surface), _ptr(self.force_qp), _ptr(self.flow_factor)
         d.k, d.glen_n, d.delta, d.rho_g = k, glen_n, delta, rho_g
         d.stream = ctypes.c_void_p(self.stream.cuda_stream)
+        self.geometry_mode = GEOMETRY[geometry] if isinstance(geometry, str) else int(geometry)
+        d.geometry_mode = self.geometry_mode
         nbytes = ctypes.c_size_t(0)
         _check(_lib().stokesfo_workspace_size(ctypes.byref(d), ctypes.byref(nbytes)), "workspace_size")
         self.workspace = torch.empty(max(int(nbytes.value), 256), dtype=torch.uint8, device=self.device)

@@ -268,6 +268,8 @@ def flow_factor(fp: Footprint, L: int, a0: float = 1e-4) -> np.ndarray:
 CONFIGS = {
     "C1": dict(desc="tiny 16x16 x 5 layers hex8, residual", layers=5, elem="hex8"),
     "C2": dict(desc="tiny 16x16 x 5 layers hex8, residual+Jacobian", layers=5, elem="hex8"),
+    "C3": dict(desc="Greenland-like 1-10 km NVB footprint x 10 layers hex8, residual+Jacobian", layers=10,
+               elem="hex8"),
     "C4": dict(desc="Antarctica-like 4 km x 10 layers hex8, residual+Jacobian", layers=10, elem="hex8"),
     "C5": dict(desc="Antarctica-like 4 km x 10 layers wedge6, residual+Jacobian", layers=10, elem="wedge6"),
 }
@@ -276,10 +278,13 @@ PHYS_DEFAULTS = dict(k=10.77, glen_n=3.0, delta=1e-10, rho_g=8.927)
 
 
 def make_config(name: str, h: float | None = None):
-    """Return (footprint, L, elem) for a named configuration."""
+    """Return (footprint, L, elem) for a named configuration (C3 is defined
+    below; the module is fully imported before this is called)."""
     cfg = CONFIGS[name]
     if name in ("C1", "C2"):
         fp = tiny_footprint()
+    elif name == "C3":
+        fp = greenland_footprint()
     elif name == "C4":
         fp = antarctica_footprint(h=h or 4.0)
     elif name == "C5":
@@ -287,3 +292,164 @@ def make_config(name: str, h: float | None = None):
     else:
         raise KeyError(name)
     return fp, cfg["layers"], cfg["elem"]
+
+
+# ----------------------------------------------------------------------------
+# C3: Greenland-like variable-resolution footprint (BASELINE.json configs[2])
+# ----------------------------------------------------------------------------
+
+def _greenland_halfwidth(y):
+    c1 = np.clip((y - 200.0) / 1100.0, 0.0, 1.0)
+    c2 = np.clip((-y - 550.0) / 550.0, 0.0, 1.0)
+    return 480.0 * (1.0 - 0.45 * c1 ** 2) * (1.0 - 0.35 * c2)
+
+
+def greenland_inside(x, y):
+    """|x/w(y)|^2.5 + |y/1150|^2.5 < 1."""
+    return np.abs(x / _greenland_halfwidth(y)) ** 2.5 + np.abs(y / 1150.0) ** 2.5 < 1.0
+
+
+def greenland_footprint(h0: float = 20.0, hmin: float = 1.0, hmax: float = 10.0, ramp: float = 150.0,
+                        raster: float = 1.0, name: str = "C3") -> Footprint:
+    """Newest-vertex-bisection refinement (with conformity closure) of a
+    criss-cross right-triangle background of h0-km squares until every
+    hypotenuse <= 2 sqrt(2) h(d(centroid)), h(d) = min(hmax, hmin + (hmax-hmin) d/ramp),
+    d = distance to the margin; keep triangles whose centroid is inside; split
+    each triangle into 3 quads through its centroid and edge midpoints; columns
+    in Hilbert order (SURVEY 8(d1) 'C3 footprint construction').
+
+    H = max(0.02, 3.2 (1 - (1 - min(d/500, 1))^(4/3))^(3/8)) km;
+    b = 0.3 sin(2 pi x/400) cos(2 pi y/300) km.
+    """
+    from scipy import ndimage
+    x0, x1, y0, y1 = -560.0, 560.0, -1200.0, 1200.0
+    nx, ny = int((x1 - x0) / h0), int((y1 - y0) / h0)
+    # margin distance on a raster (outside and inside distances, unsigned)
+    gx = np.arange(x0, x1 + raster, raster)
+    gy = np.arange(y0, y1 + raster, raster)
+    GX, GY = np.meshgrid(gx, gy, indexing="ij")
+    ins = greenland_inside(GX, GY)
+    d_in = ndimage.distance_transform_edt(ins) * raster
+    d_out = ndimage.distance_transform_edt(~ins) * raster
+    dist_r = np.where(ins, d_in, d_out)
+
+    def dist_at(px, py):
+        i = np.clip(np.rint((px - x0) / raster).astype(np.int64), 0, gx.size - 1)
+        j = np.clip(np.rint((py - y0) / raster).astype(np.int64), 0, gy.size - 1)
+        return dist_r[i, j]
+
+    def hsize(d):
+        return np.minimum(hmax, hmin + (hmax - hmin) * d / ramp)
+
+    # --- background: vertices of the h0 lattice + square centres -------------
+    verts = []
+    vid = {}
+
+    def vert(p):
+        key = (round(p[0] * 1e6), round(p[1] * 1e6))
+        if key not in vid:
+            vid[key] = len(verts)
+            verts.append((p[0], p[1]))
+        return vid[key]
+
+    # triangle = (e0, e1, apex): CCW, refinement edge e0-e1 (the hypotenuse)
+    tris = {}
+    tid = 0
+    for i in range(nx):
+        for j in range(ny):
+            a = vert((x0 + i * h0, y0 + j * h0))
+            b = vert((x0 + (i + 1) * h0, y0 + j * h0))
+            c = vert((x0 + (i + 1) * h0, y0 + (j + 1) * h0))
+            d = vert((x0 + i * h0, y0 + (j + 1) * h0))
+            m = vert((x0 + (i + 0.5) * h0, y0 + (j + 0.5) * h0))
+            for e0, e1 in ((a, b), (b, c), (c, d), (d, a)):
+                tris[tid] = (e0, e1, m)
+                tid += 1
+    edge_tris = {}
+
+    def ekey(u, v):
+        return (u, v) if u < v else (v, u)
+
+    def add_tri(t, tri):
+        tris[t] = tri
+        for u, v in ((tri[0], tri[1]), (tri[1], tri[2]), (tri[2], tri[0])):
+            edge_tris.setdefault(ekey(u, v), set()).add(t)
+
+    def del_tri(t):
+        tri = tris.pop(t)
+        for u, v in ((tri[0], tri[1]), (tri[1], tri[2]), (tri[2], tri[0])):
+            edge_tris[ekey(u, v)].discard(t)
+
+    for t, tri in list(tris.items()):
+        add_tri(t, tri)
+    next_id = [tid]
+    mids = {}
+
+    def midpoint(u, v):
+        k = ekey(u, v)
+        if k not in mids:
+            pu, pv = verts[u], verts[v]
+            mids[k] = vert((0.5 * (pu[0] + pv[0]), 0.5 * (pu[1] + pv[1])))
+        return mids[k]
+
+    def bisect(t):
+        e0, e1, ap = tris[t]
+        m = midpoint(e0, e1)
+        del_tri(t)
+        for tri in ((ap, e0, m), (e1, ap, m)):
+            add_tri(next_id[0], tri)
+            next_id[0] += 1
+
+    def refine(t):
+        if t not in tris:
+            return
+        e0, e1, _ = tris[t]
+        nb = [s for s in edge_tris.get(ekey(e0, e1), ()) if s != t]
+        if nb:
+            s = nb[0]
+            if ekey(*tris[s][:2]) != ekey(e0, e1):
+                refine(s)
+                nb = [s2 for s2 in edge_tris.get(ekey(e0, e1), ()) if s2 != t]
+            bisect(t)
+            for s in nb:
+                if s in tris and ekey(*tris[s][:2]) == ekey(e0, e1):
+                    bisect(s)
+        else:
+            bisect(t)
+
+    import sys
+    sys.setrecursionlimit(100000)
+    while True:
+        ids = np.fromiter(tris.keys(), dtype=np.int64)
+        T = np.array([tris[t] for t in ids])
+        V = np.asarray(verts)
+        cen = V[T].mean(axis=1)
+        hyp = np.hypot(*(V[T[:, 0]] - V[T[:, 1]]).T)
+        mark = hyp > 2.0 * math.sqrt(2.0) * hsize(dist_at(cen[:, 0], cen[:, 1])) + 1e-9
+        if not mark.any():
+            break
+        for t in ids[mark]:
+            refine(int(t))
+    ids = np.fromiter(tris.keys(), dtype=np.int64)
+    T = np.array([tris[t] for t in ids], dtype=np.int64)
+    V = np.asarray(verts)
+    cen = V[T].mean(axis=1)
+    T = T[greenland_inside(cen[:, 0], cen[:, 1])]
+    # --- triangle -> 3 quads through centroid and edge midpoints -------------
+    quads = []
+    for a, b, c in T:
+        g = vert(tuple(V[[a, b, c]].mean(axis=0)))
+        mab, mbc, mca = midpoint(a, b), midpoint(b, c), midpoint(c, a)
+        quads += [(a, mab, g, mca), (b, mbc, g, mab), (c, mca, g, mbc)]
+    quads = np.array(quads, dtype=np.int64)
+    V = np.asarray(verts)
+    qc = V[quads].mean(axis=1)
+    hi = np.floor((qc - np.array([x0, y0])) / 0.5).astype(np.int64)
+    order = np.argsort(hilbert_index(hi[:, 0], hi[:, 1], 13), kind="stable")
+    quads = quads[order]
+    polys, old_of_new = _renumber_vertices_by_first_use(quads, V.shape[0])
+    xy = V[old_of_new]
+    d = dist_at(xy[:, 0], xy[:, 1]) * greenland_inside(xy[:, 0], xy[:, 1])
+    H = np.maximum(0.02, 3.2 * (1.0 - (1.0 - np.minimum(d / 500.0, 1.0)) ** (4.0 / 3.0)) ** (3.0 / 8.0))
+    b = 0.3 * np.sin(2 * math.pi * xy[:, 0] / 400.0) * np.cos(2 * math.pi * xy[:, 1] / 300.0)
+    return Footprint(name, xy.astype(np.float64), polys, b, H, dist=d)

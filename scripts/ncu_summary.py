@@ -82,7 +82,7 @@ def main():
     ap.add_argument("--tag", required=True)
     ap.add_argument("--rep")
     ap.add_argument("--launches")
-    ap.add_argument("--key", default="C4:hex8:jacobian")
+    ap.add_argument("--key", default="C4:hex8:jacobian:stored")
     ap.add_argument("--note", default="")
     a = ap.parse_args()
     prof = os.path.join(ROOT, "profiles")

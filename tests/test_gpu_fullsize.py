@@ -12,20 +12,21 @@ pytestmark = pytest.mark.gpu
 TOL = 1e-12
 
 
-@pytest.mark.parametrize("cfg", ["C4", "C5"])
-def test_fullsize_sampled_parity(cfg):
+@pytest.mark.parametrize("geometry", ["stored", "on_the_fly"])
+@pytest.mark.parametrize("cfg", ["C3", "C4", "C5"])
+def test_fullsize_sampled_parity(cfg, geometry):
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     from paper_conf_sc_antepara0cw24_b200 import StokesFO
     fp, L, elem = synth.make_config(cfg)
     conn, coords = O.extrude(fp.xy, fp.polys, fp.b, fp.H, L)
-    U = synth.velocity_balance(fp, L, seed=12)
+    U = synth.velocity_balance(fp, L, seed=11 if cfg == "C3" else 12)
     s = synth.surface_nodal(fp, L)
     kc = synth.flow_factor(fp, L)
     C, N = conn.shape
     ctx = StokesFO(elem, torch.from_numpy(conn).cuda(), torch.from_numpy(coords).cuda(),
-                   surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda())
+                   surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda(), geometry=geometry)
     J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
     R = torch.zeros((coords.shape[0], 2), dtype=torch.float64, device="cuda")
     Ud = torch.from_numpy(U).cuda()

@@ -29,7 +29,10 @@ def _t(torch, a, dtype=None):
     return torch.from_numpy(a).to("cuda") if dtype is None else torch.from_numpy(a).to("cuda", dtype)
 
 
-def _setup(torch, elem="hex8", n=16, L=5, drop=0, kind="random", scalar_k=False, surface=True):
+GEOMS = ["stored", "on_the_fly"]
+
+
+def _setup(torch, elem="hex8", n=16, L=5, drop=0, kind="random", scalar_k=False, surface=True, geometry="stored"):
     fp, conn, coords = M.tiny(elem, n=n, L=L)
     if drop:
         conn = conn[:conn.shape[0] - drop]
@@ -37,7 +40,7 @@ def _setup(torch, elem="hex8", n=16, L=5, drop=0, kind="random", scalar_k=False,
     kc = kc[:conn.shape[0]]
     from paper_conf_sc_antepara0cw24_b200 import StokesFO
     ctx = StokesFO(elem, _t(torch, conn), _t(torch, coords), surface=_t(torch, s) if surface else None,
-                   flow_factor=None if scalar_k else _t(torch, kc), k=10.77)
+                   flow_factor=None if scalar_k else _t(torch, kc), k=10.77, geometry=geometry)
     e = O.ELEM[elem]
     G, wm, bad = O.geometry(e, conn, coords)
     assert bad == 0
@@ -61,9 +64,10 @@ def _assembled_check(R_gpu, orc, R_cell_orc):
     assert (err <= TOL * absR + 1e-300).all(), float((err / np.maximum(absR, 1e-300)).max())
 
 
+@pytest.mark.parametrize("geometry", GEOMS)
 @pytest.mark.parametrize("elem", ["hex8", "wedge6"])
-def test_geometry_parity(torch, elem):
-    ctx, orc = _setup(torch, elem)
+def test_geometry_parity(torch, elem, geometry):
+    ctx, orc = _setup(torch, elem, geometry=geometry)
     G, wm = ctx.geometry()
     ctx.sync()
     G = G.cpu().numpy()
@@ -82,10 +86,11 @@ def test_gather_bit_exact(torch, elem):
     assert np.array_equal(Uc.cpu().numpy(), O.gather(orc["e"], orc["conn"], orc["U"]))
 
 
+@pytest.mark.parametrize("geometry", GEOMS)
 @pytest.mark.parametrize("elem,drop,kind", [("hex8", 0, "random"), ("hex8", 5, "balance"),
                                             ("wedge6", 0, "random"), ("wedge6", 7, "balance")])
-def test_viscosity_resid_parity(torch, elem, drop, kind):
-    ctx, orc = _setup(torch, elem, drop=drop, kind=kind)
+def test_viscosity_resid_parity(torch, elem, drop, kind, geometry):
+    ctx, orc = _setup(torch, elem, drop=drop, kind=kind, geometry=geometry)
     C, N, Q = ctx.num_cells, ctx.N, ctx.Q
     mu = torch.empty((C, Q), dtype=torch.float64, device="cuda")
     Rc = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
@@ -98,9 +103,10 @@ def test_viscosity_resid_parity(torch, elem, drop, kind):
     _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
 
 
+@pytest.mark.parametrize("geometry", GEOMS)
 @pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 0), ("wedge6", 11)])
-def test_jacobian_parity(torch, elem, drop):
-    ctx, orc = _setup(torch, elem, drop=drop)
+def test_jacobian_parity(torch, elem, drop, geometry):
+    ctx, orc = _setup(torch, elem, drop=drop, geometry=geometry)
     C, N = ctx.num_cells, ctx.N
     J = torch.full((C, 2 * N, 2 * N), float("nan"), dtype=torch.float64, device="cuda")
     Rc = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
@@ -116,8 +122,9 @@ def test_jacobian_parity(torch, elem, drop):
     _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
 
 
-def test_jacobian_residual_equals_viscosity_resid(torch):
-    ctx, orc = _setup(torch, "hex8")
+@pytest.mark.parametrize("geometry", GEOMS)
+def test_jacobian_residual_equals_viscosity_resid(torch, geometry):
+    ctx, orc = _setup(torch, "hex8", geometry=geometry)
     C, N = ctx.num_cells, ctx.N
     J = torch.empty((C, 16, 16), dtype=torch.float64, device="cuda")
     R1 = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
@@ -129,9 +136,10 @@ def test_jacobian_residual_equals_viscosity_resid(torch):
     assert torch.equal(R1, R2)
 
 
+@pytest.mark.parametrize("geometry", GEOMS)
 @pytest.mark.parametrize("scalar_k,surface", [(True, True), (False, False), (True, False)])
-def test_optional_inputs(torch, scalar_k, surface):
-    ctx, orc = _setup(torch, "hex8", n=6, L=3, scalar_k=scalar_k, surface=surface)
+def test_optional_inputs(torch, scalar_k, surface, geometry):
+    ctx, orc = _setup(torch, "hex8", n=6, L=3, scalar_k=scalar_k, surface=surface, geometry=geometry)
     C = ctx.num_cells
     J = torch.empty((C, 16, 16), dtype=torch.float64, device="cuda")
     Rc = torch.empty((C, 8, 2), dtype=torch.float64, device="cuda")
@@ -143,13 +151,14 @@ def test_optional_inputs(torch, scalar_k, surface):
     assert _cell_rel(Rc.cpu().numpy(), ref["R_cell"]) <= TOL
 
 
-def test_force_qp_input(torch):
+@pytest.mark.parametrize("geometry", GEOMS)
+def test_force_qp_input(torch, geometry):
     from paper_conf_sc_antepara0cw24_b200 import StokesFO
     fp, conn, coords = M.tiny("hex8", n=6, L=3)
     U, s, kc = M.fields(fp, 3)
     f = np.random.default_rng(9).normal(0, 1, (conn.shape[0], 8, 2))
     ctx = StokesFO("hex8", _t(torch, conn), _t(torch, coords), surface=_t(torch, s), force_qp=_t(torch, f),
-                   flow_factor=_t(torch, kc))
+                   flow_factor=_t(torch, kc), geometry=geometry)
     Rc = torch.empty((conn.shape[0], 8, 2), dtype=torch.float64, device="cuda")
     ctx.viscosity_resid(_t(torch, U), R_cell=Rc)
     ctx.sync()
@@ -158,14 +167,16 @@ def test_force_qp_input(torch):
     assert _cell_rel(Rc.cpu().numpy(), ref["R_cell"]) <= TOL
 
 
+@pytest.mark.parametrize("geometry", GEOMS)
 @pytest.mark.parametrize("name", ["B", "W"])
-def test_golden_cells_gpu(torch, golden, name):
+def test_golden_cells_gpu(torch, golden, name, geometry):
     from paper_conf_sc_antepara0cw24_b200 import StokesFO
     g = golden[name]
     N = 8 if g["elem"] == "hex8" else 6
     conn = np.arange(N, dtype=np.int32)[None]
     ctx = StokesFO(g["elem"], _t(torch, conn), _t(torch, np.array(g["coords"], float)),
-                   surface=_t(torch, np.array(g["s"], float)), k=g["k"], delta=g["delta"], rho_g=g["rho_g"])
+                   surface=_t(torch, np.array(g["s"], float)), k=g["k"], delta=g["delta"], rho_g=g["rho_g"],
+                   geometry=geometry)
     J = torch.empty((1, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
     Rc = torch.empty((1, N, 2), dtype=torch.float64, device="cuda")
     mu = torch.empty((1, N), dtype=torch.float64, device="cuda")
@@ -225,16 +236,17 @@ def test_halo_pack_unpack(torch):
     assert torch.equal(R2[nodes.long()], R[nodes.long()] * 2)
 
 
-def test_edge_cases_and_errors(torch):
+@pytest.mark.parametrize("geometry", GEOMS)
+def test_edge_cases_and_errors(torch, geometry):
     from paper_conf_sc_antepara0cw24_b200 import StokesFO, StokesFOError
     fp, conn, coords = M.tiny("hex8", n=2, L=1)
     # empty mesh: every call is a no-op
-    ctx0 = StokesFO("hex8", _t(torch, conn[:0]), _t(torch, coords))
+    ctx0 = StokesFO("hex8", _t(torch, conn[:0]), _t(torch, coords), geometry=geometry)
     J0 = torch.empty((0, 16, 16), dtype=torch.float64, device="cuda")
     ctx0.jacobian(torch.zeros((coords.shape[0], 2), dtype=torch.float64, device="cuda"), J0)
     ctx0.sync()
     # one cell
-    ctx1 = StokesFO("hex8", _t(torch, conn[:1]), _t(torch, coords))
+    ctx1 = StokesFO("hex8", _t(torch, conn[:1]), _t(torch, coords), geometry=geometry)
     J1 = torch.empty((1, 16, 16), dtype=torch.float64, device="cuda")
     U = np.random.default_rng(0).normal(0, 50, (coords.shape[0], 2))
     ctx1.jacobian(_t(torch, U), J1)
@@ -244,17 +256,17 @@ def test_edge_cases_and_errors(torch):
     assert _cell_rel(J1.cpu().numpy(), ref["J_cell"]) <= TOL
     # glen_n != 3
     with pytest.raises(StokesFOError, match="EUNSUPPORTED"):
-        StokesFO("hex8", _t(torch, conn), _t(torch, coords), glen_n=2.0)
+        StokesFO("hex8", _t(torch, conn), _t(torch, coords), glen_n=2.0, geometry=geometry)
     # inverted cell -> EMESH at sync
     bad = conn.copy()
     bad[0] = bad[0][[4, 5, 6, 7, 0, 1, 2, 3]]
-    ctxb = StokesFO("hex8", _t(torch, bad), _t(torch, coords))
+    ctxb = StokesFO("hex8", _t(torch, bad), _t(torch, coords), geometry=geometry)
     with pytest.raises(StokesFOError, match="EMESH"):
         ctxb.sync()
     # conn out of range -> EMESH
     bad2 = conn.copy()
     bad2[1, 3] = coords.shape[0] + 5
-    ctxc = StokesFO("hex8", _t(torch, bad2), _t(torch, coords))
+    ctxc = StokesFO("hex8", _t(torch, bad2), _t(torch, coords), geometry=geometry)
     with pytest.raises(StokesFOError, match="EMESH"):
         ctxc.sync()
     # misaligned output pointer -> EINVAL
