@@ -141,13 +141,18 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
     qp_coords<E>(q, xq, yq, zq, wq);
     double dphi[N][3];
     double J[3][3] = {{0, 0, 0}, {0, 0, 0}, {0, 0, 0}};
+    // cell-local coordinates x_n - x_0 (sum_n grad_xi phi_n = 0): avoids the
+    // O(|x| eps) residue of ~10^3-km absolute coordinates on metre-thick cells
+    const double o0 = coords[3 * (int64_t)nid[0] + 0];
+    const double o1 = coords[3 * (int64_t)nid[0] + 1];
+    const double o2 = coords[3 * (int64_t)nid[0] + 2];
 #pragma unroll
     for (int n = 0; n < N; ++n) {
         double phi;
         basis<E>(n, xq, yq, zq, phi, dphi[n][0], dphi[n][1], dphi[n][2]);
-        const double x0 = coords[3 * (int64_t)nid[n] + 0];
-        const double x1 = coords[3 * (int64_t)nid[n] + 1];
-        const double x2 = coords[3 * (int64_t)nid[n] + 2];
+        const double x0 = coords[3 * (int64_t)nid[n] + 0] - o0;
+        const double x1 = coords[3 * (int64_t)nid[n] + 1] - o1;
+        const double x2 = coords[3 * (int64_t)nid[n] + 2] - o2;
 #pragma unroll
         for (int s = 0; s < 3; ++s) {
             J[0][s] += x0 * dphi[n][s];
@@ -662,10 +667,15 @@ __global__ void __launch_bounds__(E::TC *E::N, (E::N == 8 ? 3 : 2)) eval_otf_ker
             const int c = t % TC, q = t / TC;
             const double *dq = dphi + q * N * 3;
             double J00 = 0, J01 = 0, J02 = 0, J10 = 0, J11 = 0, J12 = 0, J20 = 0, J21 = 0, J22 = 0;
+            // cell-local coordinates x_n - x_0 (see geometry_kernel)
+            const double2 xy0 = XY[c];
+            const double z0 = ZW[c].x;
 #pragma unroll
             for (int n = 0; n < N; ++n) {
-                const double2 xy = XY[n * TC + c];
-                const double z = ZW[n * TC + c].x;
+                double2 xy = XY[n * TC + c];
+                xy.x -= xy0.x;
+                xy.y -= xy0.y;
+                const double z = ZW[n * TC + c].x - z0;
                 const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
                 J00 = fma(xy.x, d0, J00); J01 = fma(xy.x, d1, J01); J02 = fma(xy.x, d2, J02);
                 J10 = fma(xy.y, d0, J10); J11 = fma(xy.y, d1, J11); J12 = fma(xy.y, d2, J12);

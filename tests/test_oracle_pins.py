@@ -465,3 +465,28 @@ def test_partition_and_halo_sum_equals_serial():
         parts[s_][2][halo[(s_, r)]] += sent[(r, s_)]                           # then unpack-add
     for lconn, gids, Rl in parts:
         assert np.abs(Rl - Rser[gids]).max() < 1e-12 * np.abs(Rser).max()
+
+
+def test_geometry_translation_invariant_and_exact_on_offset_thin_cell():
+    """Reading Z17: GradBF and det J depend only on relative node positions.
+    A metre-thick, sloped cell 800 km from the origin must give the same
+    geometry as the same cell at the origin, and det J must match an exact
+    rational evaluation of the cofactor expansion (pins the cancellation fix)."""
+    from fractions import Fraction
+    xyz = np.array([(0, 0, 0), (1.25, 0.1, 0.006), (1.3, 1.2, 0.004), (-0.05, 1.25, -0.002),
+                    (0, 0, 0.002), (1.25, 0.1, 0.0085), (1.3, 1.2, 0.0061), (-0.05, 1.25, 0.0003)], float)
+    conn = np.arange(8, dtype=np.int32)[None]
+    G0, wm0, bad0 = O.geometry(HEX, conn, xyz)
+    off = xyz + np.array([812.345678, -655.4321, 1.7])
+    G1, wm1, bad1 = O.geometry(HEX, conn, off)
+    assert bad0 == 0 and bad1 == 0
+    assert np.abs(wm1 / wm0 - 1).max() < 1e-13
+    assert np.abs(G1 - G0).max() < 1e-13 * np.abs(G0).max()
+    _, dbf, w = O.ref_element(HEX)
+    X = [[Fraction(float(v)) for v in p] for p in off]
+    for q in range(8):
+        Jm = [[sum(X[n][r] * Fraction(float(dbf[n, q, s])) for n in range(8)) for s in range(3)] for r in range(3)]
+        det = (Jm[0][0] * (Jm[1][1] * Jm[2][2] - Jm[1][2] * Jm[2][1])
+               - Jm[0][1] * (Jm[1][0] * Jm[2][2] - Jm[1][2] * Jm[2][0])
+               + Jm[0][2] * (Jm[1][0] * Jm[2][1] - Jm[1][1] * Jm[2][0]))
+        assert abs(wm1[0, q] / float(det) - 1) < 1e-14
