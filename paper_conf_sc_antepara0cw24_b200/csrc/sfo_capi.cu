@@ -57,8 +57,7 @@ int64_t xyz4_bytes(int64_t nnodes) {
 template <class E>
 int64_t ws_bytes(int64_t ncells, int64_t nnodes, int mode) {
     const int64_t ntiles = (ncells + E::TC - 1) / E::TC;
-    if (mode == STOKESFO_GEOMETRY_ON_THE_FLY)
-        return WS_HEADER + xyz4_bytes<E>(nnodes) + ntiles * (int64_t)Rec<E>::LIGHT_BYTES;
+    if (mode == STOKESFO_GEOMETRY_ON_THE_FLY) return WS_HEADER + xyz4_bytes<E>(nnodes);
     return WS_HEADER + ntiles * (int64_t)Rec<E>::BYTES;
 }
 
@@ -71,7 +70,7 @@ int configure_otf(int *grid) {
     int dev = 0, sms = 0, per_sm = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, E::TC * E::N, S::BYTES) != cudaSuccess)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, S::BYTES) != cudaSuccess)
         return cuda_status();
     *grid = std::max(1, sms * std::max(1, per_sm));
     return STOKESFO_OK;
@@ -86,7 +85,7 @@ int configure_eval(int *grid) {
     int dev = 0, sms = 0, per_sm = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, E::TC * E::N, S::BYTES) != cudaSuccess)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, S::BYTES) != cudaSuccess)
         return cuda_status();
     *grid = std::max(1, sms * std::max(1, per_sm));
     return STOKESFO_OK;
@@ -99,10 +98,10 @@ int create_impl(stokesfo_ctx *c) {
     c->TC = E::TC;
     c->ntiles = (c->d.num_cells + E::TC - 1) / E::TC;
     const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
-    c->rec_bytes = otf ? Rec<E>::LIGHT_BYTES : Rec<E>::BYTES;
+    c->rec_bytes = otf ? 0 : Rec<E>::BYTES;
     int st;
     if (otf) {
-        c->nstage_resid = c->nstage_jac = NLIGHT;
+        c->nstage_resid = c->nstage_jac = 0;
         st = configure_otf<E, false>(&c->grid_resid);
         if (st) return st;
         st = configure_otf<E, true>(&c->grid_jac);
@@ -125,8 +124,6 @@ int create_impl(stokesfo_ctx *c) {
         if (otf) {
             xyz4_kernel<<<(unsigned)((c->d.num_nodes + bs - 1) / bs), bs, 0, c->stream>>>(c->d.num_nodes, c->d.coords,
                                                                                           c->xyz4);
-            light_record_kernel<E><<<(unsigned)((c->ntiles * E::TC + bs - 1) / bs), bs, 0, c->stream>>>(
-                c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.flow_factor, c->d.k, c->recs, c->err);
             const int64_t work = c->d.num_cells * E::Q;
             geometry_kernel<E, GEO_CHECK><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
                 c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.coords, nullptr, 0.0, nullptr, nullptr, nullptr,
@@ -147,6 +144,9 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     EvalArgs a;
     a.recs = c->recs;
     a.xyz4 = c->xyz4;
+    a.conn = c->d.conn;
+    a.kc = c->d.flow_factor;
+    a.kscal = c->d.k;
     a.err = c->err;
     a.ntiles = c->ntiles;
     a.ncells = c->d.num_cells;
@@ -161,11 +161,11 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.J_cell = J_cell;
     const int grid = (int)std::min<int64_t>(JAC ? c->grid_jac : c->grid_resid, c->ntiles);
     if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY)
-        eval_otf_kernel<E, JAC><<<grid, E::TC * E::N, OtfSmem<E, JAC>::BYTES, c->stream>>>(a);
+        eval_otf_kernel<E, JAC><<<grid, 32, OtfSmem<E, JAC>::BYTES, c->stream>>>(a);
     else if ((JAC ? c->nstage_jac : c->nstage_resid) == 3)
-        eval_kernel<E, JAC, 3><<<grid, E::TC * E::N, EvalSmem<E, JAC, 3>::BYTES, c->stream>>>(a);
+        eval_kernel<E, JAC, 3><<<grid, 32, EvalSmem<E, JAC, 3>::BYTES, c->stream>>>(a);
     else
-        eval_kernel<E, JAC, 2><<<grid, E::TC * E::N, EvalSmem<E, JAC, 2>::BYTES, c->stream>>>(a);
+        eval_kernel<E, JAC, 2><<<grid, 32, EvalSmem<E, JAC, 2>::BYTES, c->stream>>>(a);
     return cuda_status();
 }
 
@@ -223,7 +223,7 @@ int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
     char *ws = reinterpret_cast<char *>(d->workspace);
     if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY) {
         c->xyz4 = reinterpret_cast<double4 *>(ws + WS_HEADER);
-        c->recs = ws + WS_HEADER + (d->elem == STOKESFO_HEX8 ? xyz4_bytes<Hex8>(d->num_nodes) : xyz4_bytes<Wedge6>(d->num_nodes));
+        c->recs = nullptr;
     } else {
         c->xyz4 = nullptr;
         c->recs = ws + WS_HEADER;

@@ -10,56 +10,48 @@
 namespace sfo {
 
 // ---------------------------------------------------------------------------
-// Element traits.  N nodes, Q quadrature points, TC cells per tile.
-// Tile sizes are chosen so that one CTA holds TC*N threads (phase-2 mapping)
-// = TC*Q threads (phase-1 mapping); see DESIGN.md "Kernels".
+// Element traits.  N nodes, Q quadrature points (N == Q for both elements),
+// TC cells per tile.  One tile is processed by ONE warp (one CTA = one warp):
+// lane l <-> (cell l / N, node-or-qp l % N), TC = floor(32 / N) cells, so every
+// exchange between the per-QP and per-node phases stays inside a warp
+// (__syncwarp only; no CTA-wide barriers).  See DESIGN.md "Kernels".
 // ---------------------------------------------------------------------------
 struct Hex8 {
-    static constexpr int N = 8, Q = 8, TC = 16, ELEM = 0;
-    // phase-2 mapping: thread <-> (cell t/N, node t%N): the 8 threads of a cell
-    // share one warp quarter, so per-(cell,qp) scalars are read as broadcasts.
-    static constexpr bool NODE_MAJOR_P2 = false;
-    static constexpr int JPITCH = 4 * N * N;  // J staging pitch per cell (dense: one bulk store per tile)
-    // Swizzles (cell index within the tile), chosen with a bank model of 64-bit
-    // shared loads served per half-warp: every phase-1/phase-2 GradBF load and
-    // every conn load is conflict-free.
-    __host__ __device__ static constexpr int gswz(int c, int n) { return c ^ ((2 * n) & 15); }
-    __host__ __device__ static constexpr int cswz(int c, int n) { return c ^ (4 * ((n >> 1) & 3)); }
+    static constexpr int N = 8, Q = 8, TC = 4, ELEM = 0;
+    static constexpr int SLAB = 32;  // doubles per (qp, dir) slab of GradBF in a record
 };
 struct Wedge6 {
-    static constexpr int N = 6, Q = 6, TC = 32, ELEM = 1;
-    // phase-2 mapping: thread <-> (cell t%TC, node t/TC) (node-major: 6 does not
-    // divide a warp); J staging uses a padded pitch (73 x 16 B) and per-cell
-    // bulk stores so the 16-byte staging stores are conflict-free.
-    static constexpr bool NODE_MAJOR_P2 = true;
-    static constexpr int JPITCH = 4 * N * N + 2;
-    __host__ __device__ static constexpr int gswz(int c, int) { return c; }
-    __host__ __device__ static constexpr int cswz(int c, int) { return c; }
+    static constexpr int N = 6, Q = 6, TC = 5, ELEM = 1;  // 30 active lanes
+    static constexpr int SLAB = 30;
 };
 
 __host__ __device__ constexpr int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
 
 // Per-tile record in the workspace (and, identically, in shared memory):
-//   conn  int32 [N][TC]          node ids, cell fastest
-//   kc    fp64  [TC]             Glen prefactor per cell
-//   wm    fp64  [Q][TC]          w_q det J_q
-//   G     fp64  [N][Q][3][TC]    GradBF, cell fastest
-// One 1-D TMA bulk copy moves a whole record (size multiple of 128 B).
+//   conn  int32 [TC][N]                 node ids
+//   kc    fp64  [TC]                    Glen prefactor per cell
+//   wm    fp64  [Q][TC]                 w_q det J_q
+//   G     fp64  [Q][3][SLAB]            GradBF; (cell c, node n) of qp q sits at
+//                                       slot c*N + (n + q) mod N
+// The slot rotation makes both the per-QP loads (fixed n, lanes over (c, q))
+// and the per-node loads (fixed q, lanes over (c, j)) hit 16 distinct bank
+// pairs per half-warp for hex8 (bank model in DESIGN.md).  One 1-D TMA bulk
+// copy moves a whole record (size multiple of 16 B: 6,560 B hex8, 4,736 B wedge6).
 template <class E>
 struct Rec {
-    static constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    static constexpr int N = E::N, Q = E::Q, TC = E::TC, SLAB = E::SLAB;
     static constexpr int CONN_OFF = 0;
     static constexpr int CONN_BYTES = (int)round_up(N * TC * 4, 16);
     static constexpr int KC_OFF = CONN_OFF + CONN_BYTES;
-    static constexpr int WM_OFF = KC_OFF + TC * 8;
-    static constexpr int G_OFF = WM_OFF + Q * TC * 8;
-    static constexpr int BYTES = (int)round_up(G_OFF + N * Q * 3 * TC * 8, 128);
-    // light record (on-the-fly geometry mode): conn + k_c only
-    static constexpr int LIGHT_BYTES = (int)round_up(KC_OFF + TC * 8, 128);
+    static constexpr int WM_OFF = KC_OFF + (int)round_up(TC * 8, 16);
+    static constexpr int G_OFF = WM_OFF + (int)round_up(Q * TC * 8, 16);
+    static constexpr int BYTES = G_OFF + Q * 3 * SLAB * 8;
     // index helpers (in elements of the respective type)
-    __host__ __device__ static constexpr int conn(int n, int c) { return n * TC + E::cswz(c, n); }
+    __host__ __device__ static constexpr int conn(int n, int c) { return c * N + n; }
     __host__ __device__ static constexpr int wm(int q, int c) { return q * TC + c; }
-    __host__ __device__ static constexpr int g(int n, int q, int d, int c) { return ((n * Q + q) * 3 + d) * TC + E::gswz(c, n); }
+    __host__ __device__ static constexpr int g(int n, int q, int d, int c) {
+        return (q * 3 + d) * SLAB + c * N + (n + q) % N;
+    }
 };
 
 // Workspace: [0, 256) header (error flag), then ntiles records.

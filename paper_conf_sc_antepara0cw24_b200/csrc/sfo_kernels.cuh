@@ -219,11 +219,15 @@ __global__ void gather_kernel(int64_t ncells, const int32_t *__restrict__ conn, 
 }
 
 // ---------------------------------------------------------------------------
-// G3/G4: fused evaluation.
+// G3/G4: fused evaluation.  One CTA = one warp, persistent over tiles of TC
+// cells; lane l <-> (cell l / N, node-or-qp l % N).
 // ---------------------------------------------------------------------------
 struct EvalArgs {
-    const char *recs;         // per-tile records (full: stored geometry; light: conn + k_c)
-    const double4 *xyz4;      // on-the-fly geometry: node coordinates (x, y, z, 0)
+    const char *recs;         // per-tile records (stored-geometry mode)
+    const double4 *xyz4;      // node coordinates (x, y, z, 0) (on-the-fly mode)
+    const int32_t *conn;      // caller conn [C][N] (on-the-fly mode)
+    const double *kc;         // caller flow factor [C] or null (on-the-fly mode)
+    double kscal;             // scalar k if kc == null
     int *err;                 // sticky device error flag
     int64_t ntiles, ncells;
     const double *U;          // [nodes][2]
@@ -238,32 +242,38 @@ struct EvalArgs {
 
 constexpr int NQS = 9;  // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 beta12, wmu2, gamma, wf0, wf1
 
+// per-QP scalar f of (cell c, qp q): [NQS][TC][Q] (qp fastest: the per-QP
+// phase writes 32 consecutive doubles, the per-node phase reads broadcasts)
+template <class E>
+__device__ __forceinline__ int qsi(int f, int c, int q) {
+    return (f * E::TC + c) * E::Q + q;
+}
+
 // ---- shared device pieces ---------------------------------------------------
 
-// Per-QP tail of phase 1: given Ugrad and grad s_h at (cell c, qp q), evaluate
-// the effective strain rate (Z2), Glen viscosity at n = 3 (Z1, Z3) and the
-// per-QP scalars phase 2 needs.  beta = B g so that sigma = 2 mu beta gives
+// Per-QP tail: given Ugrad and grad s_h at (cell c, qp q), evaluate the
+// effective strain rate (Z2), Glen viscosity at n = 3 (Z1, Z3) and the per-QP
+// scalars the per-node phase needs.  beta = B g so that sigma = 2 mu beta gives
 // strs00..strs12 of Fig. 2.
 template <class E>
 __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, int q, int nvalid, int64_t cell0,
                                         bool have_s, double kc, double wm, double ux, double uy, double uz, double vx,
                                         double vy, double vz, double gs0, double gs1) {
-    constexpr int Q = E::Q, TC = E::TC;
+    constexpr int Q = E::Q;
     constexpr double P_EXP = -1.0 / 3.0;  // (1 - n) / (2 n) at n = 3
     const double uyvx = uy + vx;
     const double e2 = ux * ux + vy * vy + ux * vy + 0.25 * uyvx * uyvx + 0.25 * uz * uz + 0.25 * vz * vz;
     const double r = rcbrt(e2 + a.delta);  // (e2 + delta)^(-1/3)
     const double mu = kc * r;
     const double wmu2 = 2.0 * wm * mu;
-    double *qq = qs + q * TC + c;
-    qq[0 * Q * TC] = 2.0 * ux + vy;   // beta_(0,0) = strs00 / (2 mu)
-    qq[1 * Q * TC] = 0.5 * uyvx;      // beta_(0,1) = beta_(1,0) = strs01 / (2 mu)
-    qq[2 * Q * TC] = 0.5 * uz;        // beta_(0,2) = strs02 / (2 mu)
-    qq[3 * Q * TC] = ux + 2.0 * vy;   // beta_(1,1) = strs11 / (2 mu)
-    qq[4 * Q * TC] = 0.5 * vz;        // beta_(1,2) = strs12 / (2 mu)
-    qq[5 * Q * TC] = wmu2;
+    qs[qsi<E>(0, c, q)] = 2.0 * ux + vy;   // beta_(0,0) = strs00 / (2 mu)
+    qs[qsi<E>(1, c, q)] = 0.5 * uyvx;      // beta_(0,1) = beta_(1,0) = strs01 / (2 mu)
+    qs[qsi<E>(2, c, q)] = 0.5 * uz;        // beta_(0,2) = strs02 / (2 mu)
+    qs[qsi<E>(3, c, q)] = ux + 2.0 * vy;   // beta_(1,1) = strs11 / (2 mu)
+    qs[qsi<E>(4, c, q)] = 0.5 * vz;        // beta_(1,2) = strs12 / (2 mu)
+    qs[qsi<E>(5, c, q)] = wmu2;
     // gamma = wM 2 mu p / (e2 + delta) = wmu2 p r^3  (d mu / d e2, reading Z5)
-    qq[6 * Q * TC] = wmu2 * P_EXP * (r * r * r);
+    qs[qsi<E>(6, c, q)] = wmu2 * P_EXP * (r * r * r);
     double wf0 = 0.0, wf1 = 0.0;
     if (a.force_qp) {
         if (c < nvalid) {
@@ -275,14 +285,15 @@ __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, in
         wf0 = wm * a.rho_g * gs0;
         wf1 = wm * a.rho_g * gs1;
     }
-    qq[7 * Q * TC] = wf0;
-    qq[8 * Q * TC] = wf1;
+    qs[qsi<E>(7, c, q)] = wf0;
+    qs[qsi<E>(8, c, q)] = wf1;
     if (a.mu_qp && c < nvalid) a.mu_qp[(cell0 + c) * Q + q] = mu;
 }
 
-// Phase 2, thread <-> (cell c2, node i): residual rows (i,0), (i,1) and, for
-// JAC, the 2x2 tangent blocks J[(i,.),(j_k,.)], j_k = (i+k) mod N, k = 0..N/2,
-// accumulated over QPs in registers (the paper's local accumulation).
+// Per-node phase, lane <-> (cell c2, node i): residual rows (i,0), (i,1) and,
+// for JAC, the 2x2 tangent blocks J[(i,.),(j_k,.)], j_k = (i+k) mod N,
+// k = 0..N/2, accumulated over QPs in registers (the paper's local
+// accumulation).
 // J_q[(i,a),(j,b)] = sum_e M_ab[e] G_j[e],
 // M_ab = wM 2 mu (B-block (a,b) applied to G_i) + gamma h_(i,a) beta_(b,.)
 // is the exact forward derivative of the chain (seed-sparse Sacado lanes).
@@ -290,7 +301,7 @@ __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, in
 template <class E, bool JAC, class PF>
 __device__ __forceinline__ void node_accumulate(const double *rg, const double *qs, int c2, int i, const double *bfi,
                                                 double &R0, double &R1, double (&Jb)[E::N / 2 + 1][2][2], PF pf) {
-    constexpr int N = E::N, Q = E::Q, TC = E::TC, K = N / 2;
+    constexpr int N = E::N, Q = E::Q, K = N / 2;
     R0 = 0.0;
     R1 = 0.0;
     if (JAC) {
@@ -300,12 +311,11 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
         if (q == Q / 2) pf();
-        const double *qq = qs + q * TC + c2;
-        const double b00 = qq[0 * Q * TC], b01 = qq[1 * Q * TC], b02 = qq[2 * Q * TC];
-        const double b11 = qq[3 * Q * TC], b12 = qq[4 * Q * TC];
+        const double b00 = qs[qsi<E>(0, c2, q)], b01 = qs[qsi<E>(1, c2, q)], b02 = qs[qsi<E>(2, c2, q)];
+        const double b11 = qs[qsi<E>(3, c2, q)], b12 = qs[qsi<E>(4, c2, q)];
         const double b10 = b01;
-        const double wmu2 = qq[5 * Q * TC];
-        const double wf0 = qq[7 * Q * TC], wf1 = qq[8 * Q * TC];
+        const double wmu2 = qs[qsi<E>(5, c2, q)];
+        const double wf0 = qs[qsi<E>(7, c2, q)], wf1 = qs[qsi<E>(8, c2, q)];
         const double gi0 = rg[gidx<E>(i, q, 0, c2)];
         const double gi1 = rg[gidx<E>(i, q, 1, c2)];
         const double gi2 = rg[gidx<E>(i, q, 2, c2)];
@@ -315,7 +325,7 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
         R0 = fma(wf0, bfi[q], fma(wmu2, h0, R0));
         R1 = fma(wf1, bfi[q], fma(wmu2, h1, R1));
         if (JAC) {
-            const double gam = qq[6 * Q * TC];
+            const double gam = qs[qsi<E>(6, c2, q)];
             const double gh0 = gam * h0, gh1 = gam * h1;
             const double w0 = wmu2 * gi0, w1 = wmu2 * gi1, w2 = wmu2 * gi2;
             const double m00x = fma(2.0, w0, gh0 * b00), m00y = fma(0.5, w1, gh0 * b01),
@@ -352,7 +362,7 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
 template <class E>
 __device__ __forceinline__ void stage_J(double *base, int c2, int i, const double (&Jb)[E::N / 2 + 1][2][2]) {
     constexpr int N = E::N, K = N / 2, LD = 2 * N;
-    double *Jc = base + c2 * E::JPITCH;
+    double *Jc = base + c2 * (4 * N * N);
 #pragma unroll
     for (int k = 0; k <= K; ++k) {
         const int j = (i + k) % N;
@@ -365,19 +375,6 @@ __device__ __forceinline__ void stage_J(double *base, int c2, int i, const doubl
     }
 }
 
-// One thread issues the TMA bulk store(s) of the staged J image of a tile.
-template <class E>
-__device__ __forceinline__ void store_J(double *J_cell, int64_t cell0, int nvalid, const char *stage, uint64_t pol) {
-    constexpr int NN = 4 * E::N * E::N;
-    if (E::JPITCH == NN) {
-        bulk_s2g(J_cell + cell0 * NN, stage, (uint32_t)(nvalid * NN * 8), pol);
-    } else {
-        for (int c = 0; c < nvalid; ++c)
-            bulk_s2g(J_cell + (cell0 + c) * NN, stage + c * E::JPITCH * 8, (uint32_t)(NN * 8), pol);
-    }
-    bulk_commit();
-}
-
 template <class E>
 __device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
 #pragma unroll
@@ -388,85 +385,82 @@ __device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
     }
 }
 
+// Resident 1-warp CTAs per SM the register budget is sized for.
+template <class E>
+constexpr int warps_per_sm() {
+    return 12;
+}
+
 // ---- G3/G4 with stored geometry (the §8(a2) precompute streamed per tile) ----
 
-// Shared memory: NSTAGE stage buffers + per-QP scalars + mbarriers.
-// A stage buffer holds [record | gathered U (double2 [N][TC]) | s ([N][TC])];
-// once a tile's phase 2 has consumed its record, the same buffer stages the
-// tile's element Jacobians for the TMA bulk store (JAC).
+// Shared memory: NSTAGE stage buffers + per-QP scalars + mbarriers.  A stage
+// buffer holds [record | gathered U (double2 [TC][N]) | s ([TC][N])]; once the
+// warp has consumed a tile's record, the same buffer stages the tile's element
+// Jacobians (the global image) for one TMA bulk store.
 template <class E, bool JAC, int NSTAGE = 2>
 struct EvalSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static constexpr int REC = Rec<E>::BYTES;
-    static constexpr int U_OFF = REC;                        // double2 [N][TC]
-    static constexpr int S_OFF = U_OFF + N * TC * 16;        // double  [N][TC]
-    static constexpr int IN_BYTES = S_OFF + N * TC * 8;
-    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;
+    static constexpr int U_OFF = (int)round_up(REC, 16);     // double2 [TC][N]
+    static constexpr int S_OFF = U_OFF + TC * N * 16;        // double  [TC][N]
+    static constexpr int IN_BYTES = S_OFF + TC * N * 8;
+    static constexpr int J_BYTES = JAC ? TC * 4 * N * N * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
-    static constexpr int OFF_QS = NSTAGE * STAGE;            // double [NQS][Q][TC]
-    static constexpr int OFF_BAR = OFF_QS + NQS * Q * TC * 8;
+    static constexpr int OFF_QS = NSTAGE * STAGE;            // double [NQS][TC][Q]
+    static constexpr int OFF_BAR = (int)round_up(OFF_QS + NQS * TC * Q * 8, 8);
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
 };
 
-// Issue the gather of U (16 B) and s (8 B) of one tile through its conn, as
-// cp.async copies into the tile's stage buffer (thread <-> (cell, node)).
+// Gather U (16 B) and s (8 B) of one tile through its conn as cp.async copies
+// into the tile's stage buffer (lane <-> (cell, node)).
 template <class E>
 __device__ __forceinline__ void issue_gather(char *stage, const double *U, const double *surface, bool have_s) {
     using R = Rec<E>;
     using S = EvalSmem<E, false>;
-    const int t = threadIdx.x;
-    const int c = t % E::TC, n = t / E::TC;
-    const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[R::conn(n, c)];
-    cp_async16(stage + S::U_OFF + (n * E::TC + c) * 16, U + 2 * (int64_t)g);
-    if (have_s) cp_async8(stage + S::S_OFF + (n * E::TC + c) * 8, surface + g);
+    const int l = threadIdx.x;
+    if (l < E::TC * E::N) {
+        const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[l];  // conn(n, c) = l
+        cp_async16(stage + S::U_OFF + l * 16, U + 2 * (int64_t)g);
+        if (have_s) cp_async8(stage + S::S_OFF + l * 8, surface + g);
+    }
     cp_async_commit();
 }
 
-// Resident CTAs per SM the register budget is tuned for (shared memory permits
-// this many for hex8 at the given stage count).
 template <class E, bool JAC, int NSTAGE>
-constexpr int min_blocks() {
-    return E::N == 8 ? (NSTAGE == 2 ? 3 : 2) : 2;
-}
-
-template <class E, bool JAC, int NSTAGE>
-__global__ void __launch_bounds__(E::TC *E::N, (min_blocks<E, JAC, NSTAGE>())) eval_kernel(EvalArgs a) {
+__global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
-    static_assert(N == Q, "thread mappings assume N == Q");
+    static_assert(N == Q, "lane mappings assume N == Q");
     using R = Rec<E>;
     using S = EvalSmem<E, JAC, NSTAGE>;
     static_assert(S::U_OFF == EvalSmem<E, false>::U_OFF && S::S_OFF == EvalSmem<E, false>::S_OFF, "layout");
     extern __shared__ __align__(128) char smem[];
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
-    const int t = threadIdx.x;
+    const int l = threadIdx.x;
+    const int c = l / N, s = l % N;  // (cell, node-or-qp)
+    const bool act = c < TC;
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
 
     uint64_t pol_stream = 0;
-    if (t == 0) {
+    if (l == 0) {
         pol_stream = policy_evict_first();
-        for (int s = 0; s < NSTAGE; ++s) mbar_init(&bar[s], 1);
+        for (int k = 0; k < NSTAGE; ++k) mbar_init(&bar[k], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    if (t == 0) {
-        for (int s = 0; s < NSTAGE; ++s) {
-            const int64_t tile = blockIdx.x + (int64_t)s * gridDim.x;
+        for (int k = 0; k < NSTAGE; ++k) {
+            const int64_t tile = blockIdx.x + (int64_t)k * gridDim.x;
             if (tile < a.ntiles) {
-                mbar_arrive_expect_tx(&bar[s], R::BYTES);
-                bulk_g2s(smem + s * S::STAGE, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[s], pol_stream);
+                mbar_arrive_expect_tx(&bar[k], R::BYTES);
+                bulk_g2s(smem + k * S::STAGE, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[k], pol_stream);
             }
         }
     }
+    __syncwarp();
     if ((int64_t)blockIdx.x < a.ntiles) {
         mbar_wait(&bar[0], 0);
         issue_gather<E>(smem, a.U, a.surface, have_s);
     }
-
-    const int c2 = E::NODE_MAJOR_P2 ? t % TC : t / N;
-    const int i = E::NODE_MAJOR_P2 ? t / TC : t % N;
     double bfi[Q];
-    basis_row<E>(i, bfi);
+    basis_row<E>(act ? s : 0, bfi);
 
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
@@ -481,176 +475,161 @@ __global__ void __launch_bounds__(E::TC *E::N, (min_blocks<E, JAC, NSTAGE>())) e
         const int64_t cell0 = tile * TC;
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
 
-        cp_async_wait_all();  // this thread's gathers for this tile have landed
-        __syncthreads();      // ... and everyone's
+        cp_async_wait_all();  // this lane's gathers for this tile have landed
+        __syncwarp();         // ... and every lane's
 
-        // ---- phase 1: per-QP quantities (thread <-> (cell, qp)) ----
-        {
-            const int c = t % TC, q = t / TC;
+        // ---- per-QP phase: lane <-> (cell c, qp s) ----
+        if (act) {
+            const int q = s;
             double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
 #pragma unroll
             for (int n = 0; n < N; ++n) {
                 const double g0 = rg[gidx<E>(n, q, 0, c)];
                 const double g1 = rg[gidx<E>(n, q, 1, c)];
                 const double g2 = rg[gidx<E>(n, q, 2, c)];
-                const double2 uv = Us[n * TC + c];
+                const double2 uv = Us[c * N + n];
                 ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
                 vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
                 if (have_s) {
-                    const double sn = ss[n * TC + c];
+                    const double sn = ss[c * N + n];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
             }
             qp_tail<E>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy, vz, gs0,
                        gs1);
         }
-        __syncthreads();
+        __syncwarp();
 
-        // ---- phase 2 (+ prefetch of the next tile's gather at q = Q/2) ----
-        const int32_t gnode = rconn[R::conn(i, c2)];
-        double R0, R1;
-        double Jb[N / 2 + 1][2][2];
-        node_accumulate<E, JAC>(rg, qs, c2, i, bfi, R0, R1, Jb, [&]() {
+        // ---- per-node phase (+ gather of the next tile at q = Q/2) ----
+        const int32_t gnode = act ? rconn[R::conn(s, c)] : 0;
+        auto prefetch = [&]() {
             const int64_t nt = tile + gridDim.x;
             if (nt < a.ntiles) {
                 const int ns = (it + 1) % NSTAGE;
                 mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NSTAGE) & 1));
                 issue_gather<E>(smem + ns * S::STAGE, a.U, a.surface, have_s);
             }
-        });
-        __syncthreads();  // everyone is done with this stage's record and qs
+        };
+        double R0 = 0.0, R1 = 0.0;
+        double Jb[N / 2 + 1][2][2];
+        if (act) node_accumulate<E, JAC>(rg, qs, c, s, bfi, R0, R1, Jb, prefetch);
+        else prefetch();
+        __syncwarp();  // every lane is done with this stage's record and qs
 
         if (JAC) {
-            stage_J<E>(reinterpret_cast<double *>(stage), c2, i, Jb);
+            if (act) stage_J<E>(reinterpret_cast<double *>(stage), c, s, Jb);
             fence_proxy_async_smem();
-            __syncthreads();
-            if (t == 0) {
-                store_J<E>(a.J_cell, cell0, nvalid, stage, pol_stream);
-                bulk_wait_read0();  // staging read done -> the buffer may take the next record
+            __syncwarp();
+            if (l == 0) {
+                bulk_s2g(a.J_cell + cell0 * (4 * N * N), stage, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
+                bulk_commit();
+                bulk_wait_read0();  // staging read -> the buffer may take the next record
             }
         }
-        if (t == 0) {
+        if (l == 0) {
             const int64_t nt = tile + (int64_t)NSTAGE * gridDim.x;
             if (nt < a.ntiles) {
                 mbar_arrive_expect_tx(&bar[st], R::BYTES);
                 bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
             }
         }
-        if (c2 < nvalid) {
+        if (act && c < nvalid) {
             if (a.R) {
                 atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
                 atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
             }
-            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c2) * N + i) * 2) = make_double2(R0, R1);
+            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }
     }
-    if (JAC && t == 0) bulk_wait0();
+    if (JAC && l == 0) bulk_wait0();
 }
 
 // ---- G3/G4 with on-the-fly geometry ------------------------------------------
-// Same evaluation, but GradBF and wM are recomputed per tile from the gathered
-// node coordinates instead of being streamed (1,640 -> 40 streamed B/cell for
-// hex8): B200's FP64 rate per HBM byte makes recomputation cheaper than
-// streaming.  Light records (conn + k_c, 640 B per hex8 tile) ride a 4-deep TMA
-// ring; U, s and the coordinates are gathered with cp.async one tile ahead.
-
-constexpr int NLIGHT = 4;
+// Same evaluation; GradBF and wM are recomputed per tile from the gathered
+// node coordinates (cell-local, reading Z17) instead of being streamed: 40
+// streamed B/cell instead of 1,640 (hex8).  conn and k_c are read straight
+// from the caller's arrays one tile ahead; U, s and coordinates are gathered
+// with cp.async one tile ahead.
 
 template <class E, bool JAC>
 struct OtfSmem {
-    static constexpr int N = E::N, Q = E::Q, TC = E::TC;
-    static constexpr int LREC = Rec<E>::LIGHT_BYTES;
-    static constexpr int OFF_L = 0;                                         // NLIGHT light records
-    static constexpr int OFF_IN = OFF_L + NLIGHT * LREC;                    // 2 gathered-input buffers
-    static constexpr int IN_U = 0, IN_XY = N * TC * 16, IN_ZW = 2 * N * TC * 16, IN_S = 3 * N * TC * 16;
-    static constexpr int IN_BYTES = (int)round_up(IN_S + N * TC * 8, 128);
-    static constexpr int OFF_DPHI = OFF_IN + 2 * IN_BYTES;                  // double [Q][N][3]
-    static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * N * 3 * 8, 128);  // GradBF [N][Q][3][TC] (swizzled)
-    static constexpr int OFF_QS = OFF_G + N * Q * 3 * TC * 8;               // double [NQS][Q][TC]
-    static constexpr int G_QS_BYTES = OFF_QS + NQS * Q * TC * 8 - OFF_G;
-    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;            // J staging overlays G + qs
-    static_assert(J_BYTES <= G_QS_BYTES, "J staging must fit over G + qs");
-    static constexpr int OFF_BAR = OFF_QS + NQS * Q * TC * 8;
-    static constexpr int BYTES = OFF_BAR + NLIGHT * 8;
+    static constexpr int N = E::N, Q = E::Q, TC = E::TC, SLAB = E::SLAB;
+    static constexpr int IN_U = 0, IN_XY = TC * N * 16, IN_ZW = 2 * TC * N * 16, IN_S = 3 * TC * N * 16;
+    static constexpr int IN_BYTES = (int)round_up(IN_S + TC * N * 8, 128);  // one gathered-input buffer
+    static constexpr int DPITCH = 3 * N + 1;                                 // odd pitch: conflict-free
+    static constexpr int OFF_DPHI = 2 * IN_BYTES;                            // double [Q][DPITCH]
+    static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * DPITCH * 8, 128);  // GradBF [Q][3][SLAB]
+    static constexpr int OFF_QS = OFF_G + Q * 3 * SLAB * 8;                  // double [NQS][TC][Q]
+    static constexpr int J_BYTES = JAC ? TC * 4 * N * N * 8 : 0;             // J staging overlays G + qs
+    static_assert(J_BYTES <= OFF_QS + NQS * TC * Q * 8 - OFF_G, "J staging must fit over G + qs");
+    static constexpr int BYTES = OFF_QS + NQS * TC * Q * 8;
 };
 
 template <class E>
-__device__ __forceinline__ void issue_gather_otf(char *in, const int32_t *lconn, const double *U,
+__device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live, const double *U,
                                                  const double4 *xyz4, const double *surface, bool have_s) {
     using S = OtfSmem<E, false>;
-    const int t = threadIdx.x;
-    const int c = t % E::TC, n = t / E::TC;
-    const int32_t g = lconn[Rec<E>::conn(n, c)];
-    const int o = (n * E::TC + c) * 16;
-    cp_async16(in + S::IN_U + o, U + 2 * (int64_t)g);
-    cp_async16(in + S::IN_XY + o, reinterpret_cast<const double *>(xyz4 + g));
-    cp_async16(in + S::IN_ZW + o, reinterpret_cast<const double *>(xyz4 + g) + 2);
-    if (have_s) cp_async8(in + S::IN_S + (n * E::TC + c) * 8, surface + g);
+    const int l = threadIdx.x;
+    if (live) {
+        cp_async16(in + S::IN_U + l * 16, U + 2 * (int64_t)g);
+        cp_async16(in + S::IN_XY + l * 16, reinterpret_cast<const double *>(xyz4 + g));
+        cp_async16(in + S::IN_ZW + l * 16, reinterpret_cast<const double *>(xyz4 + g) + 2);
+        if (have_s) cp_async8(in + S::IN_S + l * 8, surface + g);
+    }
     cp_async_commit();
 }
 
 template <class E, bool JAC>
-__global__ void __launch_bounds__(E::TC *E::N, (E::N == 8 ? 3 : 2)) eval_otf_kernel(EvalArgs a) {
+__global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_otf_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
-    static_assert(N == Q, "thread mappings assume N == Q");
-    using R = Rec<E>;
+    static_assert(N == Q, "lane mappings assume N == Q");
     using S = OtfSmem<E, JAC>;
-    static_assert(S::OFF_IN == OtfSmem<E, false>::OFF_IN && S::IN_BYTES == OtfSmem<E, false>::IN_BYTES, "layout");
+    static_assert(S::IN_BYTES == OtfSmem<E, false>::IN_BYTES, "layout");
     extern __shared__ __align__(128) char smem[];
     double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
     double *dphi = reinterpret_cast<double *>(smem + S::OFF_DPHI);
-    uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
-    const int t = threadIdx.x;
+    const int l = threadIdx.x;
+    const int c = l / N, s = l % N;
+    const bool act = c < TC;
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
+    uint64_t pol_stream = 0;
+    if (l == 0) pol_stream = policy_evict_first();
 
     // reference gradients d phi_n / d xi at every QP (shared table)
-    for (int e = t; e < Q * N; e += blockDim.x) {
+    for (int e = l; e < Q * N; e += 32) {
         const int q = e / N, n = e % N;
         double x, y, z, w, phi;
         qp_coords<E>(q, x, y, z, w);
-        basis<E>(n, x, y, z, phi, dphi[e * 3 + 0], dphi[e * 3 + 1], dphi[e * 3 + 2]);
-    }
-    uint64_t pol_stream = 0;
-    if (t == 0) {
-        pol_stream = policy_evict_first();
-        for (int s = 0; s < NLIGHT; ++s) mbar_init(&bar[s], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    if (t == 0) {
-        for (int s = 0; s < NLIGHT; ++s) {
-            const int64_t tile = blockIdx.x + (int64_t)s * gridDim.x;
-            if (tile < a.ntiles) {
-                mbar_arrive_expect_tx(&bar[s], S::LREC);
-                bulk_g2s(smem + S::OFF_L + s * S::LREC, a.recs + tile * (int64_t)S::LREC, S::LREC, &bar[s],
-                         pol_stream);
-            }
-        }
-    }
-    if ((int64_t)blockIdx.x < a.ntiles) {
-        mbar_wait(&bar[0], 0);
-        issue_gather_otf<E>(smem + S::OFF_IN, reinterpret_cast<const int32_t *>(smem + S::OFF_L), a.U, a.xyz4,
-                            a.surface, have_s);
+        basis<E>(n, x, y, z, phi, dphi[q * S::DPITCH + n * 3 + 0], dphi[q * S::DPITCH + n * 3 + 1],
+                 dphi[q * S::DPITCH + n * 3 + 2]);
     }
     double wq;
     {
         double x, y, z;
-        qp_coords<E>(t / TC, x, y, z, wq);
+        qp_coords<E>(act ? s : 0, x, y, z, wq);
     }
-
-    const int c2 = E::NODE_MAJOR_P2 ? t % TC : t / N;
-    const int i = E::NODE_MAJOR_P2 ? t / TC : t % N;
     double bfi[Q];
-    basis_row<E>(i, bfi);
+    basis_row<E>(act ? s : 0, bfi);
+
+    // conn / k_c of a tile, one lane per (cell, node); cells past the end -> node 0
+    auto load_tile = [&](int64_t tile, int32_t &g, double &kcv, bool &live) {
+        const int64_t cell = tile * TC + c;
+        live = act && tile < a.ntiles && cell < a.ncells;
+        g = live ? __ldg(a.conn + cell * N + s) : 0;
+        kcv = live ? (a.kc ? __ldg(a.kc + cell) : a.kscal) : 0.0;
+    };
+    int32_t g_cur, g_nxt;
+    double kc_cur, kc_nxt;
+    bool live_cur, live_nxt;
+    load_tile(blockIdx.x, g_cur, kc_cur, live_cur);
+    load_tile(blockIdx.x + (int64_t)gridDim.x, g_nxt, kc_nxt, live_nxt);
+    __syncwarp();
+    if ((int64_t)blockIdx.x < a.ntiles) issue_gather_otf<E>(smem, g_cur, live_cur, a.U, a.xyz4, a.surface, have_s);
 
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
-        const int sl = it % NLIGHT;
-        const char *lrec = smem + S::OFF_L + sl * S::LREC;
-        const int32_t *lconn = reinterpret_cast<const int32_t *>(lrec + R::CONN_OFF);
-        const double *lkc = reinterpret_cast<const double *>(lrec + R::KC_OFF);
-        const char *in = smem + S::OFF_IN + (it & 1) * S::IN_BYTES;
+        const char *in = smem + (it & 1) * S::IN_BYTES;
         const double2 *Us = reinterpret_cast<const double2 *>(in + S::IN_U);
         const double2 *XY = reinterpret_cast<const double2 *>(in + S::IN_XY);
         const double2 *ZW = reinterpret_cast<const double2 *>(in + S::IN_ZW);
@@ -659,26 +638,26 @@ __global__ void __launch_bounds__(E::TC *E::N, (E::N == 8 ? 3 : 2)) eval_otf_ker
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
 
         cp_async_wait_all();
-        if (JAC && t == 0) bulk_wait_read0();  // previous tile's J staging (over G + qs) has been read
-        __syncthreads();
+        if (JAC && l == 0) bulk_wait_read0();  // previous tile's J staging (over G + qs) has been read
+        __syncwarp();
 
-        // ---- phase 1 (thread <-> (cell, qp)): geometry, GradBF -> smem, then Ugrad etc. ----
-        {
-            const int c = t % TC, q = t / TC;
-            const double *dq = dphi + q * N * 3;
+        // ---- per-QP phase: geometry, GradBF -> smem, then Ugrad etc. ----
+        // k_c of cell c lives in lane c*N (the lane that loaded it)
+        const double kc = __shfl_sync(0xffffffffu, kc_cur, act ? c * N : 0);
+        if (act) {
+            const int q = s;
+            const double *dq = dphi + q * S::DPITCH;
             double J00 = 0, J01 = 0, J02 = 0, J10 = 0, J11 = 0, J12 = 0, J20 = 0, J21 = 0, J22 = 0;
-            // cell-local coordinates x_n - x_0 (see geometry_kernel)
-            const double2 xy0 = XY[c];
-            const double z0 = ZW[c].x;
+            const double2 xy0 = XY[c * N];
+            const double z0 = ZW[c * N].x;
 #pragma unroll
             for (int n = 0; n < N; ++n) {
-                double2 xy = XY[n * TC + c];
-                xy.x -= xy0.x;
-                xy.y -= xy0.y;
-                const double z = ZW[n * TC + c].x - z0;
+                const double2 xy = XY[c * N + n];
+                const double x = xy.x - xy0.x, y = xy.y - xy0.y;  // cell-local (reading Z17)
+                const double z = ZW[c * N + n].x - z0;
                 const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
-                J00 = fma(xy.x, d0, J00); J01 = fma(xy.x, d1, J01); J02 = fma(xy.x, d2, J02);
-                J10 = fma(xy.y, d0, J10); J11 = fma(xy.y, d1, J11); J12 = fma(xy.y, d2, J12);
+                J00 = fma(x, d0, J00); J01 = fma(x, d1, J01); J02 = fma(x, d2, J02);
+                J10 = fma(y, d0, J10); J11 = fma(y, d1, J11); J12 = fma(y, d2, J12);
                 J20 = fma(z, d0, J20); J21 = fma(z, d1, J21); J22 = fma(z, d2, J22);
             }
             // cofactors: (J^-T)[r][s] = cof[r][s] / det
@@ -698,90 +677,63 @@ __global__ void __launch_bounds__(E::TC *E::N, (E::N == 8 ? 3 : 2)) eval_otf_ker
                 rg[gidx<E>(n, q, 0, c)] = g0;
                 rg[gidx<E>(n, q, 1, c)] = g1;
                 rg[gidx<E>(n, q, 2, c)] = g2;
-                const double2 uv = Us[n * TC + c];
+                const double2 uv = Us[c * N + n];
                 ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
                 vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
                 if (have_s) {
-                    const double sn = ss[n * TC + c];
+                    const double sn = ss[c * N + n];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
             }
-            qp_tail<E>(a, qs, c, q, nvalid, cell0, have_s, lkc[c], wq * det, ux, uy, uz, vx, vy, vz, gs0, gs1);
+            qp_tail<E>(a, qs, c, q, nvalid, cell0, have_s, kc, wq * det, ux, uy, uz, vx, vy, vz, gs0, gs1);
         }
-        __syncthreads();
+        __syncwarp();
 
-        // ---- phase 2 (+ prefetch of the next tile's gather at q = Q/2) ----
-        const int32_t gnode = lconn[R::conn(i, c2)];
-        double R0, R1;
-        double Jb[N / 2 + 1][2][2];
-        node_accumulate<E, JAC>(rg, qs, c2, i, bfi, R0, R1, Jb, [&]() {
+        // ---- per-node phase (+ gather of the next tile, load of the one after) ----
+        const int32_t gnode = g_cur;
+        int32_t g_nn = 0;
+        double kc_nn = 0.0;
+        bool live_nn = false;
+        auto prefetch = [&]() {
             const int64_t nt = tile + gridDim.x;
-            if (nt < a.ntiles) {
-                const int ns = (it + 1) % NLIGHT;
-                mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NLIGHT) & 1));
-                issue_gather_otf<E>(smem + S::OFF_IN + ((it + 1) & 1) * S::IN_BYTES,
-                                    reinterpret_cast<const int32_t *>(smem + S::OFF_L + ns * S::LREC), a.U, a.xyz4,
-                                    a.surface, have_s);
-            }
-        });
-        __syncthreads();  // G, qs and this light record are consumed
+            if (nt < a.ntiles)
+                issue_gather_otf<E>(smem + ((it + 1) & 1) * S::IN_BYTES, g_nxt, live_nxt, a.U, a.xyz4, a.surface,
+                                    have_s);
+            load_tile(tile + 2 * (int64_t)gridDim.x, g_nn, kc_nn, live_nn);
+        };
+        double R0 = 0.0, R1 = 0.0;
+        double Jb[N / 2 + 1][2][2];
+        if (act) node_accumulate<E, JAC>(rg, qs, c, s, bfi, R0, R1, Jb, prefetch);
+        else prefetch();
+        __syncwarp();  // G and qs are consumed
 
-        if (t == 0) {  // refill this light-record slot NLIGHT tiles ahead
-            const int64_t nt = tile + (int64_t)NLIGHT * gridDim.x;
-            if (nt < a.ntiles) {
-                mbar_arrive_expect_tx(&bar[sl], S::LREC);
-                bulk_g2s(smem + S::OFF_L + sl * S::LREC, a.recs + nt * (int64_t)S::LREC, S::LREC, &bar[sl],
-                         pol_stream);
+        if (JAC) {
+            if (act) stage_J<E>(rg, c, s, Jb);
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (l == 0) {
+                bulk_s2g(a.J_cell + cell0 * (4 * N * N), rg, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
+                bulk_commit();
             }
         }
-        if (JAC) {
-            stage_J<E>(rg, c2, i, Jb);
-            fence_proxy_async_smem();
-            __syncthreads();
-            if (t == 0) store_J<E>(a.J_cell, cell0, nvalid, smem + S::OFF_G, pol_stream);
-        }
-        if (c2 < nvalid) {
+        if (act && c < nvalid) {
             if (a.R) {
                 atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
                 atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
             }
-            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c2) * N + i) * 2) = make_double2(R0, R1);
+            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }
+        g_cur = g_nxt; kc_cur = kc_nxt; live_cur = live_nxt;
+        g_nxt = g_nn; kc_nxt = kc_nn; live_nxt = live_nn;
     }
-    if (JAC && t == 0) bulk_wait0();
+    if (JAC && l == 0) bulk_wait0();
+    (void)live_cur;
 }
 
-// Setup for the on-the-fly mode: node coordinates as double4, light records
-// (conn + k_c); conn range is checked here, det J at every evaluation.
+// Setup for the on-the-fly mode: node coordinates as double4.
 __global__ void xyz4_kernel(int64_t nnodes, const double *__restrict__ coords, double4 *__restrict__ xyz4) {
     const int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (v < nnodes) xyz4[v] = make_double4(coords[3 * v], coords[3 * v + 1], coords[3 * v + 2], 0.0);
-}
-
-template <class E>
-__global__ void light_record_kernel(int64_t ncells, int64_t nnodes, const int32_t *__restrict__ conn,
-                                    const double *__restrict__ kc_in, double kscal, char *__restrict__ recs,
-                                    int *__restrict__ err) {
-    using R = Rec<E>;
-    constexpr int N = E::N, TC = E::TC;
-    const int64_t cell = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    const int64_t ntiles = (ncells + TC - 1) / TC;
-    if (cell >= ntiles * TC) return;
-    char *rec = recs + (cell / TC) * (int64_t)R::LIGHT_BYTES;
-    const int c = (int)(cell % TC);
-    int32_t *rconn = reinterpret_cast<int32_t *>(rec + R::CONN_OFF);
-    double *rkc = reinterpret_cast<double *>(rec + R::KC_OFF);
-    bool bad = false;
-    for (int n = 0; n < N; ++n) {
-        int32_t g = cell < ncells ? conn[cell * N + n] : 0;
-        if (g < 0 || g >= nnodes) {
-            bad = true;
-            g = 0;
-        }
-        rconn[R::conn(n, c)] = g;
-    }
-    if (bad) atomicOr(err, ERR_CONN);
-    rkc[c] = cell < ncells ? (kc_in ? kc_in[cell] : kscal) : 0.0;
 }
 
 // ---------------------------------------------------------------------------
