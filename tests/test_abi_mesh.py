@@ -42,7 +42,7 @@ def test_strerror_and_create_validation_without_gpu():
     d.num_cells = 10
     n = ctypes.c_size_t()
     assert lib.stokesfo_workspace_size(ctypes.byref(d), ctypes.byref(n)) == 0
-    assert n.value >= 256 + 26240   # header + one hex8 record of 16 cells
+    assert n.value == 256 + 3 * 6560   # header + three hex8 records of 4 cells (10 cells)
     d.glen_n = 2.0
     d.delta = 1e-10
     h = ctypes.c_void_p()
