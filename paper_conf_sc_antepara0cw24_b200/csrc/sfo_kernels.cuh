@@ -509,6 +509,17 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
                 mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NSTAGE) & 1));
                 issue_gather<E>(smem + ns * S::STAGE, a.U, a.surface, have_s);
             }
+            // NSTAGE >= 3: refill the previous tile's stage here, half a tile after
+            // its J bulk store was issued (its SMEM read has long completed)
+            if (NSTAGE >= 3 && l == 0 && it >= 1) {
+                const int ps = (it - 1) % NSTAGE;
+                const int64_t rt = tile + (int64_t)(NSTAGE - 1) * gridDim.x;
+                if (JAC) bulk_wait_read0();
+                if (rt < a.ntiles) {
+                    mbar_arrive_expect_tx(&bar[ps], R::BYTES);
+                    bulk_g2s(smem + ps * S::STAGE, a.recs + rt * (int64_t)R::BYTES, R::BYTES, &bar[ps], pol_stream);
+                }
+            }
         };
         double R0 = 0.0, R1 = 0.0;
         double Jb[N / 2 + 1][2][2];
@@ -523,10 +534,10 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
             if (l == 0) {
                 bulk_s2g(a.J_cell + cell0 * (4 * N * N), stage, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
                 bulk_commit();
-                bulk_wait_read0();  // staging read -> the buffer may take the next record
+                if (NSTAGE < 3) bulk_wait_read0();  // staging read -> the buffer may take the next record
             }
         }
-        if (l == 0) {
+        if (l == 0 && NSTAGE < 3) {
             const int64_t nt = tile + (int64_t)NSTAGE * gridDim.x;
             if (nt < a.ntiles) {
                 mbar_arrive_expect_tx(&bar[st], R::BYTES);
