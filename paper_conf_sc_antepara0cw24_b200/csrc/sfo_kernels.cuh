@@ -411,19 +411,36 @@ struct EvalSmem {
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
 };
 
-// Gather U (16 B) and s (8 B) of one tile through its conn as cp.async copies
-// into the tile's stage buffer (lane <-> (cell, node)).
+// Gather of U (16 B) and s (8 B) of one tile through its conn (lane <->
+// (cell, node)): loaded into registers at the prefetch point (one tile ahead,
+// half a tile of latency slack) and stored to the tile's stage buffer with one
+// conflict-free 16-B shared store per lane (a cp.async gather would cost one
+// shared-memory wavefront per lane: the L1/shared data pipe is the busiest unit).
+struct Gathered {
+    double2 u;
+    double s;
+};
 template <class E>
-__device__ __forceinline__ void issue_gather(char *stage, const double *U, const double *surface, bool have_s) {
+__device__ __forceinline__ Gathered gather_load(const char *stage, const double *U, const double *surface,
+                                                bool have_s) {
     using R = Rec<E>;
-    using S = EvalSmem<E, false>;
+    Gathered v{make_double2(0.0, 0.0), 0.0};
     const int l = threadIdx.x;
     if (l < E::TC * E::N) {
         const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[l];  // conn(n, c) = l
-        cp_async16(stage + S::U_OFF + l * 16, U + 2 * (int64_t)g);
-        if (have_s) cp_async8(stage + S::S_OFF + l * 8, surface + g);
+        v.u = __ldg(reinterpret_cast<const double2 *>(U) + g);
+        if (have_s) v.s = __ldg(surface + g);
     }
-    cp_async_commit();
+    return v;
+}
+template <class E>
+__device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
+    using S = EvalSmem<E, false>;
+    const int l = threadIdx.x;
+    if (l < E::TC * E::N) {
+        reinterpret_cast<double2 *>(stage + S::U_OFF)[l] = v.u;
+        reinterpret_cast<double *>(stage + S::S_OFF)[l] = v.s;
+    }
 }
 
 template <class E, bool JAC, int NSTAGE>
@@ -457,7 +474,7 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
     __syncwarp();
     if ((int64_t)blockIdx.x < a.ntiles) {
         mbar_wait(&bar[0], 0);
-        issue_gather<E>(smem, a.U, a.surface, have_s);
+        gather_store<E>(smem, gather_load<E>(smem, a.U, a.surface, have_s));
     }
     double bfi[Q];
     basis_row<E>(act ? s : 0, bfi);
@@ -475,8 +492,7 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
         const int64_t cell0 = tile * TC;
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
 
-        cp_async_wait_all();  // this lane's gathers for this tile have landed
-        __syncwarp();         // ... and every lane's
+        __syncwarp();  // this tile's gathered U, s (stored by every lane) are visible
 
         // ---- per-QP phase: lane <-> (cell c, qp s) ----
         if (act) {
@@ -502,12 +518,13 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
 
         // ---- per-node phase (+ gather of the next tile at q = Q/2) ----
         const int32_t gnode = act ? rconn[R::conn(s, c)] : 0;
+        const int64_t ntile = tile + gridDim.x;
+        const int nst = (it + 1) % NSTAGE;
+        Gathered nxt{make_double2(0.0, 0.0), 0.0};
         auto prefetch = [&]() {
-            const int64_t nt = tile + gridDim.x;
-            if (nt < a.ntiles) {
-                const int ns = (it + 1) % NSTAGE;
-                mbar_wait(&bar[ns], (uint32_t)(((it + 1) / NSTAGE) & 1));
-                issue_gather<E>(smem + ns * S::STAGE, a.U, a.surface, have_s);
+            if (ntile < a.ntiles) {
+                mbar_wait(&bar[nst], (uint32_t)(((it + 1) / NSTAGE) & 1));
+                nxt = gather_load<E>(smem + nst * S::STAGE, a.U, a.surface, have_s);
             }
             // NSTAGE >= 3: refill the previous tile's stage here, half a tile after
             // its J bulk store was issued (its SMEM read has long completed)
@@ -551,6 +568,7 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
             }
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }
+        if (ntile < a.ntiles) gather_store<E>(smem + nst * S::STAGE, nxt);
     }
     if (JAC && l == 0) bulk_wait0();
 }
