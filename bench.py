@@ -34,7 +34,7 @@ WORKLOADS = {
 }
 
 
-def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored") -> int:
+def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored", op: str = "jacobian") -> int:
     """Algorithmic (compulsory) HBM bytes of one stokesfo_jacobian launch with
     assembled R.
     stored:     per cell conn 4N + GradBF 24NQ + wMeasure 8Q + k_c 8 + J_cell 8(2N)^2;
@@ -43,7 +43,7 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
                 per node U 16 + s 8 + R 32 + coordinates 32 (x, y, z, pad)."""
     N = 8 if elem == "hex8" else 6
     Q = N
-    J = 8 * (2 * N) ** 2
+    J = 8 * (2 * N) ** 2 if op == "jacobian" else 0
     if geometry == "on_the_fly":
         return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32)
     per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + J
@@ -130,7 +130,7 @@ def build_mesh(cfg: str):
 # CPU oracle leg (cpu_baseline and --impl reference)
 # ---------------------------------------------------------------------------
 
-def oracle_sample_rate(elem, conn, coords, U, s, kc, target_s=12.0, start_cell=0):
+def oracle_sample_rate(elem, conn, coords, U, s, kc, target_s=12.0, start_cell=0, mode="jac"):
     """Time the oracle (as it stands) on a bounded contiguous sample of cells;
     geometry precomputed untimed (the GPU contract).  Returns (cells/s, cells, s)."""
     import numpy as np
@@ -141,7 +141,7 @@ def oracle_sample_rate(elem, conn, coords, U, s, kc, target_s=12.0, start_cell=0
         cs = slice(start_cell, start_cell + n)
         G, wm, _ = O.geometry(e, conn[cs], coords)
         t0 = time.perf_counter()
-        O.evaluate(e, conn[cs], G, wm, U, surface=s, kc=kc[cs], mode="jac")
+        O.evaluate(e, conn[cs], G, wm, U, surface=s, kc=kc[cs], mode=mode)
         return time.perf_counter() - t0
 
     n = 4096
@@ -199,6 +199,8 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly"])
+    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid"],
+                    help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid only")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
@@ -231,7 +233,7 @@ def main():
     N = conn.shape[1]
     stream = torch.cuda.current_stream(dev)
     ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream, geometry=args.geometry)
-    J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device=dev)
+    J = torch.empty((C, 2 * N, 2 * N) if args.op == "jacobian" else (0,), dtype=torch.float64, device=dev)
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     halo = None
     if world > 1:
@@ -246,7 +248,10 @@ def main():
         R.zero_()
         if i is not None:
             k0[i].record(stream)
-        ctx.jacobian(U, J, R=R)
+        if args.op == "jacobian":
+            ctx.jacobian(U, J, R=R)
+        else:
+            ctx.viscosity_resid(U, R=R)
         if i is not None:
             k1[i].record(stream)
         if halo is not None:
@@ -310,18 +315,19 @@ def main():
 
     if rank == 0:
         peak, peak_src = load_peaks()
-        bpl = bytes_per_launch(elem, C, NN, args.geometry)
+        bpl = bytes_per_launch(elem, C, NN, args.geometry, args.op)
         achieved = bpl / (kern_ms_max * 1e-3) / 1e9
         traffic = None
         tpath = os.path.join(ROOT, "profiles", "traffic.json")
         if os.path.exists(tpath):
             with open(tpath) as f:
                 tr = json.load(f)
-            key = f"{args.config}:{elem}:jacobian:{args.geometry}"
+            key = f"{args.config}:{elem}:{args.op}:{args.geometry}"
             if key in tr and world == 1:
                 traffic = tr[key]["dram_bytes_per_launch"]
         line = {
-            "metric": METRIC,
+            "metric": METRIC if args.op == "jacobian" else
+            "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s",
             "value": total_cells / (ms_step * 1e-3),
             "unit": "cells/s",
             "n_gpus": world,
@@ -334,14 +340,15 @@ def main():
             "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": WORKLOADS[args.config], "cells": total_cells, "elem": elem, "layers": L,
-                       "geometry": args.geometry,
+                       "geometry": args.geometry, "op": args.op,
                        "cells_rank0": C, "nodes_rank0": NN, "parallelism": f"column-partition x{world}",
                        "l2": "inputs exceed L2 (no flush needed)",
                        "launch": ctx.launch_info()},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel": ("eval_otf_kernel" if args.geometry == "on_the_fly" else "eval_kernel")
-                         + ("<Hex8,true>" if elem == "hex8" else "<Wedge6,true>") + " (stokesfo_jacobian)",
+                         + ("<Hex8," if elem == "hex8" else "<Wedge6,") + ("true>" if args.op == "jacobian" else "false>")
+                         + (" (stokesfo_jacobian)" if args.op == "jacobian" else " (stokesfo_viscosity_resid)"),
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src},
             "achieved_hbm_gbs": achieved,
             "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),
@@ -353,9 +360,11 @@ def main():
                            "note": "pinned U H2D + stokesfo_jacobian + R D2H per step; J_cell stays on device"}
         if world == 1 and not args.no_cpu_baseline:
             import oracle as O
-            rate, n, dt = oracle_sample_rate(elem, conn_g, coords_g, U_g, s_g, kc_g, target_s=12.0)
+            rate, n, dt = oracle_sample_rate(elem, conn_g, coords_g, U_g, s_g, kc_g, target_s=12.0,
+                                             mode="jac" if args.op == "jacobian" else "resid")
+            what = "residual+AD Jacobian" if args.op == "jacobian" else "residual"
             line["cpu_baseline"] = {"value": rate, "unit": "cells/s", "cores": O.num_threads(), "kind": "oracle",
-                                    "sample": f"first {n} cells of {args.config} (residual+AD Jacobian, "
+                                    "sample": f"first {n} cells of {args.config} ({what}, "
                                               f"geometry precomputed untimed), {dt:.1f} s"}
         print(json.dumps(line), flush=True)
     if world > 1:
