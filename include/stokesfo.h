@@ -168,6 +168,31 @@ void stokesfo_destroy(stokesfo_ctx *c);
 int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid_resid,
                          int32_t *grid_jac, int64_t *record_bytes_per_tile);
 
+/* ---------------- NEXT-1: the paper's evaluator chain on B200 -------------- */
+
+/* Albany's unfused chain (SURVEY CS-1) with HBM intermediates, to reproduce
+ * the paper's baseline-vs-optimized experiment (Table III/IV) on
+ * B200:  GatherSolution -> DOFVecGradInterpolation (Ugrad) -> ViscosityFO
+ * (muLandIce) -> StokesFOBodyForce (force) -> StokesFOResid (Fig. 2) ->
+ * Residual.  derivs = 0: ScalarT = double (the Residual kernel); derivs = 1:
+ * ScalarT = value + 2N derivative lanes, Sacado SFad<double,2N> (the Jacobian
+ * kernel).  All intermediates live in a caller-owned device
+ * scratch of stokesfo_albany_scratch_size bytes, component-major with the cell
+ * index fastest (thread-per-cell kernels read coalesced).  The chain derives
+ * the force from desc.surface (force_qp is EUNSUPPORTED here).  Results equal
+ * stokesfo_viscosity_resid / stokesfo_jacobian up to rounding (parity-tested). */
+typedef enum { STOKESFO_FIG2_BASELINE = 0, STOKESFO_FIG2_OPTIMIZED = 1 } stokesfo_fig2_variant_t;
+int stokesfo_albany_scratch_size(stokesfo_ctx *c, int derivs, size_t *bytes);
+/* GradBF, wGradBF = GradBF wM, wBF = BF wM into the scratch (once per mesh). */
+int stokesfo_albany_setup(stokesfo_ctx *c, int derivs, double *scratch);
+/* Gather (seeded), Ugrad, muLandIce, force into the scratch. U: dev [nodes][2]. */
+int stokesfo_albany_evaluators(stokesfo_ctx *c, int derivs, const double *U, double *scratch);
+/* StokesFOResid, Fig. 2 left (BASELINE: global accumulation, two QP passes) or
+ * right column (OPTIMIZED: fused loop, local res0/res1, single store). */
+int stokesfo_albany_resid(stokesfo_ctx *c, int derivs, int variant, double *scratch);
+/* Residual -> R_cell [C][N][2] (opt) and, for derivs = 1, J_cell [C][2N][2N] (opt). */
+int stokesfo_albany_extract(stokesfo_ctx *c, int derivs, const double *scratch, double *R_cell, double *J_cell);
+
 /* ---------------- host-side mesh construction (no GPU needed) ------------- */
 
 /* Extrude a footprint by L uniform-sigma layers:

@@ -11,6 +11,7 @@
 
 #include "../../include/stokesfo.h"
 #include "sfo_kernels.cuh"
+#include "sfo_albany.cuh"
 
 using namespace sfo;
 
@@ -365,6 +366,84 @@ int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid
     if (grid_jac) *grid_jac = (int32_t)std::min<int64_t>(c->grid_jac, std::max<int64_t>(c->ntiles, 1));
     if (record_bytes_per_tile) *record_bytes_per_tile = c->rec_bytes;
     return STOKESFO_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------------------
+// NEXT-1: the paper's evaluator chain (sfo_albany.cuh)
+// ---------------------------------------------------------------------------
+namespace {
+template <class E, int ND>
+int albany_run(stokesfo_ctx *c, int stage, int variant, const double *U, double *S, double *R_cell, double *J_cell) {
+    using namespace sfo::albany;
+    const int64_t C = c->d.num_cells;
+    if (C == 0) return STOKESFO_OK;
+    const int bs = 128;
+    const unsigned gc = (unsigned)((C + bs - 1) / bs);
+    const unsigned gq = (unsigned)((C * E::Q + bs - 1) / bs);
+    switch (stage) {
+        case 0:  // setup: GradBF, wGradBF, wBF
+            geometry_kernel<E, GEO_ALBANY><<<gq, bs, 0, c->stream>>>(C, c->d.num_nodes, c->d.conn, c->d.coords,
+                                                                    nullptr, 0.0, nullptr, S, nullptr, c->err);
+            break;
+        case 1:  // evaluators
+            gather_solution_kernel<E, ND><<<gc, bs, 0, c->stream>>>(C, c->d.conn, U, S);
+            ugrad_kernel<E, ND><<<gq, bs, 0, c->stream>>>(C, S);
+            viscosity_kernel<E, ND><<<gq, bs, 0, c->stream>>>(C, c->d.flow_factor, c->d.k, c->d.delta, S);
+            bodyforce_kernel<E, ND><<<gq, bs, 0, c->stream>>>(C, c->d.conn, c->d.surface, c->d.rho_g, S);
+            break;
+        case 2:  // StokesFOResid (Fig. 2)
+            if (variant == STOKESFO_FIG2_BASELINE)
+                stokesfo_resid_baseline_kernel<E, ND><<<gc, bs, 0, c->stream>>>(C, S);
+            else
+                stokesfo_resid_optimized_kernel<E, ND><<<gc, bs, 0, c->stream>>>(C, S);
+            break;
+        case 3: {  // extract
+            const unsigned gr = (unsigned)((C * 2 * E::N + bs - 1) / bs);
+            extract_kernel<E, ND><<<gr, bs, 0, c->stream>>>(C, S, R_cell, J_cell);
+            break;
+        }
+        default:
+            return STOKESFO_EINVAL;
+    }
+    return cuda_status();
+}
+
+int albany_dispatch(stokesfo_ctx *c, int derivs, int stage, int variant, const double *U, double *S, double *R_cell,
+                    double *J_cell) {
+    if (!c || !S || (derivs != 0 && derivs != 1) || (variant != 0 && variant != 1)) return STOKESFO_EINVAL;
+    if (c->d.force_qp) return STOKESFO_EUNSUPPORTED;  // the chain derives the force from the surface
+    if (c->N == 8)
+        return derivs ? albany_run<Hex8, 16>(c, stage, variant, U, S, R_cell, J_cell)
+                      : albany_run<Hex8, 0>(c, stage, variant, U, S, R_cell, J_cell);
+    return derivs ? albany_run<Wedge6, 12>(c, stage, variant, U, S, R_cell, J_cell)
+                  : albany_run<Wedge6, 0>(c, stage, variant, U, S, R_cell, J_cell);
+}
+}  // namespace
+
+extern "C" {
+
+int stokesfo_albany_scratch_size(stokesfo_ctx *c, int derivs, size_t *bytes) {
+    if (!c || !bytes || (derivs != 0 && derivs != 1)) return STOKESFO_EINVAL;
+    int64_t per;
+    if (c->N == 8) per = derivs ? sfo::albany::Scratch<Hex8, 16>::TOTAL : sfo::albany::Scratch<Hex8, 0>::TOTAL;
+    else per = derivs ? sfo::albany::Scratch<Wedge6, 12>::TOTAL : sfo::albany::Scratch<Wedge6, 0>::TOTAL;
+    *bytes = (size_t)(per * c->d.num_cells * 8);
+    return STOKESFO_OK;
+}
+int stokesfo_albany_setup(stokesfo_ctx *c, int derivs, double *scratch) {
+    return albany_dispatch(c, derivs, 0, 0, nullptr, scratch, nullptr, nullptr);
+}
+int stokesfo_albany_evaluators(stokesfo_ctx *c, int derivs, const double *U, double *scratch) {
+    if (!U) return STOKESFO_EINVAL;
+    return albany_dispatch(c, derivs, 1, 0, U, scratch, nullptr, nullptr);
+}
+int stokesfo_albany_resid(stokesfo_ctx *c, int derivs, int variant, double *scratch) {
+    return albany_dispatch(c, derivs, 2, variant, nullptr, scratch, nullptr, nullptr);
+}
+int stokesfo_albany_extract(stokesfo_ctx *c, int derivs, const double *scratch, double *R_cell, double *J_cell) {
+    return albany_dispatch(c, derivs, 3, 0, nullptr, const_cast<double *>(scratch), R_cell, J_cell);
 }
 
 // CSR pattern: host-side construction from a device->host copy of conn.

@@ -88,8 +88,10 @@ __host__ __device__ __forceinline__ int gidx(int n, int q, int d, int c) {
 //   OUT = GEO_RECORDS: full per-tile records (stored-geometry mode, at create)
 //   OUT = GEO_CANON:   canonical grad_bf [C][N][Q][3], w_measure [C][Q] (export)
 //   OUT = GEO_CHECK:   only the det J > 0 / conn range checks
+//   OUT = GEO_ALBANY:  GradBF, wGradBF, wBF component-major [entry][cell] at
+//                      grad_bf (NEXT-1 scratch, see sfo_albany.cuh)
 // ---------------------------------------------------------------------------
-enum { GEO_RECORDS = 0, GEO_CANON = 1, GEO_CHECK = 2 };
+enum { GEO_RECORDS = 0, GEO_CANON = 1, GEO_CHECK = 2, GEO_ALBANY = 3 };
 
 template <class E, int OUT>
 __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *__restrict__ conn,
@@ -180,9 +182,24 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
 #pragma unroll
         for (int r = 0; r < 3; ++r) {
             const double g = (cof[r][0] * dphi[n][0] + cof[r][1] * dphi[n][1] + cof[r][2] * dphi[n][2]) * idet;
-            if (OUT == GEO_RECORDS) rg[gidx<E>(n, q, r, c)] = g;
-            else if (grad_bf) grad_bf[((cell * N + n) * Q + q) * 3 + r] = g;
+            if (OUT == GEO_RECORDS) {
+                rg[gidx<E>(n, q, r, c)] = g;
+            } else if (OUT == GEO_ALBANY) {
+                grad_bf[((int64_t)(n * Q + q) * 3 + r) * ncells + cell] = g;
+                grad_bf[((int64_t)(N * Q * 3) + (n * Q + q) * 3 + r) * ncells + cell] = g * (wq * det);
+            } else if (grad_bf) {
+                grad_bf[((cell * N + n) * Q + q) * 3 + r] = g;
+            }
         }
+    if (OUT == GEO_ALBANY) {
+#pragma unroll
+        for (int n = 0; n < N; ++n) {
+            double phi, dx, dy, dz;
+            basis<E>(n, xq, yq, zq, phi, dx, dy, dz);
+            grad_bf[((int64_t)(2 * N * Q * 3) + n * Q + q) * ncells + cell] = phi * (wq * det);
+        }
+        return;
+    }
     if (OUT == GEO_RECORDS) rwm[R::wm(q, c)] = wq * det;
     else if (w_measure) w_measure[cell * Q + q] = wq * det;
 }

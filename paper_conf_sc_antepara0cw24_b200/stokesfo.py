@@ -52,7 +52,10 @@ EXPORTS = [
     "stokesfo_halo_pack", "stokesfo_halo_unpack_add", "stokesfo_sync", "stokesfo_strerror",
     "stokesfo_destroy", "stokesfo_launch_info", "stokesfo_mesh_extrude",
     "stokesfo_mesh_partition_columns", "stokesfo_mesh_localize", "stokesfo_mesh_halo_list",
+    "stokesfo_albany_scratch_size", "stokesfo_albany_setup", "stokesfo_albany_evaluators",
+    "stokesfo_albany_resid", "stokesfo_albany_extract",
 ]
+FIG2 = {"baseline": 0, "optimized": 1}
 
 
 def lib_path() -> str:
@@ -89,6 +92,11 @@ def _lib():
         L.stokesfo_mesh_partition_columns.argtypes = [I64, I32, P]
         L.stokesfo_mesh_localize.argtypes = [I32, I64, P, ctypes.POINTER(I64), P, P]
         L.stokesfo_mesh_halo_list.argtypes = [I64, P, I64, P, ctypes.POINTER(I64), P]
+        L.stokesfo_albany_scratch_size.argtypes = [P, ctypes.c_int, ctypes.POINTER(ctypes.c_size_t)]
+        L.stokesfo_albany_setup.argtypes = [P, ctypes.c_int, P]
+        L.stokesfo_albany_evaluators.argtypes = [P, ctypes.c_int, P, P]
+        L.stokesfo_albany_resid.argtypes = [P, ctypes.c_int, ctypes.c_int, P]
+        L.stokesfo_albany_extract.argtypes = [P, ctypes.c_int, P, P, P]
         _LIB = L
     return _LIB
 
@@ -231,6 +239,27 @@ class StokesFO:
 
     def sync(self):
         _check(_lib().stokesfo_sync(self._h), "sync")
+
+    # -- NEXT-1: the paper's evaluator chain (baseline / optimized Fig. 2) -----
+    def albany_scratch(self, derivs: bool):
+        import torch
+        n = ctypes.c_size_t(0)
+        _check(_lib().stokesfo_albany_scratch_size(self._h, int(derivs), ctypes.byref(n)), "albany_scratch_size")
+        return torch.empty(max(int(n.value) // 8, 1), dtype=torch.float64, device=self.device)
+
+    def albany_setup(self, derivs: bool, scratch):
+        _check(_lib().stokesfo_albany_setup(self._h, int(derivs), _ptr(scratch)), "albany_setup")
+
+    def albany_evaluators(self, derivs: bool, U, scratch):
+        _check(_lib().stokesfo_albany_evaluators(self._h, int(derivs), _ptr(U), _ptr(scratch)), "albany_evaluators")
+
+    def albany_resid(self, derivs: bool, variant, scratch):
+        v = FIG2[variant] if isinstance(variant, str) else int(variant)
+        _check(_lib().stokesfo_albany_resid(self._h, int(derivs), v, _ptr(scratch)), "albany_resid")
+
+    def albany_extract(self, derivs: bool, scratch, R_cell=None, J_cell=None):
+        _check(_lib().stokesfo_albany_extract(self._h, int(derivs), _ptr(scratch), _ptr(R_cell), _ptr(J_cell)),
+               "albany_extract")
 
     def launch_info(self):
         tc, gr, gj = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
