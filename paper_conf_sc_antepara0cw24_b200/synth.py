@@ -271,6 +271,8 @@ CONFIGS = {
     "C3": dict(desc="Greenland-like 1-10 km NVB footprint x 10 layers hex8, residual+Jacobian", layers=10,
                elem="hex8"),
     "C4": dict(desc="Antarctica-like 4 km x 10 layers hex8, residual+Jacobian", layers=10, elem="hex8"),
+    "C4p": dict(desc="paper-shaped: Antarctica-like 16 km x 20 layers hex8 (~256K hex per GPU at 4 GPUs, "
+                     "PAPER.md P:L74-82)", layers=20, elem="hex8"),
     "C5": dict(desc="Antarctica-like 4 km x 10 layers wedge6, residual+Jacobian", layers=10, elem="wedge6"),
 }
 
@@ -287,6 +289,8 @@ def make_config(name: str, h: float | None = None):
         fp = greenland_footprint()
     elif name == "C4":
         fp = antarctica_footprint(h=h or 4.0)
+    elif name == "C4p":
+        fp = antarctica_footprint(h=h or 16.0, name="C4p")
     elif name == "C5":
         fp = split_to_triangles(antarctica_footprint(h=h or 4.0), name="C5")
     else:
