@@ -215,10 +215,17 @@ def main():
     from paper_conf_sc_antepara0cw24_b200 import StokesFO
     from paper_conf_sc_antepara0cw24_b200.halo import Halo, LocalPart
 
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # STOKESFO_BENCH_BACKEND=gloo (debug only): ranks may share a GPU and the
+    # halo buffers are staged through host memory; the timed product path is NCCL.
+    backend = os.environ.get("STOKESFO_BENCH_BACKEND", "nccl")
+    gpu = local % max(1, torch.cuda.device_count()) if backend == "gloo" else local
+    torch.cuda.set_device(gpu)
+    dev = torch.device("cuda", gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
 
     fp, L, elem, conn_g, coords_g, U_g, s_g, kc_g = build_mesh(args.config)
     part = LocalPart(conn_g, L, fp.nf, rank, world)
@@ -237,7 +244,8 @@ def main():
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     halo = None
     if world > 1:
-        halo = Halo(part.neighbors, dev, pack=ctx.halo_pack, unpack_add=ctx.halo_unpack_add)
+        halo = Halo(part.neighbors, dev, pack=ctx.halo_pack, unpack_add=ctx.halo_unpack_add,
+                    host_staging=(backend != "nccl"))
     ctx.sync()
     torch.cuda.synchronize(dev)
 

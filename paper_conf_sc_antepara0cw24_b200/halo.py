@@ -45,9 +45,10 @@ class LocalPart:
 class Halo:
     """Grouped halo exchange; `pack(R, idx, buf)` / `unpack_add(buf, idx, R)`."""
 
-    def __init__(self, neighbors: dict, device, pack=None, unpack_add=None, group=None):
+    def __init__(self, neighbors: dict, device, pack=None, unpack_add=None, group=None, host_staging=False):
         import torch
         self.group = group
+        self.host_staging = host_staging  # gloo debug runs: send/recv host copies of the buffers
         self.idx = {r: torch.from_numpy(np.ascontiguousarray(v, dtype=np.int32)).to(device)
                     for r, v in sorted(neighbors.items())}
         self.send = {r: torch.empty((v.numel(), 2), dtype=torch.float64, device=device) for r, v in self.idx.items()}
@@ -65,11 +66,18 @@ class Halo:
             return
         for r, idx in self.idx.items():          # pack everything first
             self.pack(R, idx, self.send[r])
+        send, recv = self.send, self.recv
+        if self.host_staging:
+            send = {r: b.cpu() for r, b in self.send.items()}
+            recv = {r: b.cpu() for r, b in self.recv.items()}
         ops = []
         for r in self.idx:
-            ops.append(dist.P2POp(dist.isend, self.send[r], r, group=self.group))
-            ops.append(dist.P2POp(dist.irecv, self.recv[r], r, group=self.group))
+            ops.append(dist.P2POp(dist.isend, send[r], r, group=self.group))
+            ops.append(dist.P2POp(dist.irecv, recv[r], r, group=self.group))
         for req in dist.batch_isend_irecv(ops):
             req.wait()
+        if self.host_staging:
+            for r in self.idx:
+                self.recv[r].copy_(recv[r])
         for r, idx in self.idx.items():          # then unpack-add
             self.unpack_add(self.recv[r], idx, R)
