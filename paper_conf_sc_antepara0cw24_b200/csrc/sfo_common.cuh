@@ -18,11 +18,28 @@ namespace sfo {
 // ---------------------------------------------------------------------------
 struct Hex8 {
     static constexpr int N = 8, Q = 8, TC = 4, ELEM = 0;
-    static constexpr int SLAB = 32;  // doubles per (qp, dir) slab of GradBF in a record
+    static constexpr int SLAB = 32;        // doubles per (qp, dir) slab of GradBF in a record
+    static constexpr int JPITCH = 4 * N * N;  // J staging pitch per cell = the global image (one bulk store)
+    // lane l <-> (cell l / 8, node-or-qp l % 8): a quarter-warp is one cell
+    __host__ __device__ static constexpr int lane_cell(int l) { return l / N; }
+    __host__ __device__ static constexpr int lane_sub(int l) { return l % N; }
+    __host__ __device__ static constexpr int lane_of(int c, int sub) { return c * N + sub; }
+    // slot of (cell c, node n) in the slab of qp q: both the per-QP loads (fixed n,
+    // lanes over (c,q)) and the per-node loads (fixed q, lanes over (c,j)) hit 16
+    // distinct bank pairs per half-warp
+    __host__ __device__ static constexpr int slot(int c, int n, int q) { return c * N + (n + q) % N; }
 };
 struct Wedge6 {
     static constexpr int N = 6, Q = 6, TC = 5, ELEM = 1;  // 30 active lanes
     static constexpr int SLAB = 30;
+    static constexpr int JPITCH = 4 * N * N + 2;  // odd 16-B pitch: conflict-free staging, per-cell bulk stores
+    // lane l <-> (cell l % 5, node-or-qp l / 5) (node-major), slot (29c + 25n) mod 30:
+    // chosen by a search over affine slot maps with the shared-memory bank model
+    // (per-QP loads 57 vs 108 wavefronts per tile, per-node loads 162 vs 240)
+    __host__ __device__ static constexpr int lane_cell(int l) { return l % TC; }
+    __host__ __device__ static constexpr int lane_sub(int l) { return l / TC; }
+    __host__ __device__ static constexpr int lane_of(int c, int sub) { return sub * TC + c; }
+    __host__ __device__ static constexpr int slot(int c, int n, int) { return (29 * c + 25 * n) % 30; }
 };
 
 __host__ __device__ constexpr int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
@@ -32,10 +49,10 @@ __host__ __device__ constexpr int64_t round_up(int64_t x, int64_t m) { return (x
 //   kc    fp64  [TC]                    Glen prefactor per cell
 //   wm    fp64  [Q][TC]                 w_q det J_q
 //   G     fp64  [Q][3][SLAB]            GradBF; (cell c, node n) of qp q sits at
-//                                       slot c*N + (n + q) mod N
-// The slot rotation makes both the per-QP loads (fixed n, lanes over (c, q))
-// and the per-node loads (fixed q, lanes over (c, j)) hit 16 distinct bank
-// pairs per half-warp for hex8 (bank model in DESIGN.md).  One 1-D TMA bulk
+//                                       slot E::slot(c, n, q) (hex8: c*N + (n+q) mod N)
+// The slot map makes both the per-QP loads (fixed n, lanes over (c, q)) and
+// the per-node loads (fixed q, lanes over (c, j)) conflict-free for hex8
+// (bank model in DESIGN.md).  One 1-D TMA bulk
 // copy moves a whole record (size multiple of 16 B: 6,560 B hex8, 4,736 B wedge6).
 template <class E>
 struct Rec {
@@ -49,9 +66,7 @@ struct Rec {
     // index helpers (in elements of the respective type)
     __host__ __device__ static constexpr int conn(int n, int c) { return c * N + n; }
     __host__ __device__ static constexpr int wm(int q, int c) { return q * TC + c; }
-    __host__ __device__ static constexpr int g(int n, int q, int d, int c) {
-        return (q * 3 + d) * SLAB + c * N + (n + q) % N;
-    }
+    __host__ __device__ static constexpr int g(int n, int q, int d, int c) { return (q * 3 + d) * SLAB + E::slot(c, n, q); }
 };
 
 // Workspace: [0, 256) header (error flag), then ntiles records.

@@ -237,7 +237,7 @@ __global__ void gather_kernel(int64_t ncells, const int32_t *__restrict__ conn, 
 
 // ---------------------------------------------------------------------------
 // G3/G4: fused evaluation.  One CTA = one warp, persistent over tiles of TC
-// cells; lane l <-> (cell l / N, node-or-qp l % N).
+// cells; lane l <-> (cell E::lane_cell(l), node-or-qp E::lane_sub(l)).
 // ---------------------------------------------------------------------------
 struct EvalArgs {
     const char *recs;         // per-tile records (stored-geometry mode)
@@ -379,7 +379,7 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
 template <class E>
 __device__ __forceinline__ void stage_J(double *base, int c2, int i, const double (&Jb)[E::N / 2 + 1][2][2]) {
     constexpr int N = E::N, K = N / 2, LD = 2 * N;
-    double *Jc = base + c2 * (4 * N * N);
+    double *Jc = base + c2 * E::JPITCH;
 #pragma unroll
     for (int k = 0; k <= K; ++k) {
         const int j = (i + k) % N;
@@ -390,6 +390,20 @@ __device__ __forceinline__ void stage_J(double *base, int c2, int i, const doubl
             *reinterpret_cast<double2 *>(Jc + (2 * j + 1) * LD + 2 * i) = make_double2(Jb[k][0][1], Jb[k][1][1]);
         }
     }
+}
+
+// One lane issues the TMA bulk store(s) of a staged tile of element Jacobians
+// (one copy when the staging pitch is the global image, else one per cell).
+template <class E>
+__device__ __forceinline__ void store_J(double *J_cell, int64_t cell0, int nvalid, const char *stage, uint64_t pol) {
+    constexpr int NN = 4 * E::N * E::N;
+    if (E::JPITCH == NN) {
+        bulk_s2g(J_cell + cell0 * NN, stage, (uint32_t)(nvalid * NN * 8), pol);
+    } else {
+        for (int c = 0; c < nvalid; ++c)
+            bulk_s2g(J_cell + (cell0 + c) * NN, stage + c * E::JPITCH * 8, (uint32_t)(NN * 8), pol);
+    }
+    bulk_commit();
 }
 
 template <class E>
@@ -421,7 +435,7 @@ struct EvalSmem {
     static constexpr int U_OFF = (int)round_up(REC, 16);     // double2 [TC][N]
     static constexpr int S_OFF = U_OFF + TC * N * 16;        // double  [TC][N]
     static constexpr int IN_BYTES = S_OFF + TC * N * 8;
-    static constexpr int J_BYTES = JAC ? TC * 4 * N * N * 8 : 0;
+    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
     static constexpr int OFF_QS = NSTAGE * STAGE;            // double [NQS][TC][Q]
     static constexpr int OFF_BAR = (int)round_up(OFF_QS + NQS * TC * Q * 8, 8);
@@ -444,7 +458,8 @@ __device__ __forceinline__ Gathered gather_load(const char *stage, const double 
     Gathered v{make_double2(0.0, 0.0), 0.0};
     const int l = threadIdx.x;
     if (l < E::TC * E::N) {
-        const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[l];  // conn(n, c) = l
+        const int c = E::lane_cell(l), n = E::lane_sub(l);
+        const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[R::conn(n, c)];
         v.u = __ldg(reinterpret_cast<const double2 *>(U) + g);
         if (have_s) v.s = __ldg(surface + g);
     }
@@ -455,8 +470,9 @@ __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
     using S = EvalSmem<E, false>;
     const int l = threadIdx.x;
     if (l < E::TC * E::N) {
-        reinterpret_cast<double2 *>(stage + S::U_OFF)[l] = v.u;
-        reinterpret_cast<double *>(stage + S::S_OFF)[l] = v.s;
+        const int e = E::lane_cell(l) * E::N + E::lane_sub(l);  // [cell][node]
+        reinterpret_cast<double2 *>(stage + S::U_OFF)[e] = v.u;
+        reinterpret_cast<double *>(stage + S::S_OFF)[e] = v.s;
     }
 }
 
@@ -471,8 +487,8 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
     const int l = threadIdx.x;
-    const int c = l / N, s = l % N;  // (cell, node-or-qp)
-    const bool act = c < TC;
+    const bool act = l < TC * N;
+    const int c = act ? E::lane_cell(l) : TC, s = act ? E::lane_sub(l) : 0;  // (cell, node-or-qp)
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
 
     uint64_t pol_stream = 0;
@@ -566,8 +582,7 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
             fence_proxy_async_smem();
             __syncwarp();
             if (l == 0) {
-                bulk_s2g(a.J_cell + cell0 * (4 * N * N), stage, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
-                bulk_commit();
+                store_J<E>(a.J_cell, cell0, nvalid, stage, pol_stream);
                 if (NSTAGE < 3) bulk_wait_read0();  // staging read -> the buffer may take the next record
             }
         }
@@ -606,7 +621,7 @@ struct OtfSmem {
     static constexpr int OFF_DPHI = 2 * IN_BYTES;                            // double [Q][DPITCH]
     static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * DPITCH * 8, 128);  // GradBF [Q][3][SLAB]
     static constexpr int OFF_QS = OFF_G + Q * 3 * SLAB * 8;                  // double [NQS][TC][Q]
-    static constexpr int J_BYTES = JAC ? TC * 4 * N * N * 8 : 0;             // J staging overlays G + qs
+    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;             // J staging overlays G + qs
     static_assert(J_BYTES <= OFF_QS + NQS * TC * Q * 8 - OFF_G, "J staging must fit over G + qs");
     static constexpr int BYTES = OFF_QS + NQS * TC * Q * 8;
 };
@@ -617,10 +632,11 @@ __device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live,
     using S = OtfSmem<E, false>;
     const int l = threadIdx.x;
     if (live) {
-        cp_async16(in + S::IN_U + l * 16, U + 2 * (int64_t)g);
-        cp_async16(in + S::IN_XY + l * 16, reinterpret_cast<const double *>(xyz4 + g));
-        cp_async16(in + S::IN_ZW + l * 16, reinterpret_cast<const double *>(xyz4 + g) + 2);
-        if (have_s) cp_async8(in + S::IN_S + l * 8, surface + g);
+        const int e = E::lane_cell(l) * E::N + E::lane_sub(l);  // [cell][node]
+        cp_async16(in + S::IN_U + e * 16, U + 2 * (int64_t)g);
+        cp_async16(in + S::IN_XY + e * 16, reinterpret_cast<const double *>(xyz4 + g));
+        cp_async16(in + S::IN_ZW + e * 16, reinterpret_cast<const double *>(xyz4 + g) + 2);
+        if (have_s) cp_async8(in + S::IN_S + e * 8, surface + g);
     }
     cp_async_commit();
 }
@@ -636,8 +652,8 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_otf_kernel(EvalArg
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
     double *dphi = reinterpret_cast<double *>(smem + S::OFF_DPHI);
     const int l = threadIdx.x;
-    const int c = l / N, s = l % N;
-    const bool act = c < TC;
+    const bool act = l < TC * N;
+    const int c = act ? E::lane_cell(l) : TC, s = act ? E::lane_sub(l) : 0;
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
     uint64_t pol_stream = 0;
     if (l == 0) pol_stream = policy_evict_first();
@@ -688,8 +704,8 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_otf_kernel(EvalArg
         __syncwarp();
 
         // ---- per-QP phase: geometry, GradBF -> smem, then Ugrad etc. ----
-        // k_c of cell c lives in lane c*N (the lane that loaded it)
-        const double kc = __shfl_sync(0xffffffffu, kc_cur, act ? c * N : 0);
+        // every lane of cell c loaded its k_c; take it from the cell's node-0 lane
+        const double kc = __shfl_sync(0xffffffffu, kc_cur, act ? E::lane_of(c, 0) : 0);
         if (act) {
             const int q = s;
             const double *dq = dphi + q * S::DPITCH;
@@ -757,10 +773,7 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_otf_kernel(EvalArg
             if (act) stage_J<E>(rg, c, s, Jb);
             fence_proxy_async_smem();
             __syncwarp();
-            if (l == 0) {
-                bulk_s2g(a.J_cell + cell0 * (4 * N * N), rg, (uint32_t)(nvalid * 4 * N * N * 8), pol_stream);
-                bulk_commit();
-            }
+            if (l == 0) store_J<E>(a.J_cell, cell0, nvalid, reinterpret_cast<const char *>(rg), pol_stream);
         }
         if (act && c < nvalid) {
             if (a.R) {
