@@ -28,6 +28,9 @@ struct Hex8 {
     // lanes over (c,q)) and the per-node loads (fixed q, lanes over (c,j)) hit 16
     // distinct bank pairs per half-warp
     __host__ __device__ static constexpr int slot(int c, int n, int q) { return c * N + (n + q) % N; }
+    // gathered U/s per (cell, node) and per-QP scalars (f, cell, qp) in shared memory
+    static constexpr int UPITCH = N;
+    __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * TC + c) * Q + q; }
 };
 struct Wedge6 {
     static constexpr int N = 6, Q = 6, TC = 5, ELEM = 1;  // 30 active lanes
@@ -40,6 +43,10 @@ struct Wedge6 {
     __host__ __device__ static constexpr int lane_sub(int l) { return l / TC; }
     __host__ __device__ static constexpr int lane_of(int c, int sub) { return sub * TC + c; }
     __host__ __device__ static constexpr int slot(int c, int n, int) { return (29 * c + 25 * n) % 30; }
+    // odd 16-B cell pitch for the gathered U rows; per-QP scalars qp-major
+    // (lanes (c, q) of the per-QP phase then write consecutive addresses)
+    static constexpr int UPITCH = 7;
+    __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * Q + q) * TC + c; }
 };
 
 __host__ __device__ constexpr int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }

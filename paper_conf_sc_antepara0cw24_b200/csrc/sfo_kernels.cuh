@@ -263,7 +263,7 @@ constexpr int NQS = 9;  // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 b
 // phase writes 32 consecutive doubles, the per-node phase reads broadcasts)
 template <class E>
 __device__ __forceinline__ int qsi(int f, int c, int q) {
-    return (f * E::TC + c) * E::Q + q;
+    return E::qsi(f, c, q);
 }
 
 // ---- shared device pieces ---------------------------------------------------
@@ -416,10 +416,11 @@ __device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
     }
 }
 
-// Resident 1-warp CTAs per SM the register budget is sized for.
-template <class E>
+// Resident 1-warp CTAs per SM the register budget is sized for (12 with the
+// Jacobian accumulators, 16 for the residual-only kernels: <= 128 registers).
+template <class E, bool JAC>
 constexpr int warps_per_sm() {
-    return 12;
+    return JAC ? 12 : 16;
 }
 
 // ---- G3/G4 with stored geometry (the §8(a2) precompute streamed per tile) ----
@@ -432,9 +433,9 @@ template <class E, bool JAC, int NSTAGE = 2>
 struct EvalSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static constexpr int REC = Rec<E>::BYTES;
-    static constexpr int U_OFF = (int)round_up(REC, 16);     // double2 [TC][N]
-    static constexpr int S_OFF = U_OFF + TC * N * 16;        // double  [TC][N]
-    static constexpr int IN_BYTES = S_OFF + TC * N * 8;
+    static constexpr int U_OFF = (int)round_up(REC, 16);     // double2 [TC][UPITCH]
+    static constexpr int S_OFF = U_OFF + TC * E::UPITCH * 16;  // double  [TC][UPITCH]
+    static constexpr int IN_BYTES = S_OFF + TC * E::UPITCH * 8;
     static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
     static constexpr int OFF_QS = NSTAGE * STAGE;            // double [NQS][TC][Q]
@@ -470,14 +471,14 @@ __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
     using S = EvalSmem<E, false>;
     const int l = threadIdx.x;
     if (l < E::TC * E::N) {
-        const int e = E::lane_cell(l) * E::N + E::lane_sub(l);  // [cell][node]
+        const int e = E::lane_cell(l) * E::UPITCH + E::lane_sub(l);  // [cell][node]
         reinterpret_cast<double2 *>(stage + S::U_OFF)[e] = v.u;
         reinterpret_cast<double *>(stage + S::S_OFF)[e] = v.s;
     }
 }
 
 template <class E, bool JAC, int NSTAGE>
-__global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a) {
+__global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "lane mappings assume N == Q");
     using R = Rec<E>;
@@ -536,11 +537,11 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
                 const double g0 = rg[gidx<E>(n, q, 0, c)];
                 const double g1 = rg[gidx<E>(n, q, 1, c)];
                 const double g2 = rg[gidx<E>(n, q, 2, c)];
-                const double2 uv = Us[c * N + n];
+                const double2 uv = Us[c * E::UPITCH + n];
                 ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
                 vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
                 if (have_s) {
-                    const double sn = ss[c * N + n];
+                    const double sn = ss[c * E::UPITCH + n];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
             }
@@ -615,8 +616,9 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_kernel(EvalArgs a)
 template <class E, bool JAC>
 struct OtfSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC, SLAB = E::SLAB;
-    static constexpr int IN_U = 0, IN_XY = TC * N * 16, IN_ZW = 2 * TC * N * 16, IN_S = 3 * TC * N * 16;
-    static constexpr int IN_BYTES = (int)round_up(IN_S + TC * N * 8, 128);  // one gathered-input buffer
+    static constexpr int UP = E::UPITCH;
+    static constexpr int IN_U = 0, IN_XY = TC * UP * 16, IN_ZW = 2 * TC * UP * 16, IN_S = 3 * TC * UP * 16;
+    static constexpr int IN_BYTES = (int)round_up(IN_S + TC * UP * 8, 128);  // one gathered-input buffer
     static constexpr int DPITCH = 3 * N + 1;                                 // odd pitch: conflict-free
     static constexpr int OFF_DPHI = 2 * IN_BYTES;                            // double [Q][DPITCH]
     static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * DPITCH * 8, 128);  // GradBF [Q][3][SLAB]
@@ -632,7 +634,7 @@ __device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live,
     using S = OtfSmem<E, false>;
     const int l = threadIdx.x;
     if (live) {
-        const int e = E::lane_cell(l) * E::N + E::lane_sub(l);  // [cell][node]
+        const int e = E::lane_cell(l) * E::UPITCH + E::lane_sub(l);  // [cell][node]
         cp_async16(in + S::IN_U + e * 16, U + 2 * (int64_t)g);
         cp_async16(in + S::IN_XY + e * 16, reinterpret_cast<const double *>(xyz4 + g));
         cp_async16(in + S::IN_ZW + e * 16, reinterpret_cast<const double *>(xyz4 + g) + 2);
@@ -642,7 +644,7 @@ __device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live,
 }
 
 template <class E, bool JAC>
-__global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_otf_kernel(EvalArgs a) {
+__global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "lane mappings assume N == Q");
     using S = OtfSmem<E, JAC>;
@@ -710,13 +712,13 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_otf_kernel(EvalArg
             const int q = s;
             const double *dq = dphi + q * S::DPITCH;
             double J00 = 0, J01 = 0, J02 = 0, J10 = 0, J11 = 0, J12 = 0, J20 = 0, J21 = 0, J22 = 0;
-            const double2 xy0 = XY[c * N];
-            const double z0 = ZW[c * N].x;
+            const double2 xy0 = XY[c * E::UPITCH];
+            const double z0 = ZW[c * E::UPITCH].x;
 #pragma unroll
             for (int n = 0; n < N; ++n) {
-                const double2 xy = XY[c * N + n];
+                const double2 xy = XY[c * E::UPITCH + n];
                 const double x = xy.x - xy0.x, y = xy.y - xy0.y;  // cell-local (reading Z17)
-                const double z = ZW[c * N + n].x - z0;
+                const double z = ZW[c * E::UPITCH + n].x - z0;
                 const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
                 J00 = fma(x, d0, J00); J01 = fma(x, d1, J01); J02 = fma(x, d2, J02);
                 J10 = fma(y, d0, J10); J11 = fma(y, d1, J11); J12 = fma(y, d2, J12);
@@ -739,11 +741,11 @@ __global__ void __launch_bounds__(32, warps_per_sm<E>()) eval_otf_kernel(EvalArg
                 rg[gidx<E>(n, q, 0, c)] = g0;
                 rg[gidx<E>(n, q, 1, c)] = g1;
                 rg[gidx<E>(n, q, 2, c)] = g2;
-                const double2 uv = Us[c * N + n];
+                const double2 uv = Us[c * E::UPITCH + n];
                 ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
                 vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
                 if (have_s) {
-                    const double sn = ss[c * N + n];
+                    const double sn = ss[c * E::UPITCH + n];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
             }
