@@ -129,6 +129,13 @@ int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, do
  * as above. */
 int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *R_cell, double *R);
 
+/* Matrix-free Jacobian-vector product (NEXT-3, Newton-Krylov operator apply):
+ * Y += J(U) X with J = dR/dU assembled over all cells, computed as the forward
+ * directional derivative of the fused chain along X (no element matrices are
+ * formed); optionally R += R(U) in the same pass.  U, X: dev [num_nodes][2];
+ * Y, R: dev [num_nodes][2] (+=). */
+int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, double *R);
+
 /* Assembly: R[2 conn[c][n] + a] += R_cell[c][n][a] (if R_cell and R are non-NULL)
  * and csr_vals[pos(row, col)] += J_cell[c][k][l] (if J_cell and csr_vals are
  * non-NULL; requires an earlier stokesfo_csr_pattern call with non-NULL rowptr

@@ -24,7 +24,7 @@ struct stokesfo_ctx {
     char *recs;            // device records (full or light)
     double4 *xyz4;         // node coordinates (on-the-fly geometry mode)
     int mode;              // stokesfo_geometry_mode_t
-    int grid_resid, grid_jac;
+    int grid_resid, grid_jac, grid_jvp;
     int rec_bytes;
     int nstage_resid, nstage_jac;  // TMA record ring depth of the eval kernels
     const int64_t *rowptr = nullptr;  // CSR pattern (set by stokesfo_csr_pattern)
@@ -62,10 +62,10 @@ int64_t ws_bytes(int64_t ncells, int64_t nnodes, int mode) {
     return WS_HEADER + ntiles * (int64_t)Rec<E>::BYTES;
 }
 
-template <class E, bool JAC>
+template <class E, int MODE>
 int configure_otf(int *grid) {
-    using S = OtfSmem<E, JAC>;
-    auto fn = eval_otf_kernel<E, JAC>;
+    using S = OtfSmem<E, MODE>;
+    auto fn = eval_otf_kernel<E, MODE>;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES) != cudaSuccess)
         return cuda_status();
     int dev = 0, sms = 0, per_sm = 0;
@@ -77,10 +77,10 @@ int configure_otf(int *grid) {
     return STOKESFO_OK;
 }
 
-template <class E, bool JAC, int NS>
+template <class E, int MODE, int NS>
 int configure_eval(int *grid) {
-    using S = EvalSmem<E, JAC, NS>;
-    auto fn = eval_kernel<E, JAC, NS>;
+    using S = EvalSmem<E, MODE, NS>;
+    auto fn = eval_kernel<E, MODE, NS>;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES) != cudaSuccess)
         return cuda_status();
     int dev = 0, sms = 0, per_sm = 0;
@@ -103,9 +103,11 @@ int create_impl(stokesfo_ctx *c) {
     int st;
     if (otf) {
         c->nstage_resid = c->nstage_jac = 0;
-        st = configure_otf<E, false>(&c->grid_resid);
+        st = configure_otf<E, M_RESID>(&c->grid_resid);
         if (st) return st;
-        st = configure_otf<E, true>(&c->grid_jac);
+        st = configure_otf<E, M_JAC>(&c->grid_jac);
+        if (st) return st;
+        st = configure_otf<E, M_JVP>(&c->grid_jvp);
         if (st) return st;
     } else {
         // ring depth: default per element, STOKESFO_STAGES_{RESID,JAC} override (2 or 3)
@@ -113,10 +115,13 @@ int create_impl(stokesfo_ctx *c) {
         c->nstage_jac = default_stages<E, true>();
         if (const char *e = getenv("STOKESFO_STAGES_RESID")) c->nstage_resid = atoi(e) == 3 ? 3 : 2;
         if (const char *e = getenv("STOKESFO_STAGES_JAC")) c->nstage_jac = atoi(e) == 3 ? 3 : 2;
-        st = c->nstage_resid == 3 ? configure_eval<E, false, 3>(&c->grid_resid)
-                                  : configure_eval<E, false, 2>(&c->grid_resid);
+        st = c->nstage_resid == 3 ? configure_eval<E, M_RESID, 3>(&c->grid_resid)
+                                  : configure_eval<E, M_RESID, 2>(&c->grid_resid);
         if (st) return st;
-        st = c->nstage_jac == 3 ? configure_eval<E, true, 3>(&c->grid_jac) : configure_eval<E, true, 2>(&c->grid_jac);
+        st = c->nstage_jac == 3 ? configure_eval<E, M_JAC, 3>(&c->grid_jac)
+                                : configure_eval<E, M_JAC, 2>(&c->grid_jac);
+        if (st) return st;
+        st = configure_eval<E, M_JVP, 2>(&c->grid_jvp);
         if (st) return st;
     }
     if (cudaMemsetAsync(c->err, 0, sizeof(int), c->stream) != cudaSuccess) return cuda_status();
@@ -139,8 +144,9 @@ int create_impl(stokesfo_ctx *c) {
     return cuda_status();
 }
 
-template <class E, bool JAC>
-int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R, double *J_cell) {
+template <class E, int MODE>
+int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R, double *J_cell,
+              const double *X = nullptr, double *Y = nullptr) {
     if (c->ntiles == 0) return STOKESFO_OK;
     EvalArgs a;
     a.recs = c->recs;
@@ -160,13 +166,17 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.R_cell = R_cell;
     a.R = R;
     a.J_cell = J_cell;
-    const int grid = (int)std::min<int64_t>(JAC ? c->grid_jac : c->grid_resid, c->ntiles);
+    a.X = X;
+    a.Y = Y;
+    const int g = MODE == M_JAC ? c->grid_jac : (MODE == M_JVP ? c->grid_jvp : c->grid_resid);
+    const int grid = (int)std::min<int64_t>(g, c->ntiles);
+    const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_JVP ? 2 : c->nstage_resid);
     if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY)
-        eval_otf_kernel<E, JAC><<<grid, 32, OtfSmem<E, JAC>::BYTES, c->stream>>>(a);
-    else if ((JAC ? c->nstage_jac : c->nstage_resid) == 3)
-        eval_kernel<E, JAC, 3><<<grid, 32, EvalSmem<E, JAC, 3>::BYTES, c->stream>>>(a);
+        eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
+    else if (ns == 3)
+        eval_kernel<E, MODE, 3><<<grid, 32, EvalSmem<E, MODE, 3>::BYTES, c->stream>>>(a);
     else
-        eval_kernel<E, JAC, 2><<<grid, 32, EvalSmem<E, JAC, 2>::BYTES, c->stream>>>(a);
+        eval_kernel<E, MODE, 2><<<grid, 32, EvalSmem<E, MODE, 2>::BYTES, c->stream>>>(a);
     return cuda_status();
 }
 
@@ -262,7 +272,7 @@ int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, do
     const void *ps[] = {mu_qp, R_cell, R};
     for (const void *p : ps)
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
-#define CALL(E) eval_impl<E, false>(c, U, mu_qp, R_cell, R, nullptr)
+#define CALL(E) eval_impl<E, M_RESID>(c, U, mu_qp, R_cell, R, nullptr)
     return DISPATCH(c, CALL);
 #undef CALL
 }
@@ -274,7 +284,17 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
     const void *ps[] = {R_cell, R};
     for (const void *p : ps)
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
-#define CALL(E) eval_impl<E, true>(c, U, nullptr, R_cell, R, J_cell)
+#define CALL(E) eval_impl<E, M_JAC>(c, U, nullptr, R_cell, R, J_cell)
+    return DISPATCH(c, CALL);
+#undef CALL
+}
+
+int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, double *R) {
+    if (!c) return STOKESFO_EINVAL;
+    if (c->d.num_cells == 0) return STOKESFO_OK;
+    if (!U || !X || !Y || !aligned(U, 16) || !aligned(X, 16) || !aligned(Y, 16) || (R && !aligned(R, 16)))
+        return STOKESFO_EINVAL;
+#define CALL(E) eval_impl<E, M_JVP>(c, U, nullptr, nullptr, R, nullptr, X, Y)
     return DISPATCH(c, CALL);
 #undef CALL
 }

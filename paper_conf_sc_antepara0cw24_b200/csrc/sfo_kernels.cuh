@@ -254,10 +254,20 @@ struct EvalArgs {
     double *mu_qp;            // [C][Q] or null
     double *R_cell;           // [C][N][2] or null
     double *R;                // [nodes][2] or null (+=)
-    double *J_cell;           // [C][2N][2N] (JAC)
+    double *J_cell;           // [C][2N][2N] (M_JAC)
+    const double *X;          // [nodes][2] direction (M_JVP)
+    double *Y;                // [nodes][2] += J(U) X (M_JVP)
 };
 
-constexpr int NQS = 9;  // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 beta12, wmu2, gamma, wf0, wf1
+// Evaluation modes of the fused kernels
+enum { M_RESID = 0, M_JAC = 1, M_JVP = 2 };
+// per-(cell, qp) scalars: beta00 beta01 beta02 beta11 beta12, wmu2, gamma, wf0, wf1
+// (+ for M_JVP: dbeta00 dbeta01 dbeta02 dbeta11 dbeta12, gamma * tau)
+constexpr int NQS = 9;
+template <int MODE>
+constexpr int nqs() {
+    return MODE == M_JVP ? 15 : 9;
+}
 
 // per-QP scalar f of (cell c, qp q): [NQS][TC][Q] (qp fastest: the per-QP
 // phase writes 32 consecutive doubles, the per-node phase reads broadcasts)
@@ -272,10 +282,10 @@ __device__ __forceinline__ int qsi(int f, int c, int q) {
 // effective strain rate (Z2), Glen viscosity at n = 3 (Z1, Z3) and the per-QP
 // scalars the per-node phase needs.  beta = B g so that sigma = 2 mu beta gives
 // strs00..strs12 of Fig. 2.
-template <class E>
+template <class E, int MODE = M_RESID>
 __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, int q, int nvalid, int64_t cell0,
                                         bool have_s, double kc, double wm, double ux, double uy, double uz, double vx,
-                                        double vy, double vz, double gs0, double gs1) {
+                                        double vy, double vz, double gs0, double gs1, const double *dg = nullptr) {
     constexpr int Q = E::Q;
     constexpr double P_EXP = -1.0 / 3.0;  // (1 - n) / (2 n) at n = 3
     const double uyvx = uy + vx;
@@ -304,6 +314,19 @@ __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, in
     }
     qs[qsi<E>(7, c, q)] = wf0;
     qs[qsi<E>(8, c, q)] = wf1;
+    if (MODE == M_JVP) {
+        // directional derivative along X: dg = grad of X at the QP; d beta = B dg;
+        // tau = (B g) . dg = d(eps_e^2); d sigma = 2 mu (d beta + p tau beta / (e2 + delta))
+        const double dux = dg[0], duy = dg[1], duz = dg[2], dvx = dg[3], dvy = dg[4], dvz = dg[5];
+        const double b00 = 2.0 * ux + vy, b01 = 0.5 * uyvx, b02 = 0.5 * uz, b11 = ux + 2.0 * vy, b12 = 0.5 * vz;
+        const double tau = b00 * dux + b01 * (duy + dvx) + b02 * duz + b11 * dvy + b12 * dvz;
+        qs[qsi<E>(9, c, q)] = 2.0 * dux + dvy;
+        qs[qsi<E>(10, c, q)] = 0.5 * (duy + dvx);
+        qs[qsi<E>(11, c, q)] = 0.5 * duz;
+        qs[qsi<E>(12, c, q)] = dux + 2.0 * dvy;
+        qs[qsi<E>(13, c, q)] = 0.5 * dvz;
+        qs[qsi<E>(14, c, q)] = wmu2 * P_EXP * (r * r * r) * tau;
+    }
     if (a.mu_qp && c < nvalid) a.mu_qp[(cell0 + c) * Q + q] = mu;
 }
 
@@ -315,12 +338,16 @@ __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, in
 // M_ab = wM 2 mu (B-block (a,b) applied to G_i) + gamma h_(i,a) beta_(b,.)
 // is the exact forward derivative of the chain (seed-sparse Sacado lanes).
 // pf() is called once at q = Q/2 (prefetch hook).
-template <class E, bool JAC, class PF>
+template <class E, int MODE, class PF>
 __device__ __forceinline__ void node_accumulate(const double *rg, const double *qs, int c2, int i, const double *bfi,
-                                                double &R0, double &R1, double (&Jb)[E::N / 2 + 1][2][2], PF pf) {
+                                                double &R0, double &R1, double (&Jb)[E::N / 2 + 1][2][2], double &dR0,
+                                                double &dR1, PF pf) {
     constexpr int N = E::N, Q = E::Q, K = N / 2;
+    constexpr bool JAC = MODE == M_JAC;
     R0 = 0.0;
     R1 = 0.0;
+    dR0 = 0.0;
+    dR1 = 0.0;
     if (JAC) {
 #pragma unroll
         for (int k = 0; k <= K; ++k) Jb[k][0][0] = Jb[k][0][1] = Jb[k][1][0] = Jb[k][1][1] = 0.0;
@@ -341,6 +368,16 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
         const double h1 = fma(gi2, b12, fma(gi1, b11, gi0 * b10));
         R0 = fma(wf0, bfi[q], fma(wmu2, h0, R0));
         R1 = fma(wf1, bfi[q], fma(wmu2, h1, R1));
+        if (MODE == M_JVP) {
+            // dR_(i,a) += wmu2 G_i . dbeta_a + gamma tau h_(i,a)
+            const double d00 = qs[qsi<E>(9, c2, q)], d01 = qs[qsi<E>(10, c2, q)], d02 = qs[qsi<E>(11, c2, q)];
+            const double d11 = qs[qsi<E>(12, c2, q)], d12 = qs[qsi<E>(13, c2, q)];
+            const double gt = qs[qsi<E>(14, c2, q)];
+            const double e0 = fma(gi2, d02, fma(gi1, d01, gi0 * d00));
+            const double e1 = fma(gi2, d12, fma(gi1, d11, gi0 * d01));
+            dR0 = fma(gt, h0, fma(wmu2, e0, dR0));
+            dR1 = fma(gt, h1, fma(wmu2, e1, dR1));
+        }
         if (JAC) {
             const double gam = qs[qsi<E>(6, c2, q)];
             const double gh0 = gam * h0, gh1 = gam * h1;
@@ -418,9 +455,9 @@ __device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
 
 // Resident 1-warp CTAs per SM the register budget is sized for (12 with the
 // Jacobian accumulators, 16 for the residual-only kernels: <= 128 registers).
-template <class E, bool JAC>
+template <class E, int MODE>
 constexpr int warps_per_sm() {
-    return JAC ? 12 : 16;
+    return MODE == M_JAC ? 12 : 16;
 }
 
 // ---- G3/G4 with stored geometry (the §8(a2) precompute streamed per tile) ----
@@ -429,17 +466,18 @@ constexpr int warps_per_sm() {
 // buffer holds [record | gathered U (double2 [TC][N]) | s ([TC][N])]; once the
 // warp has consumed a tile's record, the same buffer stages the tile's element
 // Jacobians (the global image) for one TMA bulk store.
-template <class E, bool JAC, int NSTAGE = 2>
+template <class E, int MODE, int NSTAGE = 2>
 struct EvalSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static constexpr int REC = Rec<E>::BYTES;
     static constexpr int U_OFF = (int)round_up(REC, 16);     // double2 [TC][UPITCH]
     static constexpr int S_OFF = U_OFF + TC * E::UPITCH * 16;  // double  [TC][UPITCH]
-    static constexpr int IN_BYTES = S_OFF + TC * E::UPITCH * 8;
-    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;
+    static constexpr int X_OFF = S_OFF + TC * E::UPITCH * 8;   // double2 [TC][UPITCH] (M_JVP)
+    static constexpr int IN_BYTES = X_OFF + (MODE == M_JVP ? TC * E::UPITCH * 16 : 0);
+    static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
-    static constexpr int OFF_QS = NSTAGE * STAGE;            // double [NQS][TC][Q]
-    static constexpr int OFF_BAR = (int)round_up(OFF_QS + NQS * TC * Q * 8, 8);
+    static constexpr int OFF_QS = NSTAGE * STAGE;            // double [nqs][TC][Q]
+    static constexpr int OFF_BAR = (int)round_up(OFF_QS + nqs<MODE>() * TC * Q * 8, 8);
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
 };
 
@@ -451,39 +489,42 @@ struct EvalSmem {
 struct Gathered {
     double2 u;
     double s;
+    double2 x;
 };
-template <class E>
+template <class E, int MODE>
 __device__ __forceinline__ Gathered gather_load(const char *stage, const double *U, const double *surface,
-                                                bool have_s) {
+                                                bool have_s, const double *X) {
     using R = Rec<E>;
-    Gathered v{make_double2(0.0, 0.0), 0.0};
+    Gathered v{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
     const int l = threadIdx.x;
     if (l < E::TC * E::N) {
         const int c = E::lane_cell(l), n = E::lane_sub(l);
         const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[R::conn(n, c)];
         v.u = __ldg(reinterpret_cast<const double2 *>(U) + g);
         if (have_s) v.s = __ldg(surface + g);
+        if (MODE == M_JVP) v.x = __ldg(reinterpret_cast<const double2 *>(X) + g);
     }
     return v;
 }
-template <class E>
+template <class E, int MODE>
 __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
-    using S = EvalSmem<E, false>;
+    using S = EvalSmem<E, MODE>;
     const int l = threadIdx.x;
     if (l < E::TC * E::N) {
         const int e = E::lane_cell(l) * E::UPITCH + E::lane_sub(l);  // [cell][node]
         reinterpret_cast<double2 *>(stage + S::U_OFF)[e] = v.u;
         reinterpret_cast<double *>(stage + S::S_OFF)[e] = v.s;
+        if (MODE == M_JVP) reinterpret_cast<double2 *>(stage + S::X_OFF)[e] = v.x;
     }
 }
 
-template <class E, bool JAC, int NSTAGE>
-__global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(EvalArgs a) {
+template <class E, int MODE, int NSTAGE>
+__global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP;
     static_assert(N == Q, "lane mappings assume N == Q");
     using R = Rec<E>;
-    using S = EvalSmem<E, JAC, NSTAGE>;
-    static_assert(S::U_OFF == EvalSmem<E, false>::U_OFF && S::S_OFF == EvalSmem<E, false>::S_OFF, "layout");
+    using S = EvalSmem<E, MODE, NSTAGE>;
     extern __shared__ __align__(128) char smem[];
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
@@ -508,7 +549,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
     __syncwarp();
     if ((int64_t)blockIdx.x < a.ntiles) {
         mbar_wait(&bar[0], 0);
-        gather_store<E>(smem, gather_load<E>(smem, a.U, a.surface, have_s));
+        gather_store<E, MODE>(smem, gather_load<E, MODE>(smem, a.U, a.surface, have_s, a.X));
     }
     double bfi[Q];
     basis_row<E>(act ? s : 0, bfi);
@@ -523,6 +564,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
         const double *rg = reinterpret_cast<const double *>(stage + R::G_OFF);
         const double2 *Us = reinterpret_cast<const double2 *>(stage + S::U_OFF);
         const double *ss = reinterpret_cast<const double *>(stage + S::S_OFF);
+        const double2 *Xs = reinterpret_cast<const double2 *>(stage + S::X_OFF);
         const int64_t cell0 = tile * TC;
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
 
@@ -532,6 +574,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
         if (act) {
             const int q = s;
             double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+            double dg[6] = {0, 0, 0, 0, 0, 0};
 #pragma unroll
             for (int n = 0; n < N; ++n) {
                 const double g0 = rg[gidx<E>(n, q, 0, c)];
@@ -544,9 +587,14 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
                     const double sn = ss[c * E::UPITCH + n];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
+                if (JVP) {
+                    const double2 xv = Xs[c * E::UPITCH + n];
+                    dg[0] = fma(xv.x, g0, dg[0]); dg[1] = fma(xv.x, g1, dg[1]); dg[2] = fma(xv.x, g2, dg[2]);
+                    dg[3] = fma(xv.y, g0, dg[3]); dg[4] = fma(xv.y, g1, dg[4]); dg[5] = fma(xv.y, g2, dg[5]);
+                }
             }
-            qp_tail<E>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy, vz, gs0,
-                       gs1);
+            qp_tail<E, MODE>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy, vz,
+                             gs0, gs1, dg);
         }
         __syncwarp();
 
@@ -554,11 +602,11 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
         const int32_t gnode = act ? rconn[R::conn(s, c)] : 0;
         const int64_t ntile = tile + gridDim.x;
         const int nst = (it + 1) % NSTAGE;
-        Gathered nxt{make_double2(0.0, 0.0), 0.0};
+        Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
         auto prefetch = [&]() {
             if (ntile < a.ntiles) {
                 mbar_wait(&bar[nst], (uint32_t)(((it + 1) / NSTAGE) & 1));
-                nxt = gather_load<E>(smem + nst * S::STAGE, a.U, a.surface, have_s);
+                nxt = gather_load<E, MODE>(smem + nst * S::STAGE, a.U, a.surface, have_s, a.X);
             }
             // NSTAGE >= 3: refill the previous tile's stage here, half a tile after
             // its J bulk store was issued (its SMEM read has long completed)
@@ -572,9 +620,9 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
                 }
             }
         };
-        double R0 = 0.0, R1 = 0.0;
+        double R0 = 0.0, R1 = 0.0, dR0 = 0.0, dR1 = 0.0;
         double Jb[N / 2 + 1][2][2];
-        if (act) node_accumulate<E, JAC>(rg, qs, c, s, bfi, R0, R1, Jb, prefetch);
+        if (act) node_accumulate<E, MODE>(rg, qs, c, s, bfi, R0, R1, Jb, dR0, dR1, prefetch);
         else prefetch();
         __syncwarp();  // every lane is done with this stage's record and qs
 
@@ -600,8 +648,12 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
                 atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
             }
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
+            if (JVP) {
+                atomicAdd(a.Y + 2 * (int64_t)gnode + 0, dR0);
+                atomicAdd(a.Y + 2 * (int64_t)gnode + 1, dR1);
+            }
         }
-        if (ntile < a.ntiles) gather_store<E>(smem + nst * S::STAGE, nxt);
+        if (ntile < a.ntiles) gather_store<E, MODE>(smem + nst * S::STAGE, nxt);
     }
     if (JAC && l == 0) bulk_wait0();
 }
@@ -613,25 +665,27 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_kernel(Eval
 // from the caller's arrays one tile ahead; U, s and coordinates are gathered
 // with cp.async one tile ahead.
 
-template <class E, bool JAC>
+template <class E, int MODE>
 struct OtfSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC, SLAB = E::SLAB;
     static constexpr int UP = E::UPITCH;
-    static constexpr int IN_U = 0, IN_XY = TC * UP * 16, IN_ZW = 2 * TC * UP * 16, IN_S = 3 * TC * UP * 16;
+    static constexpr int IN_U = 0, IN_XY = TC * UP * 16, IN_ZW = 2 * TC * UP * 16, IN_X = 3 * TC * UP * 16;
+    static constexpr int IN_S = IN_X + (MODE == M_JVP ? TC * UP * 16 : 0);
     static constexpr int IN_BYTES = (int)round_up(IN_S + TC * UP * 8, 128);  // one gathered-input buffer
     static constexpr int DPITCH = 3 * N + 1;                                 // odd pitch: conflict-free
     static constexpr int OFF_DPHI = 2 * IN_BYTES;                            // double [Q][DPITCH]
     static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * DPITCH * 8, 128);  // GradBF [Q][3][SLAB]
     static constexpr int OFF_QS = OFF_G + Q * 3 * SLAB * 8;                  // double [NQS][TC][Q]
-    static constexpr int J_BYTES = JAC ? TC * E::JPITCH * 8 : 0;             // J staging overlays G + qs
-    static_assert(J_BYTES <= OFF_QS + NQS * TC * Q * 8 - OFF_G, "J staging must fit over G + qs");
-    static constexpr int BYTES = OFF_QS + NQS * TC * Q * 8;
+    static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;   // J staging overlays G + qs
+    static_assert(J_BYTES <= OFF_QS + nqs<MODE>() * TC * Q * 8 - OFF_G, "J staging must fit over G + qs");
+    static constexpr int BYTES = OFF_QS + nqs<MODE>() * TC * Q * 8;
 };
 
-template <class E>
+template <class E, int MODE>
 __device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live, const double *U,
-                                                 const double4 *xyz4, const double *surface, bool have_s) {
-    using S = OtfSmem<E, false>;
+                                                 const double4 *xyz4, const double *surface, bool have_s,
+                                                 const double *X) {
+    using S = OtfSmem<E, MODE>;
     const int l = threadIdx.x;
     if (live) {
         const int e = E::lane_cell(l) * E::UPITCH + E::lane_sub(l);  // [cell][node]
@@ -639,16 +693,17 @@ __device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live,
         cp_async16(in + S::IN_XY + e * 16, reinterpret_cast<const double *>(xyz4 + g));
         cp_async16(in + S::IN_ZW + e * 16, reinterpret_cast<const double *>(xyz4 + g) + 2);
         if (have_s) cp_async8(in + S::IN_S + e * 8, surface + g);
+        if (MODE == M_JVP) cp_async16(in + S::IN_X + e * 16, X + 2 * (int64_t)g);
     }
     cp_async_commit();
 }
 
-template <class E, bool JAC>
-__global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(EvalArgs a) {
+template <class E, int MODE>
+__global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_otf_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "lane mappings assume N == Q");
-    using S = OtfSmem<E, JAC>;
-    static_assert(S::IN_BYTES == OtfSmem<E, false>::IN_BYTES, "layout");
+    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP;
+    using S = OtfSmem<E, MODE>;
     extern __shared__ __align__(128) char smem[];
     double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
     double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
@@ -689,7 +744,8 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(
     load_tile(blockIdx.x, g_cur, kc_cur, live_cur);
     load_tile(blockIdx.x + (int64_t)gridDim.x, g_nxt, kc_nxt, live_nxt);
     __syncwarp();
-    if ((int64_t)blockIdx.x < a.ntiles) issue_gather_otf<E>(smem, g_cur, live_cur, a.U, a.xyz4, a.surface, have_s);
+    if ((int64_t)blockIdx.x < a.ntiles)
+        issue_gather_otf<E, MODE>(smem, g_cur, live_cur, a.U, a.xyz4, a.surface, have_s, a.X);
 
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
@@ -698,6 +754,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(
         const double2 *XY = reinterpret_cast<const double2 *>(in + S::IN_XY);
         const double2 *ZW = reinterpret_cast<const double2 *>(in + S::IN_ZW);
         const double *ss = reinterpret_cast<const double *>(in + S::IN_S);
+        const double2 *Xs = reinterpret_cast<const double2 *>(in + S::IN_X);
         const int64_t cell0 = tile * TC;
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
 
@@ -732,6 +789,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(
             if (!(det > 0.0) && c < nvalid) atomicOr(a.err, ERR_DETJ);
             const double id = 1.0 / det;
             double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+            double dg[6] = {0, 0, 0, 0, 0, 0};
 #pragma unroll
             for (int n = 0; n < N; ++n) {
                 const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
@@ -748,8 +806,14 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(
                     const double sn = ss[c * E::UPITCH + n];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
+                if (JVP) {
+                    const double2 xv = Xs[c * E::UPITCH + n];
+                    dg[0] = fma(xv.x, g0, dg[0]); dg[1] = fma(xv.x, g1, dg[1]); dg[2] = fma(xv.x, g2, dg[2]);
+                    dg[3] = fma(xv.y, g0, dg[3]); dg[4] = fma(xv.y, g1, dg[4]); dg[5] = fma(xv.y, g2, dg[5]);
+                }
             }
-            qp_tail<E>(a, qs, c, q, nvalid, cell0, have_s, kc, wq * det, ux, uy, uz, vx, vy, vz, gs0, gs1);
+            qp_tail<E, MODE>(a, qs, c, q, nvalid, cell0, have_s, kc, wq * det, ux, uy, uz, vx, vy, vz, gs0, gs1,
+                             dg);
         }
         __syncwarp();
 
@@ -761,13 +825,13 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(
         auto prefetch = [&]() {
             const int64_t nt = tile + gridDim.x;
             if (nt < a.ntiles)
-                issue_gather_otf<E>(smem + ((it + 1) & 1) * S::IN_BYTES, g_nxt, live_nxt, a.U, a.xyz4, a.surface,
-                                    have_s);
+                issue_gather_otf<E, MODE>(smem + ((it + 1) & 1) * S::IN_BYTES, g_nxt, live_nxt, a.U, a.xyz4,
+                                          a.surface, have_s, a.X);
             load_tile(tile + 2 * (int64_t)gridDim.x, g_nn, kc_nn, live_nn);
         };
-        double R0 = 0.0, R1 = 0.0;
+        double R0 = 0.0, R1 = 0.0, dR0 = 0.0, dR1 = 0.0;
         double Jb[N / 2 + 1][2][2];
-        if (act) node_accumulate<E, JAC>(rg, qs, c, s, bfi, R0, R1, Jb, prefetch);
+        if (act) node_accumulate<E, MODE>(rg, qs, c, s, bfi, R0, R1, Jb, dR0, dR1, prefetch);
         else prefetch();
         __syncwarp();  // G and qs are consumed
 
@@ -781,6 +845,10 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, JAC>())) eval_otf_kernel(
             if (a.R) {
                 atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
                 atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
+            }
+            if (JVP) {
+                atomicAdd(a.Y + 2 * (int64_t)gnode + 0, dR0);
+                atomicAdd(a.Y + 2 * (int64_t)gnode + 1, dR1);
             }
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }

@@ -53,7 +53,7 @@ EXPORTS = [
     "stokesfo_destroy", "stokesfo_launch_info", "stokesfo_mesh_extrude",
     "stokesfo_mesh_partition_columns", "stokesfo_mesh_localize", "stokesfo_mesh_halo_list",
     "stokesfo_albany_scratch_size", "stokesfo_albany_setup", "stokesfo_albany_evaluators",
-    "stokesfo_albany_resid", "stokesfo_albany_extract",
+    "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp",
 ]
 FIG2 = {"baseline": 0, "optimized": 1}
 
@@ -76,6 +76,7 @@ def _lib():
         L.stokesfo_gather.argtypes = [P, P, P]
         L.stokesfo_viscosity_resid.argtypes = [P, P, P, P, P]
         L.stokesfo_jacobian.argtypes = [P, P, P, P, P]
+        L.stokesfo_jvp.argtypes = [P, P, P, P, P]
         L.stokesfo_scatter_assemble.argtypes = [P, P, P, P, P]
         L.stokesfo_csr_pattern.argtypes = [P, ctypes.POINTER(I64), P, P]
         L.stokesfo_geometry.argtypes = [P, P, P]
@@ -206,6 +207,14 @@ class StokesFO:
         _dev(R_cell, torch.float64, (self.num_cells, self.N, 2), "R_cell")
         _dev(R, torch.float64, (self.num_nodes, 2), "R")
         _check(_lib().stokesfo_jacobian(self._h, _ptr(U), _ptr(J_cell), _ptr(R_cell), _ptr(R)), "jacobian")
+
+    def jvp(self, U, X, Y, R=None):
+        """Y += J(U) X (matrix-free, no element matrices); optionally R += R(U)."""
+        import torch
+        for t, n in ((U, "U"), (X, "X"), (Y, "Y")):
+            _dev(t, torch.float64, (self.num_nodes, 2), n)
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_jvp(self._h, _ptr(U), _ptr(X), _ptr(Y), _ptr(R)), "jvp")
 
     def csr_pattern(self):
         import torch

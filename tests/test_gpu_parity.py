@@ -279,3 +279,34 @@ def test_edge_cases_and_errors(torch, geometry):
     st = lib.stokesfo_jacobian(ctx1._h, ctypes.c_void_p(_t(torch, U).data_ptr()),
                                ctypes.c_void_p(big.data_ptr() + 8), None, None)
     assert st == 1
+
+
+@pytest.mark.parametrize("geometry", GEOMS)
+@pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 7)])
+def test_jvp_matrix_free_parity(torch, elem, drop, geometry):
+    """NEXT-3: Y += J(U) X computed matrix-free (directional derivative of the
+    fused chain) equals the oracle's assembled AD Jacobian applied to X; the
+    residual of the same pass equals the oracle residual."""
+    ctx, orc = _setup(torch, elem, drop=drop, geometry=geometry)
+    nn = ctx.num_nodes
+    X = np.random.default_rng(77).normal(0, 30.0, (nn, 2))
+    Y = torch.zeros((nn, 2), dtype=torch.float64, device="cuda")
+    R = torch.zeros((nn, 2), dtype=torch.float64, device="cuda")
+    ctx.jvp(_t(torch, orc["U"]), _t(torch, X), Y, R=R)
+    ctx.sync()
+    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
+                     mode="jac")
+    C, N = orc["conn"].shape
+    Xc = X[orc["conn"]].reshape(C, 2 * N)
+    JX = np.einsum("ckl,cl->ck", ref["J_cell"], Xc).reshape(C, N, 2)
+    # per-entry bound: element tolerance (1e-12 of max|J_c| |X_c|) summed over contributing cells
+    scale_c = (np.abs(ref["J_cell"]).reshape(C, -1).max(1) * np.abs(Xc).sum(1))[:, None, None] * np.ones((C, N, 2))
+    Yref = O.scatter(orc["e"], orc["conn"], JX, nn)
+    Yscale = O.scatter(orc["e"], orc["conn"], scale_c, nn)
+    assert (np.abs(Y.cpu().numpy() - Yref) <= TOL * Yscale).all()
+    _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
+    # linearity in X: J(U)(2X) = 2 J(U) X (bitwise up to the atomics' order -> 1e-15)
+    Y2 = torch.zeros((nn, 2), dtype=torch.float64, device="cuda")
+    ctx.jvp(_t(torch, orc["U"]), _t(torch, 2 * X), Y2)
+    ctx.sync()
+    assert torch.allclose(Y2, 2 * Y, rtol=1e-14, atol=1e-14 * float(Y.abs().max()))
