@@ -44,10 +44,11 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
     N = 8 if elem == "hex8" else 6
     Q = N
     J = 8 * (2 * N) ** 2 if op == "jacobian" else 0
+    xy = (16 + 32) if op == "jvp" else 0  # X gather, Y read+write
     if geometry == "on_the_fly":
-        return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32)
+        return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32 + xy)
     per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + J
-    return cells * per_cell + nodes * (16 + 8 + 32)
+    return cells * per_cell + nodes * (16 + 8 + 32 + xy)
 
 
 def load_peaks():
@@ -199,8 +200,9 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly"])
-    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid"],
-                    help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid only")
+    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp"],
+                    help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
+                         "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
@@ -241,6 +243,8 @@ def main():
     stream = torch.cuda.current_stream(dev)
     ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream, geometry=args.geometry)
     J = torch.empty((C, 2 * N, 2 * N) if args.op == "jacobian" else (0,), dtype=torch.float64, device=dev)
+    Xd = torch.from_numpy(np.random.default_rng(5).normal(0, 10.0, (NN, 2))).to(dev) if args.op == "jvp" else None
+    Yd = torch.zeros((NN, 2), dtype=torch.float64, device=dev) if args.op == "jvp" else None
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     halo = None
     if world > 1:
@@ -258,6 +262,8 @@ def main():
             k0[i].record(stream)
         if args.op == "jacobian":
             ctx.jacobian(U, J, R=R)
+        elif args.op == "jvp":
+            ctx.jvp(U, Xd, Yd, R=R)
         else:
             ctx.viscosity_resid(U, R=R)
         if i is not None:
@@ -333,9 +339,11 @@ def main():
             key = f"{args.config}:{elem}:{args.op}:{args.geometry}"
             if key in tr and world == 1:
                 traffic = tr[key]["dram_bytes_per_launch"]
+        l2_bytes = 126 * 2 ** 20
         line = {
-            "metric": METRIC if args.op == "jacobian" else
-            "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s",
+            "metric": METRIC if args.op == "jacobian" else (
+                "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s" if args.op == "resid"
+                else "Stokes-FO matrix-free J(U)X + residual (stokesfo_jvp) cells/s and achieved HBM GB/s"),
             "value": total_cells / (ms_step * 1e-3),
             "unit": "cells/s",
             "n_gpus": world,
@@ -350,13 +358,16 @@ def main():
             "config": {"workload": WORKLOADS[args.config], "cells": total_cells, "elem": elem, "layers": L,
                        "geometry": args.geometry, "op": args.op,
                        "cells_rank0": C, "nodes_rank0": NN, "parallelism": f"column-partition x{world}",
-                       "l2": "inputs exceed L2 (no flush needed)",
+                       "l2": "inputs exceed L2 (no flush needed)" if bpl > 4 * l2_bytes
+                       else "inputs fit in L2 (not flushed; small-config line)",
                        "launch": ctx.launch_info()},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel": ("eval_otf_kernel" if args.geometry == "on_the_fly" else "eval_kernel")
-                         + ("<Hex8," if elem == "hex8" else "<Wedge6,") + ("true>" if args.op == "jacobian" else "false>")
-                         + (" (stokesfo_jacobian)" if args.op == "jacobian" else " (stokesfo_viscosity_resid)"),
+                         + ("<Hex8," if elem == "hex8" else "<Wedge6,")
+                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>"}[args.op]
+                         + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
+                            "jvp": " (stokesfo_jvp)"}[args.op],
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src},
             "achieved_hbm_gbs": achieved,
             "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),
@@ -369,8 +380,8 @@ def main():
         if world == 1 and not args.no_cpu_baseline:
             import oracle as O
             rate, n, dt = oracle_sample_rate(elem, conn_g, coords_g, U_g, s_g, kc_g, target_s=12.0,
-                                             mode="jac" if args.op == "jacobian" else "resid")
-            what = "residual+AD Jacobian" if args.op == "jacobian" else "residual"
+                                             mode="resid" if args.op == "resid" else "jac")
+            what = "residual" if args.op == "resid" else "residual+AD Jacobian"
             line["cpu_baseline"] = {"value": rate, "unit": "cells/s", "cores": O.num_threads(), "kind": "oracle",
                                     "sample": f"first {n} cells of {args.config} ({what}, "
                                               f"geometry precomputed untimed), {dt:.1f} s"}
