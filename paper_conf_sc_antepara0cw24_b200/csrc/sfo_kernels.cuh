@@ -472,13 +472,14 @@ struct EvalSmem {
     static constexpr int REC = Rec<E>::BYTES;
     static constexpr int U_OFF = (int)round_up(REC, 16);     // double2 [TC][UPITCH]
     static constexpr int S_OFF = U_OFF + TC * E::UPITCH * 16;  // double  [TC][UPITCH]
-    static constexpr int X_OFF = S_OFF + TC * E::UPITCH * 8;   // double2 [TC][UPITCH] (M_JVP)
+    static constexpr int X_OFF = (int)round_up(S_OFF + TC * E::UPITCH * 8, 16);  // double2 [TC][UPITCH] (M_JVP)
     static constexpr int IN_BYTES = X_OFF + (MODE == M_JVP ? TC * E::UPITCH * 16 : 0);
     static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
     static constexpr int OFF_QS = NSTAGE * STAGE;            // double [nqs][TC][Q]
     static constexpr int OFF_BAR = (int)round_up(OFF_QS + nqs<MODE>() * TC * Q * 8, 8);
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
+    static_assert(U_OFF % 16 == 0 && X_OFF % 16 == 0 && STAGE % 128 == 0 && OFF_QS % 16 == 0, "alignment");
 };
 
 // Gather of U (16 B) and s (8 B) of one tile through its conn (lane <->
@@ -679,6 +680,7 @@ struct OtfSmem {
     static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;   // J staging overlays G + qs
     static_assert(J_BYTES <= OFF_QS + nqs<MODE>() * TC * Q * 8 - OFF_G, "J staging must fit over G + qs");
     static constexpr int BYTES = OFF_QS + nqs<MODE>() * TC * Q * 8;
+    static_assert(IN_X % 16 == 0 && IN_BYTES % 128 == 0 && OFF_G % 128 == 0 && OFF_QS % 16 == 0, "alignment");
 };
 
 template <class E, int MODE>
