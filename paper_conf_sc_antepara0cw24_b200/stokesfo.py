@@ -59,15 +59,16 @@ FIG2 = {"baseline": 0, "optimized": 1}
 
 
 def lib_path() -> str:
-    return _build.LIB
+    # STOKESFO_LIB: load another build of the same ABI (same-box A/B measurements)
+    return os.environ.get("STOKESFO_LIB", _build.LIB)
 
 
 def _lib():
     """Load libstokesfo.so (building it in-tree with nvcc if absent)."""
     global _LIB
     if _LIB is None:
-        path = _build.LIB
-        if not os.path.exists(path):
+        path = lib_path()
+        if path == _build.LIB and not os.path.exists(path):
             _build.build()
         L = ctypes.CDLL(path)
         P, I64, I32, D = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_double
@@ -76,7 +77,8 @@ def _lib():
         L.stokesfo_gather.argtypes = [P, P, P]
         L.stokesfo_viscosity_resid.argtypes = [P, P, P, P, P]
         L.stokesfo_jacobian.argtypes = [P, P, P, P, P]
-        L.stokesfo_jvp.argtypes = [P, P, P, P, P]
+        if hasattr(L, "stokesfo_jvp"):  # absent only in older builds loaded via STOKESFO_LIB
+            L.stokesfo_jvp.argtypes = [P, P, P, P, P]
         L.stokesfo_scatter_assemble.argtypes = [P, P, P, P, P]
         L.stokesfo_csr_pattern.argtypes = [P, ctypes.POINTER(I64), P, P]
         L.stokesfo_geometry.argtypes = [P, P, P]
