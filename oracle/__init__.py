@@ -10,6 +10,7 @@ Contents:
   oracle.c      plain C fp64: reference elements, geometry, residual (both
                 Fig. 2 loop orders), forward-AD Jacobian, closed-form tangent,
                 gather, scatter, CSR scatter.
+  basal.py      numpy basal-friction side-set term (NEXT-4, reading Z18)
   ref.py        ctypes wrapper of oracle.c + numpy O1 extrusion, O9 CSR
                 pattern / partition / halo lists, and a numpy complex-step
                 residual used as an independent derivative pin.
