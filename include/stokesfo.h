@@ -136,6 +136,15 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
  * Y, R: dev [num_nodes][2] (+=). */
 int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, double *R);
 
+/* Basal friction side-set term (NEXT-4; P:L59 -> [24]; reading Z18):
+ * on the bottom face of each listed basal cell (local nodes 0..3 hex8 /
+ * 0..2 wedge6), R[2 node_i + a] += int beta_h u_h,a phi_i dGamma and
+ * J_face[f][(i,a)][(j,b)] = delta_ab int beta_h phi_i phi_j dGamma (row-major
+ * [2NB][2NB], NB = 4 / 3; optional).  basal_cells: dev int32 [nfaces] cell
+ * ids; beta: dev [num_nodes] friction coefficient; U, R: dev [num_nodes][2]. */
+int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nfaces, const double *beta,
+                            const double *U, double *R, double *J_face);
+
 /* Assembly: R[2 conn[c][n] + a] += R_cell[c][n][a] (if R_cell and R are non-NULL)
  * and csr_vals[pos(row, col)] += J_cell[c][k][l] (if J_cell and csr_vals are
  * non-NULL; requires an earlier stokesfo_csr_pattern call with non-NULL rowptr

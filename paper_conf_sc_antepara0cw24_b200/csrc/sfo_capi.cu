@@ -299,6 +299,23 @@ int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, d
 #undef CALL
 }
 
+int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nfaces, const double *beta,
+                            const double *U, double *R, double *J_face) {
+    if (!c || nfaces < 0) return STOKESFO_EINVAL;
+    if (nfaces == 0) return STOKESFO_OK;
+    if (!basal_cells || !beta || !U || !R || !aligned(U, 16) || !aligned(R, 16) || (J_face && !aligned(J_face, 16)))
+        return STOKESFO_EINVAL;
+    const int bs = 128;
+    const unsigned g = (unsigned)((nfaces + bs - 1) / bs);
+    if (c->N == 8)
+        basal_friction_kernel<Hex8><<<g, bs, 0, c->stream>>>(nfaces, basal_cells, c->d.conn, c->d.coords, beta, U, R,
+                                                              J_face);
+    else
+        basal_friction_kernel<Wedge6><<<g, bs, 0, c->stream>>>(nfaces, basal_cells, c->d.conn, c->d.coords, beta, U,
+                                                                R, J_face);
+    return cuda_status();
+}
+
 int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, const double *J_cell,
                               double *csr_vals) {
     if (!c) return STOKESFO_EINVAL;

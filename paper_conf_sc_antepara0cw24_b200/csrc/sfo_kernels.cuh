@@ -868,6 +868,111 @@ __global__ void xyz4_kernel(int64_t nnodes, const double *__restrict__ coords, d
 }
 
 // ---------------------------------------------------------------------------
+// NEXT-4: basal friction side-set term (PAPER.md P:L59 -> [24]; reading Z18).
+// Bed = bottom face of each listed basal cell (local nodes 0..NB-1).  Thread
+// <-> face: face QPs (2x2 Gauss / 3-point triangle), surface measure
+// |dx/dxi x dx/deta| in face-local coordinates, beta_h and u_h interpolated
+// with the face basis; R += int beta u phi_i, J_face = delta_ab int beta phi_i phi_j.
+// ---------------------------------------------------------------------------
+template <int NB>
+__device__ __forceinline__ void face_basis(int q, double &w, double (&phi)[NB], double (&dxi)[NB], double (&deta)[NB]) {
+    if (NB == 4) {
+        const double g = 1.0 / sqrt(3.0);
+        const double x = (q & 1) ? g : -g, y = (q & 2) ? g : -g;
+        w = 1.0;
+#pragma unroll
+        for (int n = 0; n < NB; ++n) {
+            const double sx = (n == 1 || n == 2) ? 1.0 : -1.0, sy = (n >= 2) ? 1.0 : -1.0;
+            phi[n] = 0.25 * (1.0 + sx * x) * (1.0 + sy * y);
+            dxi[n] = 0.25 * sx * (1.0 + sy * y);
+            deta[n] = 0.25 * (1.0 + sx * x) * sy;
+        }
+    } else {
+        const double x = (q == 1) ? 2.0 / 3.0 : 1.0 / 6.0, y = (q == 2) ? 2.0 / 3.0 : 1.0 / 6.0;
+        w = 1.0 / 6.0;
+        const double l[3] = {1.0 - x - y, x, y}, lx[3] = {-1.0, 1.0, 0.0}, ly[3] = {-1.0, 0.0, 1.0};
+#pragma unroll
+        for (int n = 0; n < NB; ++n) {
+            phi[n] = l[n];
+            dxi[n] = lx[n];
+            deta[n] = ly[n];
+        }
+    }
+}
+
+template <class E>
+__global__ void basal_friction_kernel(int64_t nfaces, const int32_t *__restrict__ cells, const int32_t *__restrict__ conn,
+                                      const double *__restrict__ coords, const double *__restrict__ beta,
+                                      const double *__restrict__ U, double *__restrict__ R, double *__restrict__ Jf) {
+    constexpr int N = E::N, NB = N / 2, NQF = NB == 4 ? 4 : 3, ND = 2 * NB;
+    const int64_t f = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (f >= nfaces) return;
+    const int64_t cell = cells[f];
+    int32_t nid[NB];
+    double x[NB][3], b[NB], u[NB][2];
+#pragma unroll
+    for (int n = 0; n < NB; ++n) {
+        nid[n] = conn[cell * N + n];
+        b[n] = beta[nid[n]];
+        u[n][0] = U[2 * (int64_t)nid[n]];
+        u[n][1] = U[2 * (int64_t)nid[n] + 1];
+    }
+#pragma unroll
+    for (int n = 0; n < NB; ++n)
+#pragma unroll
+        for (int r = 0; r < 3; ++r) x[n][r] = coords[3 * (int64_t)nid[n] + r] - coords[3 * (int64_t)nid[0] + r];
+    double Rf[NB][2] = {};
+    double M[NB][NB] = {};
+#pragma unroll
+    for (int q = 0; q < NQF; ++q) {
+        double w, phi[NB], dxi[NB], deta[NB];
+        face_basis<NB>(q, w, phi, dxi, deta);
+        double t0[3] = {0, 0, 0}, t1[3] = {0, 0, 0};
+#pragma unroll
+        for (int n = 0; n < NB; ++n)
+#pragma unroll
+            for (int r = 0; r < 3; ++r) {
+                t0[r] = fma(x[n][r], dxi[n], t0[r]);
+                t1[r] = fma(x[n][r], deta[n], t1[r]);
+            }
+        const double cx = t0[1] * t1[2] - t0[2] * t1[1], cy = t0[2] * t1[0] - t0[0] * t1[2],
+                     cz = t0[0] * t1[1] - t0[1] * t1[0];
+        const double ds = sqrt(cx * cx + cy * cy + cz * cz) * w;
+        double bq = 0.0, u0 = 0.0, u1 = 0.0;
+#pragma unroll
+        for (int n = 0; n < NB; ++n) {
+            bq = fma(b[n], phi[n], bq);
+            u0 = fma(u[n][0], phi[n], u0);
+            u1 = fma(u[n][1], phi[n], u1);
+        }
+        const double wb = ds * bq;
+#pragma unroll
+        for (int i = 0; i < NB; ++i) {
+            Rf[i][0] = fma(wb * u0, phi[i], Rf[i][0]);
+            Rf[i][1] = fma(wb * u1, phi[i], Rf[i][1]);
+#pragma unroll
+            for (int j = 0; j < NB; ++j) M[i][j] = fma(wb * phi[i], phi[j], M[i][j]);
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < NB; ++i) {
+        atomicAdd(R + 2 * (int64_t)nid[i], Rf[i][0]);
+        atomicAdd(R + 2 * (int64_t)nid[i] + 1, Rf[i][1]);
+    }
+    if (Jf) {
+        double *J = Jf + f * ND * ND;
+#pragma unroll
+        for (int i = 0; i < NB; ++i)
+#pragma unroll
+            for (int a = 0; a < 2; ++a)
+#pragma unroll
+                for (int j = 0; j < NB; ++j)
+#pragma unroll
+                    for (int bb = 0; bb < 2; ++bb) J[(2 * i + a) * ND + 2 * j + bb] = (a == bb) ? M[i][j] : 0.0;
+    }
+}
+
+// ---------------------------------------------------------------------------
 // G5: assembly.  R part: thread <-> (cell, node).  CSR part: thread <-> (cell, row).
 // ---------------------------------------------------------------------------
 template <int N>

@@ -53,7 +53,7 @@ EXPORTS = [
     "stokesfo_destroy", "stokesfo_launch_info", "stokesfo_mesh_extrude",
     "stokesfo_mesh_partition_columns", "stokesfo_mesh_localize", "stokesfo_mesh_halo_list",
     "stokesfo_albany_scratch_size", "stokesfo_albany_setup", "stokesfo_albany_evaluators",
-    "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp",
+    "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp", "stokesfo_basal_friction",
 ]
 FIG2 = {"baseline": 0, "optimized": 1}
 
@@ -79,6 +79,8 @@ def _lib():
         L.stokesfo_jacobian.argtypes = [P, P, P, P, P]
         if hasattr(L, "stokesfo_jvp"):  # absent only in older builds loaded via STOKESFO_LIB
             L.stokesfo_jvp.argtypes = [P, P, P, P, P]
+        if hasattr(L, "stokesfo_basal_friction"):
+            L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
         L.stokesfo_scatter_assemble.argtypes = [P, P, P, P, P]
         L.stokesfo_csr_pattern.argtypes = [P, ctypes.POINTER(I64), P, P]
         L.stokesfo_geometry.argtypes = [P, P, P]
@@ -217,6 +219,17 @@ class StokesFO:
             _dev(t, torch.float64, (self.num_nodes, 2), n)
         _dev(R, torch.float64, (self.num_nodes, 2), "R")
         _check(_lib().stokesfo_jvp(self._h, _ptr(U), _ptr(X), _ptr(Y), _ptr(R)), "jvp")
+
+    def basal_friction(self, basal_cells, beta, U, R, J_face=None):
+        """R += basal friction term on the bottom faces of basal_cells (int32 cuda);
+        optional J_face [nfaces][2NB][2NB] (NB = 4 hex8 / 3 wedge6)."""
+        import torch
+        _dev(basal_cells, torch.int32, None, "basal_cells")
+        _dev(beta, torch.float64, (self.num_nodes,), "beta")
+        _dev(U, torch.float64, (self.num_nodes, 2), "U")
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_basal_friction(self._h, _ptr(basal_cells), int(basal_cells.numel()), _ptr(beta),
+                                              _ptr(U), _ptr(R), _ptr(J_face)), "basal_friction")
 
     def csr_pattern(self):
         import torch

@@ -310,3 +310,23 @@ def test_jvp_matrix_free_parity(torch, elem, drop, geometry):
     ctx.jvp(_t(torch, orc["U"]), _t(torch, 2 * X), Y2)
     ctx.sync()
     assert torch.allclose(Y2, 2 * Y, rtol=1e-14, atol=1e-14 * float(Y.abs().max()))
+
+
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_basal_friction_parity(torch, elem):
+    """NEXT-4 (reading Z18): GPU basal-friction side-set term vs the numpy oracle."""
+    from oracle import basal as B
+    L = 5
+    ctx, orc = _setup(torch, elem, n=8, L=L)
+    nb = 4 if elem == "hex8" else 3
+    cells = np.arange(0, ctx.num_cells, L, dtype=np.int32)    # k = 0: bed cells
+    beta = np.random.default_rng(8).uniform(0.1, 3.0, ctx.num_nodes)
+    R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+    Jf = torch.empty((cells.size, 2 * nb, 2 * nb), dtype=torch.float64, device="cuda")
+    ctx.basal_friction(_t(torch, cells), _t(torch, beta), _t(torch, orc["U"]), R, J_face=Jf)
+    ctx.sync()
+    Rr, Jr, _ = B.basal_friction(nb, orc["conn"], orc["coords"], cells, beta, orc["U"])
+    Jg = Jf.cpu().numpy()
+    sc = np.abs(Jr).reshape(cells.size, -1).max(1)
+    assert (np.abs(Jg - Jr).reshape(cells.size, -1).max(1) <= TOL * sc).all()
+    assert np.abs(R.cpu().numpy() - Rr).max() <= TOL * np.abs(Rr).max()
