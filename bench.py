@@ -203,6 +203,11 @@ def main():
     ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp"],
                     help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
                          "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
+    ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
+                    help="N>1 halo sum: p2p = fused into the evaluation kernel over NVLink-mapped peer memory "
+                         "(falls back to nccl if peer mapping fails); nccl = pack / grouped send-recv / unpack-add")
+    ap.add_argument("--check", action="store_true",
+                    help="N>1: compare every rank's halo-summed R with a one-GPU evaluation of the whole mesh")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
@@ -215,7 +220,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_sc_antepara0cw24_b200 import StokesFO
-    from paper_conf_sc_antepara0cw24_b200.halo import Halo, LocalPart
+    from paper_conf_sc_antepara0cw24_b200.halo import Halo, LocalPart, P2PHalo
 
     # STOKESFO_BENCH_BACKEND=gloo (debug only): ranks may share a GPU and the
     # halo buffers are staged through host memory; the timed product path is NCCL.
@@ -247,29 +252,48 @@ def main():
     Yd = torch.zeros((NN, 2), dtype=torch.float64, device=dev) if args.op == "jvp" else None
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     halo = None
+    p2p = None
+    halo_mode = "none"
     if world > 1:
-        halo = Halo(part.neighbors, dev, pack=ctx.halo_pack, unpack_add=ctx.halo_unpack_add,
-                    host_staging=(backend != "nccl"))
+        if args.halo == "p2p":
+            p2p = P2PHalo(ctx, part, dev, gloo_debug=(backend != "nccl"))
+            if not p2p.ok:
+                p2p.close()
+                p2p = None
+        if p2p is None:
+            halo = Halo(part.neighbors, dev, pack=ctx.halo_pack, unpack_add=ctx.halo_unpack_add,
+                        host_staging=(backend != "nccl"))
+            halo_mode = "nccl pack/send-recv/unpack"
+        else:
+            halo_mode = "fused: peer-memory atomics in the evaluation kernel + 1 barrier"
     ctx.sync()
     torch.cuda.synchronize(dev)
 
     k0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     k1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    R_last = [R]
 
     def step(i=None):
-        R.zero_()
+        if p2p is not None:
+            Rc = p2p.begin()
+        else:
+            Rc = R
+            Rc.zero_()
         if i is not None:
             k0[i].record(stream)
         if args.op == "jacobian":
-            ctx.jacobian(U, J, R=R)
+            ctx.jacobian(U, J, R=Rc)
         elif args.op == "jvp":
-            ctx.jvp(U, Xd, Yd, R=R)
+            ctx.jvp(U, Xd, Yd, R=Rc)
         else:
-            ctx.viscosity_resid(U, R=R)
+            ctx.viscosity_resid(U, R=Rc)
         if i is not None:
             k1[i].record(stream)
-        if halo is not None:
-            halo.exchange(R)
+        if p2p is not None:
+            p2p.end()
+        elif halo is not None:
+            halo.exchange(Rc)
+        R_last[0] = Rc
 
     for _ in range(args.warmup):
         step()
@@ -302,7 +326,7 @@ def main():
         for _ in range(2):
             U.copy_(U_host, non_blocking=True)
             step()
-            R_host.copy_(R, non_blocking=True)
+            R_host.copy_(R_last[0], non_blocking=True)
         torch.cuda.synchronize(dev)
         if world > 1:
             dist.barrier()
@@ -312,11 +336,30 @@ def main():
         for i in range(args.steps):
             U.copy_(U_host, non_blocking=True)
             step()
-            R_host.copy_(R, non_blocking=True)
+            R_host.copy_(R_last[0], non_blocking=True)
         e1.record(stream)
         torch.cuda.synchronize(dev)
         e2e_ms = e0.elapsed_time(e1) / args.steps
         e2e = [e2e_ms, U_host.numel() * 8, R_host.numel() * 8]
+
+    # ---- optional correctness check of the N>1 halo sum ----
+    check = None
+    if args.check and world > 1:
+        step()
+        torch.cuda.synchronize(dev)
+        Rmine = R_last[0].cpu().numpy()
+        full = StokesFO(elem, torch.from_numpy(conn_g).to(dev), torch.from_numpy(coords_g).to(dev),
+                        surface=torch.from_numpy(s_g).to(dev), flow_factor=torch.from_numpy(kc_g).to(dev),
+                        geometry=args.geometry)
+        Rf = torch.zeros((coords_g.shape[0], 2), dtype=torch.float64, device=dev)
+        Jf = torch.empty((conn_g.shape[0], 2 * N, 2 * N), dtype=torch.float64, device=dev)
+        full.jacobian(torch.from_numpy(U_g).to(dev), Jf, R=Rf)
+        full.sync()
+        Rref = Rf.cpu().numpy()[gids]
+        err = torch.tensor([float(np.abs(Rmine - Rref).max() / max(np.abs(Rref).max(), 1e-300))], dtype=torch.float64,
+                           device="cpu" if backend != "nccl" else dev)
+        dist.all_reduce(err, op=dist.ReduceOp.MAX)
+        check = float(err.item())
 
     # ---- reduce over ranks (max time) ----
     stats = torch.tensor([ms_total / args.steps, kern_ms, e2e[0] if e2e else 0.0], dtype=torch.float64, device=dev)
@@ -371,8 +414,11 @@ def main():
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src},
             "achieved_hbm_gbs": achieved,
             "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),
+            "halo": halo_mode,
             "clocks": clk,
         }
+        if check is not None:
+            line["halo_check_max_rel_err"] = check
         if e2e:
             line["e2e"] = {"value": total_cells / (e2e_ms * 1e-3), "unit": "cells/s",
                            "h2d_bytes_per_step": e2e[1], "d2h_bytes_per_step": e2e[2],
@@ -387,6 +433,10 @@ def main():
                                               f"geometry precomputed untimed), {dt:.1f} s"}
         print(json.dumps(line), flush=True)
     if world > 1:
+        if p2p is not None:
+            torch.cuda.synchronize(dev)
+            dist.barrier()
+            p2p.close()
         dist.barrier()
         dist.destroy_process_group()
     return 0

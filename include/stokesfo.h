@@ -170,6 +170,24 @@ int stokesfo_halo_pack(stokesfo_ctx *c, const double *R, const int32_t *send_nod
 int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *recv_nodes,
                              int64_t n, double *R);
 
+/* Fused halo sum over peer memory: after
+ * this call, the residual scatter of stokesfo_viscosity_resid / _jacobian /
+ * _jvp also adds every contribution to a partition-boundary node into the R
+ * of each other GPU holding that node, with atomics through NVLink-mapped
+ * peer pointers, so no pack / exchange / unpack is needed (one stream-ordered
+ * barrier per evaluation; R passed to the calls must be the buffer the peers
+ * mapped).  rem: dev int32 [num_nodes], row of remtab or -1; remtab: dev int32
+ * [rows][15] = {count <= 7, peer, remote_local_index, ...}; peers: dev array of
+ * device pointers (one per peer index; entries for this rank unused).  All
+ * stay owned by the caller and must outlive their use; rem = NULL detaches. */
+int stokesfo_set_remote(stokesfo_ctx *c, const int32_t *rem, const int32_t *remtab, double *const *peers);
+/* CUDA IPC plumbing for the above (handle = 64 opaque bytes).  A handle maps
+ * the whole allocation containing dev_ptr; *offset = dev_ptr - allocation
+ * base, to add to the pointer the peer obtains from stokesfo_ipc_open_handle. */
+int stokesfo_ipc_get_handle(const void *dev_ptr, void *handle, int64_t *offset);
+int stokesfo_ipc_open_handle(const void *handle, void **dev_ptr);
+int stokesfo_ipc_close(void *dev_ptr);
+
 /* Synchronise the ctx stream; returns ECUDA on a CUDA error, else EMESH if a
  * device-side error flag was raised since create, else OK. */
 int stokesfo_sync(stokesfo_ctx *c);

@@ -27,6 +27,9 @@ struct stokesfo_ctx {
     int grid_resid, grid_jac, grid_jvp;
     int rec_bytes;
     int nstage_resid, nstage_jac;  // TMA record ring depth of the eval kernels
+    const int32_t *rem = nullptr;     // fused halo over peer memory (stokesfo_set_remote)
+    const int32_t *remtab = nullptr;
+    double *const *peers = nullptr;
     const int64_t *rowptr = nullptr;  // CSR pattern (set by stokesfo_csr_pattern)
     const int32_t *colidx = nullptr;
     int64_t csr_rows = 0;
@@ -168,6 +171,9 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.J_cell = J_cell;
     a.X = X;
     a.Y = Y;
+    a.rem = c->rem;
+    a.remtab = c->remtab;
+    a.peers = c->peers;
     const int g = MODE == M_JAC ? c->grid_jac : (MODE == M_JVP ? c->grid_jvp : c->grid_resid);
     const int grid = (int)std::min<int64_t>(g, c->ntiles);
     const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_JVP ? 2 : c->nstage_resid);
@@ -385,6 +391,55 @@ int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *
     halo_unpack_add_kernel<<<(unsigned)((n + bs - 1) / bs), bs, 0, c->stream>>>(
         n, recv_nodes, reinterpret_cast<const double2 *>(buf), reinterpret_cast<double2 *>(R));
     return cuda_status();
+}
+
+int stokesfo_set_remote(stokesfo_ctx *c, const int32_t *rem, const int32_t *remtab, double *const *peers) {
+    if (!c) return STOKESFO_EINVAL;
+    if (!rem) {  // detach
+        c->rem = nullptr;
+        c->remtab = nullptr;
+        c->peers = nullptr;
+        return STOKESFO_OK;
+    }
+    if (!remtab || !peers) return STOKESFO_EINVAL;
+    c->rem = rem;
+    c->remtab = remtab;
+    c->peers = peers;
+    return STOKESFO_OK;
+}
+
+int stokesfo_ipc_get_handle(const void *dev_ptr, void *handle, int64_t *offset) {
+    if (!dev_ptr || !handle || !offset) return STOKESFO_EINVAL;
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, const_cast<void *>(dev_ptr)) != cudaSuccess) return cuda_status();
+    memcpy(handle, &h, sizeof(h));
+    // the handle maps the whole allocation: report dev_ptr's offset from its base
+    // (cuMemGetAddressRange through the runtime's driver entry point)
+    typedef int (*GetRange)(unsigned long long *, size_t *, unsigned long long);
+    void *fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn)
+        return cuda_status() ? STOKESFO_ECUDA : STOKESFO_ECUDA;
+    unsigned long long base = 0;
+    size_t size = 0;
+    if (reinterpret_cast<GetRange>(fn)(&base, &size, reinterpret_cast<unsigned long long>(dev_ptr)) != 0)
+        return STOKESFO_ECUDA;
+    *offset = (int64_t)(reinterpret_cast<unsigned long long>(dev_ptr) - base);
+    return STOKESFO_OK;
+}
+
+int stokesfo_ipc_open_handle(const void *handle, void **dev_ptr) {
+    if (!dev_ptr || !handle) return STOKESFO_EINVAL;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof(h));
+    if (cudaIpcOpenMemHandle(dev_ptr, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) return cuda_status();
+    return STOKESFO_OK;
+}
+
+int stokesfo_ipc_close(void *dev_ptr) {
+    if (!dev_ptr) return STOKESFO_EINVAL;
+    if (cudaIpcCloseMemHandle(dev_ptr) != cudaSuccess) return cuda_status();
+    return STOKESFO_OK;
 }
 
 int stokesfo_sync(stokesfo_ctx *c) {

@@ -257,7 +257,37 @@ struct EvalArgs {
     double *J_cell;           // [C][2N][2N] (M_JAC)
     const double *X;          // [nodes][2] direction (M_JVP)
     double *Y;                // [nodes][2] += J(U) X (M_JVP)
+    // fused halo over peer memory (null = none): rem[node] = row of remtab or -1;
+    // remtab[row] = {count, peer_0, idx_0, peer_1, idx_1, ...} (REM_ROW ints);
+    // peers[p] = device pointer of peer p's R, mapped into this process
+    const int32_t *rem;
+    const int32_t *remtab;
+    double *const *peers;
 };
+
+constexpr int REM_MAX = 7;                 // remote copies of one node (<= 8 parts meet at a vertex)
+constexpr int REM_ROW = 1 + 2 * REM_MAX;
+
+// R[node] += (r0, r1) locally and, for nodes on a partition boundary, into the
+// R of every other GPU that holds the node (red.global.add.f64 through the
+// NVLink-mapped peer pointer): the halo sum happens inside the evaluation
+// kernel, no pack / exchange / unpack.
+__device__ __forceinline__ void scatter_node(const EvalArgs &a, int32_t node, double r0, double r1) {
+    atomicAdd(a.R + 2 * (int64_t)node + 0, r0);
+    atomicAdd(a.R + 2 * (int64_t)node + 1, r1);
+    if (a.rem) {
+        const int32_t row = __ldg(a.rem + node);
+        if (row >= 0) {
+            const int32_t *t = a.remtab + (int64_t)row * REM_ROW;
+            const int cnt = t[0];
+            for (int k = 0; k < cnt; ++k) {
+                double *pr = a.peers[t[1 + 2 * k]] + 2 * (int64_t)t[2 + 2 * k];
+                atomicAdd(pr + 0, r0);
+                atomicAdd(pr + 1, r1);
+            }
+        }
+    }
+}
 
 // Evaluation modes of the fused kernels
 enum { M_RESID = 0, M_JAC = 1, M_JVP = 2 };
@@ -644,10 +674,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
             }
         }
         if (act && c < nvalid) {
-            if (a.R) {
-                atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
-                atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
-            }
+            if (a.R) scatter_node(a, gnode, R0, R1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
             if (JVP) {
                 atomicAdd(a.Y + 2 * (int64_t)gnode + 0, dR0);
@@ -844,10 +871,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_otf_kernel
             if (l == 0) store_J<E>(a.J_cell, cell0, nvalid, reinterpret_cast<const char *>(rg), pol_stream);
         }
         if (act && c < nvalid) {
-            if (a.R) {
-                atomicAdd(a.R + 2 * (int64_t)gnode + 0, R0);
-                atomicAdd(a.R + 2 * (int64_t)gnode + 1, R1);
-            }
+            if (a.R) scatter_node(a, gnode, R0, R1);
             if (JVP) {
                 atomicAdd(a.Y + 2 * (int64_t)gnode + 0, dR0);
                 atomicAdd(a.Y + 2 * (int64_t)gnode + 1, dR1);

@@ -30,6 +30,7 @@ class LocalPart:
         self.conn, self.gids = S.mesh_localize(conn_global[self.cell_lo:self.cell_hi])
         # every rank derives every part's node set (deterministic) -> halo lists
         self.neighbors = {}
+        self.remote_index = {}   # r -> local ids ON RANK r of the nodes in neighbors[r] (same gid order)
         for r in range(world):
             if r == rank:
                 continue
@@ -40,6 +41,99 @@ class LocalPart:
             idx = S.mesh_halo_list(self.gids, g_other)
             if idx.size:
                 self.neighbors[r] = idx
+                self.remote_index[r] = S.mesh_halo_list(g_other, self.gids)
+
+    def remote_table(self, rem_max: int = 7):
+        """(rem [num_local_nodes] int32, remtab [rows][1+2*rem_max] int32) for
+        stokesfo_set_remote: row of a boundary node = {count, peer, index on peer, ...}."""
+        per_node = {}
+        for r in sorted(self.neighbors):
+            for m, t in zip(self.neighbors[r].tolist(), self.remote_index[r].tolist()):
+                per_node.setdefault(m, []).append((r, t))
+        rem = np.full(self.gids.size, -1, dtype=np.int32)
+        remtab = np.zeros((max(len(per_node), 1), 1 + 2 * rem_max), dtype=np.int32)
+        for row, m in enumerate(sorted(per_node)):
+            lst = per_node[m]
+            if len(lst) > rem_max:
+                raise ValueError(f"node shared by {len(lst) + 1} parts > {rem_max + 1}")
+            rem[m] = row
+            remtab[row, 0] = len(lst)
+            for k, (r, t) in enumerate(lst):
+                remtab[row, 1 + 2 * k] = r
+                remtab[row, 2 + 2 * k] = t
+        return rem, remtab
+
+
+class P2PHalo:
+    """Fused halo sum over peer memory: the evaluation kernels add boundary-node
+    contributions straight into the peers' R (CUDA IPC-mapped, NVLink), so a
+    step is  zero(R_next) -> evaluate(R_cur) -> one stream-ordered barrier.
+    R is double-buffered (step t writes R[t % 2]; R[(t+1) % 2] is zeroed before
+    the barrier of step t, so no peer can write it before it is clear).
+
+    Use: h = P2PHalo(ctx, part, nodes, device); for each step: R = h.begin();
+    ctx.jacobian(U, J, R=R); h.end()  (R now holds the full sum)."""
+
+    def __init__(self, ctx, part: LocalPart, device, gloo_debug: bool = False):
+        import torch
+        import torch.distributed as dist
+        self.ctx, self.device, self.gloo = ctx, device, gloo_debug
+        self.rank, self.world = part.rank, part.world
+        nn = part.gids.size
+        self.R = [torch.zeros((nn, 2), dtype=torch.float64, device=device) for _ in range(2)]
+        rem, remtab = part.remote_table()
+        self.rem = torch.from_numpy(rem).to(device)
+        self.remtab = torch.from_numpy(remtab).to(device)
+        handles = [S.ipc_get_handle(R) for R in self.R]
+        allh = [None] * self.world
+        dist.all_gather_object(allh, handles)
+        self.opened = []
+        ok = 1
+        ptrs = [[0] * self.world for _ in range(2)]
+        bases = {}   # one mapping per distinct peer allocation (handles may repeat)
+        try:
+            for b in range(2):
+                ptrs[b][self.rank] = self.R[b].data_ptr()
+                for r in part.neighbors:
+                    raw, off = allh[r][b]
+                    if raw not in bases:
+                        bases[raw] = S.ipc_open_handle((raw, 0))
+                        self.opened.append(bases[raw])
+                    ptrs[b][r] = bases[raw] + off
+        except Exception:
+            ok = 0
+        flag = torch.tensor([ok], dtype=torch.int32, device="cpu" if gloo_debug else device)
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        self.ok = bool(flag.item())
+        self.peers = [torch.tensor(ptrs[b], dtype=torch.int64, device=device) for b in range(2)]
+        self.token = torch.zeros(1, dtype=torch.float32, device=device)
+        self.t = 0
+        self.launches_per_step = 0  # no pack/unpack kernels: the halo rides the evaluation kernel
+
+    def begin(self):
+        """Returns this step's R (already zero); zeroes the next step's buffer."""
+        cur = self.R[self.t % 2]
+        self.R[(self.t + 1) % 2].zero_()
+        self.ctx.set_remote(self.rem, self.remtab, self.peers[self.t % 2])
+        return cur
+
+    def end(self):
+        """Stream-ordered barrier: after it, every rank's kernel of this step is complete."""
+        import torch
+        import torch.distributed as dist
+        if self.gloo:
+            torch.cuda.synchronize(self.device)
+            dist.barrier()
+        else:
+            dist.all_reduce(self.token)
+        self.t += 1
+        return self.R[(self.t - 1) % 2]
+
+    def close(self):
+        self.ctx.set_remote(None, None, None)
+        for p in self.opened:
+            S.ipc_close(p)
+        self.opened = []
 
 
 class Halo:

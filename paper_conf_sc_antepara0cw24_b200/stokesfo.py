@@ -54,6 +54,7 @@ EXPORTS = [
     "stokesfo_mesh_partition_columns", "stokesfo_mesh_localize", "stokesfo_mesh_halo_list",
     "stokesfo_albany_scratch_size", "stokesfo_albany_setup", "stokesfo_albany_evaluators",
     "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp", "stokesfo_basal_friction",
+    "stokesfo_set_remote", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
 ]
 FIG2 = {"baseline": 0, "optimized": 1}
 
@@ -81,6 +82,11 @@ def _lib():
             L.stokesfo_jvp.argtypes = [P, P, P, P, P]
         if hasattr(L, "stokesfo_basal_friction"):
             L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
+        if hasattr(L, "stokesfo_set_remote"):
+            L.stokesfo_set_remote.argtypes = [P, P, P, P]
+            L.stokesfo_ipc_get_handle.argtypes = [P, P, ctypes.POINTER(I64)]
+            L.stokesfo_ipc_open_handle.argtypes = [P, ctypes.POINTER(ctypes.c_void_p)]
+            L.stokesfo_ipc_close.argtypes = [P]
         L.stokesfo_scatter_assemble.argtypes = [P, P, P, P, P]
         L.stokesfo_csr_pattern.argtypes = [P, ctypes.POINTER(I64), P, P]
         L.stokesfo_geometry.argtypes = [P, P, P]
@@ -231,6 +237,11 @@ class StokesFO:
         _check(_lib().stokesfo_basal_friction(self._h, _ptr(basal_cells), int(basal_cells.numel()), _ptr(beta),
                                               _ptr(U), _ptr(R), _ptr(J_face)), "basal_friction")
 
+    def set_remote(self, rem, remtab, peers):
+        """Fused halo over peer memory (stokesfo_set_remote); rem=None detaches."""
+        self._remote_keep = (rem, remtab, peers)
+        _check(_lib().stokesfo_set_remote(self._h, _ptr(rem), _ptr(remtab), _ptr(peers)), "set_remote")
+
     def csr_pattern(self):
         import torch
         nnz = ctypes.c_int64(0)
@@ -292,6 +303,26 @@ class StokesFO:
                                            ctypes.byref(rb)), "launch_info")
         return {"cells_per_tile": tc.value, "grid_resid": gr.value, "grid_jac": gj.value,
                 "record_bytes_per_tile": rb.value}
+
+
+def ipc_get_handle(t):
+    """(64-byte CUDA IPC handle of the tensor's allocation, offset of the tensor in it)."""
+    buf = ctypes.create_string_buffer(64)
+    off = ctypes.c_int64(0)
+    _check(_lib().stokesfo_ipc_get_handle(ctypes.c_void_p(t.data_ptr()), buf, ctypes.byref(off)), "ipc_get_handle")
+    return buf.raw, int(off.value)
+
+
+def ipc_open_handle(h) -> int:
+    """Map a peer's (handle, offset); returns the device pointer of the peer tensor."""
+    raw, off = h
+    p = ctypes.c_void_p()
+    _check(_lib().stokesfo_ipc_open_handle(ctypes.create_string_buffer(raw, 64), ctypes.byref(p)), "ipc_open_handle")
+    return int(p.value) + off
+
+
+def ipc_close(p: int):
+    _check(_lib().stokesfo_ipc_close(ctypes.c_void_p(p)), "ipc_close")
 
 
 # ---------------------------------------------------------------------------
