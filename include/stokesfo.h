@@ -202,6 +202,33 @@ void stokesfo_destroy(stokesfo_ctx *c);
 int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid_resid,
                          int32_t *grid_jac, int64_t *record_bytes_per_tile);
 
+/* ---------------- NEXT-3: damped Newton-Krylov driver ---------------------- */
+
+/* Solves F(U) = R_visc(U) + R_basal(U) = 0 (damped Newton, Jacobian at
+ * every nonlinear step): per step, J dU = -F by Jacobi-preconditioned CG on the
+ * matrix-free operator stokesfo_jvp + basal face term (J is SPD once basal
+ * friction removes the rigid null space; Jacobi diagonal from stokesfo_jacobian
+ * and the basal face matrices), then Armijo backtracking on ||F||.  Stops when
+ * ||F|| <= max(atol, rtol ||F_0||) or after max_newton steps.  Single-GPU ctx
+ * (no stokesfo_set_remote).  U: dev [num_nodes][2], initial guess in, solution
+ * out.  work: dev, stokesfo_newton_work_size bytes, 256-B aligned.  hist_F:
+ * host [max_newton + 1] ||F|| per step; hist_cg: host [max_newton] CG
+ * iterations (may be NULL); *iters = Newton steps taken. */
+typedef struct {
+    int32_t max_newton;   /* e.g. 8 */
+    int32_t max_cg;       /* CG iterations per Newton step */
+    int32_t max_ls;       /* backtracking halvings */
+    int32_t reserved;
+    double rtol_newton;   /* on ||F|| / ||F_0|| */
+    double atol_newton;
+    double rtol_cg;       /* linear solve ||r|| <= rtol_cg ||F|| (1e-6) */
+    double ls_c;          /* Armijo constant, e.g. 1e-4 */
+} stokesfo_newton_opts_t;
+int stokesfo_newton_work_size(stokesfo_ctx *c, int64_t nbasal, size_t *bytes);
+int stokesfo_newton_solve(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nbasal, const double *beta,
+                          double *U, void *work, const stokesfo_newton_opts_t *opts, double *hist_F,
+                          int32_t *hist_cg, int32_t *iters);
+
 /* ---------------- NEXT-1: the paper's evaluator chain on B200 -------------- */
 
 /* Albany's unfused chain (SURVEY CS-1) with HBM intermediates, to reproduce

@@ -12,6 +12,7 @@
 #include "../../include/stokesfo.h"
 #include "sfo_kernels.cuh"
 #include "sfo_albany.cuh"
+#include "sfo_newton.cuh"
 
 using namespace sfo;
 
@@ -536,6 +537,151 @@ int stokesfo_albany_resid(stokesfo_ctx *c, int derivs, int variant, double *scra
 }
 int stokesfo_albany_extract(stokesfo_ctx *c, int derivs, const double *scratch, double *R_cell, double *J_cell) {
     return albany_dispatch(c, derivs, 3, 0, nullptr, const_cast<double *>(scratch), R_cell, J_cell);
+}
+
+// ---------------------------------------------------------------------------
+// NEXT-3: damped Newton-Krylov driver (sfo_newton.cuh)
+// ---------------------------------------------------------------------------
+}  // extern "C"
+
+namespace {
+struct NewtonWork {
+    double *F, *D, *Rr, *P, *AP, *Z, *Ut, *diag, *Jc, *Jf, *scal;
+    int64_t bytes;
+};
+NewtonWork newton_layout(const stokesfo_ctx *c, int64_t nbasal, char *base) {
+    NewtonWork w{};
+    const int64_t n = 2 * c->d.num_nodes, C = c->d.num_cells, ND = 2 * c->N, NFD = c->N;  // face: 2*NB = N
+    int64_t off = 0;
+    auto take = [&](int64_t count) {
+        double *p = reinterpret_cast<double *>(base + off);
+        off += round_up(std::max<int64_t>(count, 1) * 8, 256);
+        return p;
+    };
+    w.F = take(n); w.D = take(n); w.Rr = take(n); w.P = take(n); w.AP = take(n); w.Z = take(n); w.Ut = take(n);
+    w.diag = take(n); w.Jc = take(C * ND * ND); w.Jf = take(nbasal * NFD * NFD); w.scal = take(32);
+    w.bytes = off;
+    return w;
+}
+}  // namespace
+
+extern "C" {
+
+int stokesfo_newton_work_size(stokesfo_ctx *c, int64_t nbasal, size_t *bytes) {
+    if (!c || !bytes || nbasal < 0) return STOKESFO_EINVAL;
+    *bytes = (size_t)newton_layout(c, nbasal, nullptr).bytes;
+    return STOKESFO_OK;
+}
+
+int stokesfo_newton_solve(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nbasal, const double *beta,
+                          double *U, void *work, const stokesfo_newton_opts_t *o, double *hist_F, int32_t *hist_cg,
+                          int32_t *iters) {
+    using namespace sfo::newton;
+    if (!c || !U || !work || !o || !hist_F || !iters || nbasal < 0 || (nbasal > 0 && (!basal_cells || !beta)))
+        return STOKESFO_EINVAL;
+    if (!aligned(U, 16) || !aligned(work, 256)) return STOKESFO_EINVAL;
+    NewtonWork w = newton_layout(c, nbasal, reinterpret_cast<char *>(work));
+    const int64_t n = 2 * c->d.num_nodes;
+    const size_t vb = (size_t)n * 8;
+    cudaStream_t st = c->stream;
+    const int bs = 256;
+    const unsigned gv = (unsigned)std::min<int64_t>((n + bs - 1) / bs, 148 * 8);
+    int rc = STOKESFO_OK;
+#define CK(x)                     \
+    do {                          \
+        rc = (x);                 \
+        if (rc != STOKESFO_OK) return rc; \
+    } while (0)
+    auto dot = [&](const double *x, const double *y, double &out) -> int {
+        if (cudaMemsetAsync(w.scal, 0, 8, st) != cudaSuccess) return cuda_status();
+        dot_kernel<<<gv, bs, 0, st>>>(n, x, y, w.scal);
+        if (cudaMemcpyAsync(&out, w.scal, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess) return cuda_status();
+        if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_status();
+        return STOKESFO_OK;
+    };
+    auto eval_F = [&](const double *u, double *F) -> int {  // F = R_visc(u) + R_basal(u)
+        if (cudaMemsetAsync(F, 0, vb, st) != cudaSuccess) return cuda_status();
+        int r = stokesfo_viscosity_resid(c, u, nullptr, nullptr, F);
+        if (r == STOKESFO_OK && nbasal > 0) r = stokesfo_basal_friction(c, basal_cells, nbasal, beta, u, F, nullptr);
+        return r;
+    };
+    auto apply_A = [&](const double *v, double *Av) -> int {  // Av = J(U) v + J_basal v
+        if (cudaMemsetAsync(Av, 0, vb, st) != cudaSuccess) return cuda_status();
+        int r = stokesfo_jvp(c, U, v, Av, nullptr);
+        if (r == STOKESFO_OK && nbasal > 0) r = stokesfo_basal_friction(c, basal_cells, nbasal, beta, v, Av, nullptr);
+        return r;
+    };
+    double nF0 = 0.0;
+    int k = 0;
+    for (;; ++k) {
+        CK(eval_F(U, w.F));
+        double ff;
+        CK(dot(w.F, w.F, ff));
+        const double nF = sqrt(ff);
+        hist_F[k] = nF;
+        if (k == 0) nF0 = nF;
+        if (nF <= std::max(o->atol_newton, o->rtol_newton * nF0) || k >= o->max_newton) break;
+        // Jacobi diagonal of J(U) + J_basal
+        CK(stokesfo_jacobian(c, U, w.Jc, nullptr, nullptr));
+        if (cudaMemsetAsync(w.diag, 0, vb, st) != cudaSuccess) return cuda_status();
+        {
+            const int64_t work_c = c->d.num_cells * 2 * c->N;
+            const unsigned g = (unsigned)((work_c + bs - 1) / bs);
+            if (c->N == 8) diag_cells_kernel<8><<<g, bs, 0, st>>>(c->d.num_cells, c->d.conn, w.Jc, w.diag);
+            else diag_cells_kernel<6><<<g, bs, 0, st>>>(c->d.num_cells, c->d.conn, w.Jc, w.diag);
+        }
+        if (nbasal > 0) {
+            if (cudaMemsetAsync(w.Z, 0, vb, st) != cudaSuccess) return cuda_status();
+            CK(stokesfo_basal_friction(c, basal_cells, nbasal, beta, U, w.Z, w.Jf));
+            const unsigned g = (unsigned)((nbasal * c->N + bs - 1) / bs);
+            if (c->N == 8) diag_faces_kernel<8><<<g, bs, 0, st>>>(nbasal, basal_cells, c->d.conn, w.Jf, w.diag);
+            else diag_faces_kernel<6><<<g, bs, 0, st>>>(nbasal, basal_cells, c->d.conn, w.Jf, w.diag);
+        }
+        // CG on J D = -F
+        if (cudaMemsetAsync(w.D, 0, vb, st) != cudaSuccess) return cuda_status();
+        if (cudaMemsetAsync(w.Rr, 0, vb, st) != cudaSuccess) return cuda_status();
+        axpby_kernel<<<gv, bs, 0, st>>>(n, -1.0, w.F, 0.0, w.Rr);            // r = -F
+        jacobi_kernel<<<gv, bs, 0, st>>>(n, w.Rr, w.diag, w.Z);             // z = r / diag
+        if (cudaMemcpyAsync(w.P, w.Z, vb, cudaMemcpyDeviceToDevice, st) != cudaSuccess) return cuda_status();
+        double rz;
+        CK(dot(w.Rr, w.Z, rz));
+        int j = 0;
+        for (; j < o->max_cg; ++j) {
+            CK(apply_A(w.P, w.AP));
+            double pAp;
+            CK(dot(w.P, w.AP, pAp));
+            const double alpha = rz / pAp;
+            axpby_kernel<<<gv, bs, 0, st>>>(n, alpha, w.P, 1.0, w.D);       // D += alpha p
+            axpby_kernel<<<gv, bs, 0, st>>>(n, -alpha, w.AP, 1.0, w.Rr);    // r -= alpha A p
+            double rr;
+            CK(dot(w.Rr, w.Rr, rr));
+            if (sqrt(rr) <= o->rtol_cg * nF) {
+                ++j;
+                break;
+            }
+            jacobi_kernel<<<gv, bs, 0, st>>>(n, w.Rr, w.diag, w.Z);
+            double rz_new;
+            CK(dot(w.Rr, w.Z, rz_new));
+            axpby_kernel<<<gv, bs, 0, st>>>(n, 1.0, w.Z, rz_new / rz, w.P);  // p = z + (rz_new / rz) p
+            rz = rz_new;
+        }
+        if (hist_cg) hist_cg[k] = j;
+        // Armijo backtracking on ||F||
+        double a = 1.0;
+        for (int ls = 0;; ++ls) {
+            if (cudaMemcpyAsync(w.Ut, U, vb, cudaMemcpyDeviceToDevice, st) != cudaSuccess) return cuda_status();
+            axpby_kernel<<<gv, bs, 0, st>>>(n, a, w.D, 1.0, w.Ut);
+            CK(eval_F(w.Ut, w.Rr));
+            double ft;
+            CK(dot(w.Rr, w.Rr, ft));
+            if (sqrt(ft) <= (1.0 - o->ls_c * a) * nF || ls >= o->max_ls) break;
+            a *= 0.5;
+        }
+        if (cudaMemcpyAsync(U, w.Ut, vb, cudaMemcpyDeviceToDevice, st) != cudaSuccess) return cuda_status();
+    }
+#undef CK
+    *iters = k;
+    return cuda_status();
 }
 
 // CSR pattern: host-side construction from a device->host copy of conn.

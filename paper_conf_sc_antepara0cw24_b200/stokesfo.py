@@ -55,7 +55,14 @@ EXPORTS = [
     "stokesfo_albany_scratch_size", "stokesfo_albany_setup", "stokesfo_albany_evaluators",
     "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp", "stokesfo_basal_friction",
     "stokesfo_set_remote", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
+    "stokesfo_newton_work_size", "stokesfo_newton_solve",
 ]
+
+
+class NewtonOpts(ctypes.Structure):
+    _fields_ = [("max_newton", ctypes.c_int32), ("max_cg", ctypes.c_int32), ("max_ls", ctypes.c_int32),
+                ("reserved", ctypes.c_int32), ("rtol_newton", ctypes.c_double), ("atol_newton", ctypes.c_double),
+                ("rtol_cg", ctypes.c_double), ("ls_c", ctypes.c_double)]
 FIG2 = {"baseline": 0, "optimized": 1}
 
 
@@ -82,6 +89,10 @@ def _lib():
             L.stokesfo_jvp.argtypes = [P, P, P, P, P]
         if hasattr(L, "stokesfo_basal_friction"):
             L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
+        if hasattr(L, "stokesfo_newton_solve"):
+            L.stokesfo_newton_work_size.argtypes = [P, I64, ctypes.POINTER(ctypes.c_size_t)]
+            L.stokesfo_newton_solve.argtypes = [P, P, I64, P, P, P, ctypes.POINTER(NewtonOpts), P, P,
+                                                ctypes.POINTER(I32)]
         if hasattr(L, "stokesfo_set_remote"):
             L.stokesfo_set_remote.argtypes = [P, P, P, P]
             L.stokesfo_ipc_get_handle.argtypes = [P, P, ctypes.POINTER(I64)]
@@ -236,6 +247,25 @@ class StokesFO:
         _dev(R, torch.float64, (self.num_nodes, 2), "R")
         _check(_lib().stokesfo_basal_friction(self._h, _ptr(basal_cells), int(basal_cells.numel()), _ptr(beta),
                                               _ptr(U), _ptr(R), _ptr(J_face)), "basal_friction")
+
+    def newton_solve(self, basal_cells, beta, U, max_newton=8, max_cg=500, max_ls=20, rtol_newton=1e-10,
+                     atol_newton=0.0, rtol_cg=1e-6, ls_c=1e-4):
+        """Damped Newton-Krylov solve of R_visc(U) + R_basal(U) = 0 in place on U
+        (stokesfo_newton_solve).  Returns {"F": [||F_k||], "cg": [iters], "iters": k}."""
+        import torch
+        _dev(U, torch.float64, (self.num_nodes, 2), "U")
+        nb = 0 if basal_cells is None else int(basal_cells.numel())
+        n = ctypes.c_size_t(0)
+        _check(_lib().stokesfo_newton_work_size(self._h, nb, ctypes.byref(n)), "newton_work_size")
+        work = torch.empty(int(n.value), dtype=torch.uint8, device=self.device)
+        o = NewtonOpts(max_newton, max_cg, max_ls, 0, rtol_newton, atol_newton, rtol_cg, ls_c)
+        hF = (ctypes.c_double * (max_newton + 1))()
+        hc = (ctypes.c_int32 * max(max_newton, 1))()
+        it = ctypes.c_int32(0)
+        _check(_lib().stokesfo_newton_solve(self._h, _ptr(basal_cells), nb, _ptr(beta), _ptr(U), _ptr(work),
+                                            ctypes.byref(o), hF, hc, ctypes.byref(it)), "newton_solve")
+        k = it.value
+        return {"F": [hF[i] for i in range(k + 1)], "cg": [hc[i] for i in range(k)], "iters": k}
 
     def set_remote(self, rem, remtab, peers):
         """Fused halo over peer memory (stokesfo_set_remote); rem=None detaches."""
