@@ -95,3 +95,29 @@ def test_partition_localize_halo_bit_exact(P):
                 assert np.array_equal(idx, halo[(r, s)])
             else:
                 assert idx.size == 0
+
+
+def test_create_rejects_bad_descriptors_without_gpu():
+    """Validation happens before any CUDA call: sizes beyond int32 node ids, negative
+    counts, bad element/geometry modes, wrong ABI version, non-positive delta."""
+    lib = S._lib()
+
+    def desc(**kw):
+        d = S.Desc()
+        d.abi_version, d.elem, d.num_cells, d.num_nodes = 1, 0, 4, 10
+        d.conn, d.coords = ctypes.c_void_p(256), ctypes.c_void_p(512)
+        d.glen_n, d.delta, d.k = 3.0, 1e-10, 1.0
+        d.workspace, d.workspace_bytes = ctypes.c_void_p(1024), 1 << 20
+        for k, v in kw.items():
+            setattr(d, k, v)
+        return d
+
+    h = ctypes.c_void_p()
+    for bad, code in ((dict(num_nodes=2 ** 31), 1), (dict(num_cells=-1), 1), (dict(elem=7), 1),
+                      (dict(abi_version=2), 1), (dict(delta=0.0), 1), (dict(glen_n=4.0), 5),
+                      (dict(geometry_mode=3), 1), (dict(workspace=ctypes.c_void_p(1032)), 1),
+                      (dict(coords=ctypes.c_void_p(520)), 1), (dict(workspace_bytes=100), 4)):
+        assert lib.stokesfo_create(ctypes.byref(desc(**bad)), ctypes.byref(h)) == code, bad
+    n = ctypes.c_size_t()
+    assert lib.stokesfo_workspace_size(ctypes.byref(desc(geometry_mode=1)), ctypes.byref(n)) == 0
+    assert n.value == 256 + ((10 * 32 + 255) // 256) * 256      # header + double4 coordinates
