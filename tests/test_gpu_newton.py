@@ -70,9 +70,10 @@ def test_newton_krylov_matches_oracle_newton(elem):
                          max_cg=2000, rtol_newton=1e-11, rtol_cg=1e-10)
     F = h["F"]
     assert F[-1] <= 1e-9 * F[0], F
-    # quadratic tail: once below 1e-3 of the start, each step at least squares the relative residual (x10 slack)
+    # quadratic tail of an inexact Newton: once below 1e-3 of the start, each step
+    # squares the relative residual up to the linear-solve tolerance (rtol_cg 1e-10)
     rel = [f / F[0] for f in F]
     tail = [(a, b) for a, b in zip(rel, rel[1:]) if a < 1e-3 and b > 1e-13]
-    assert all(b <= 10 * a * a + 1e-14 for a, b in tail), rel
+    assert all(b <= 10 * a * a + 1e-8 * a + 1e-14 for a, b in tail), rel
     Ug = Ud.cpu().numpy()
     assert np.abs(Ug - Uo).max() <= 1e-8 * np.abs(Uo).max()
