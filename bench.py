@@ -31,6 +31,7 @@ WORKLOADS = {
     "C5": "C5 Antarctica-like wedge6 (quads split), 10 layers, 6 QPs, residual+Jacobian (BASELINE.json configs[4])",
     "C1": "C1/C2 tiny 16x16 footprint x 5 layers, hex8, residual+Jacobian (BASELINE.json configs[1])",
     "C3": "C3 Greenland-like 1-10 km NVB footprint x 10 layers, hex8, residual+Jacobian (BASELINE.json configs[2])",
+    "C4p": "C4p paper-shaped Antarctica-like 16 km x 20 layers, hex8 (~1.05M cells; the paper's ~256K/GPU at 4 GPUs)",
 }
 
 
