@@ -11,6 +11,8 @@ Contents:
                 Fig. 2 loop orders), forward-AD Jacobian, closed-form tangent,
                 gather, scatter, CSR scatter.
   basal.py      numpy basal-friction side-set term (NEXT-4, reading Z18)
+  lateral.py    numpy lateral (calving-front) pressure side-set term and the
+                footprint boundary-side set (NEXT-4, reading Z19)
   ref.py        ctypes wrapper of oracle.c + numpy O1 extrusion, O9 CSR
                 pattern / partition / halo lists, and a numpy complex-step
                 residual used as an independent derivative pin.
