@@ -145,6 +145,22 @@ int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, d
 int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nfaces, const double *beta,
                             const double *U, double *R, double *J_face);
 
+/* Lateral (calving-front / ocean) pressure side-set term (NEXT-4; P:L59 ->
+ * [24]; reading Z19).  On each listed lateral face -- the quad of
+ * cell `cell` over its footprint polygon side k (local nodes k, k+1, k+1+P,
+ * k+P; P = 4 hex8 / 3 wedge6, indices mod P; xi along the side, eta upward) --
+ *     R[2 node_i + a] -= int psi(z) n_a phi_i dGamma,  a = 0, 1,
+ *     psi(z) = rho_i_g (s_h - z) - rho_w_g max(sea_level - z, 0),
+ * with 2x2 Gauss, n dGamma = dx/dxi x dx/deta (outward for counter-clockwise
+ * footprint polygons) and s_h, z interpolated with the bilinear face basis.
+ * The term does not depend on U (no Jacobian contribution).  faces: dev int32
+ * [nfaces][2] = (cell, side), 8-B aligned (stokesfo_mesh_lateral_faces builds
+ * the footprint boundary's list); surface: dev [num_nodes] s; R: dev
+ * [num_nodes][2] (+=).  A side outside [0, P) or a cell outside [0, C) raises
+ * the sticky EMESH flag. */
+int stokesfo_lateral_pressure(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
+                              double rho_i_g, double rho_w_g, double sea_level, double *R);
+
 /* Assembly: R[2 conn[c][n] + a] += R_cell[c][n][a] (if R_cell and R are non-NULL)
  * and csr_vals[pos(row, col)] += J_cell[c][k][l] (if J_cell and csr_vals are
  * non-NULL; requires an earlier stokesfo_csr_pattern call with non-NULL rowptr
@@ -281,6 +297,14 @@ int stokesfo_mesh_localize(int32_t npc, int64_t ncells, const int32_t *conn_glob
  * two sorted lists share, ordered by global id.  Size query with idx == NULL. */
 int stokesfo_mesh_halo_list(int64_t n_mine, const int64_t *gids_mine, int64_t n_other,
                             const int64_t *gids_other, int64_t *n_shared, int32_t *idx);
+
+/* Lateral faces of the extruded mesh: every footprint polygon side whose edge
+ * belongs to exactly one polygon (the footprint boundary), times the L layers:
+ * faces[m] = (cell f L + l, side k), ordered by (f, k, l).  polys: host
+ * [nf][npoly].  Size query with faces == NULL (sets *nfaces); fill faces host
+ * int32 [nfaces][2]. */
+int stokesfo_mesh_lateral_faces(int32_t npoly, int64_t nf, const int32_t *polys, int32_t L, int64_t *nfaces,
+                                int32_t *faces);
 
 #ifdef __cplusplus
 }

@@ -8,4 +8,4 @@ rebuilt as hand-written sm_100a CUDA behind a C ABI (include/stokesfo.h).
     build     -- in-tree nvcc build for sm_100a
 """
 from .stokesfo import (StokesFO, StokesFOError, mesh_extrude, mesh_halo_list, mesh_localize,  # noqa: F401
-                       mesh_partition_columns)
+                       mesh_lateral_faces, mesh_partition_columns)

@@ -13,7 +13,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libstokesfo.so")
 SOURCES = ["sfo_capi.cu", "sfo_mesh.cpp"]
-HEADERS = ["sfo_common.cuh", "sfo_kernels.cuh"]
+HEADERS = ["sfo_common.cuh", "sfo_kernels.cuh", "sfo_albany.cuh", "sfo_newton.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

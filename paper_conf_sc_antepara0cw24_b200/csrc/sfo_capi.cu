@@ -323,6 +323,23 @@ int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t
     return cuda_status();
 }
 
+int stokesfo_lateral_pressure(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
+                              double rho_i_g, double rho_w_g, double sea_level, double *R) {
+    if (!c || nfaces < 0) return STOKESFO_EINVAL;
+    if (nfaces == 0) return STOKESFO_OK;
+    if (!faces || !surface || !R || !aligned(faces, 8) || !aligned(R, 16)) return STOKESFO_EINVAL;
+    const int bs = 128;
+    const unsigned g = (unsigned)((nfaces + bs - 1) / bs);
+    const int64_t C = c->d.num_cells;
+    if (c->N == 8)
+        lateral_pressure_kernel<Hex8><<<g, bs, 0, c->stream>>>(nfaces, C, faces, c->d.conn, c->d.coords, surface,
+                                                                rho_i_g, rho_w_g, sea_level, R, c->err);
+    else
+        lateral_pressure_kernel<Wedge6><<<g, bs, 0, c->stream>>>(nfaces, C, faces, c->d.conn, c->d.coords, surface,
+                                                                  rho_i_g, rho_w_g, sea_level, R, c->err);
+    return cuda_status();
+}
+
 int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, const double *J_cell,
                               double *csr_vals) {
     if (!c) return STOKESFO_EINVAL;

@@ -997,6 +997,84 @@ __global__ void basal_friction_kernel(int64_t nfaces, const int32_t *__restrict_
 }
 
 // ---------------------------------------------------------------------------
+// NEXT-4: lateral (calving-front) pressure side-set term (PAPER.md P:L59 ->
+// [24]; reading Z19).  Thread <-> face (cell, side k): the quad over the
+// footprint edge k -> k+1, local nodes (k, k+1, k+1+P, k+P) (P = N/2, mod P).
+// 2x2 Gauss; n dGamma = dx/dxi x dx/deta (face-local coordinates, outward for
+// CCW footprints); psi = rho_i g (s_h - z_h) - rho_w g max(z_sl - z_h, 0);
+// R[i][a] -= sum_q psi n_a dGamma phi_i.  Independent of U (no Jacobian term).
+// ---------------------------------------------------------------------------
+template <class E>
+__global__ void lateral_pressure_kernel(int64_t nfaces, int64_t ncells, const int32_t *__restrict__ faces,
+                                        const int32_t *__restrict__ conn, const double *__restrict__ coords,
+                                        const double *__restrict__ surface, double rho_i_g, double rho_w_g,
+                                        double z_sl, double *__restrict__ R, int *__restrict__ err) {
+    constexpr int N = E::N, P = N / 2;
+    const int64_t f = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (f >= nfaces) return;
+    const int2 cs = reinterpret_cast<const int2 *>(faces)[f];
+    const int64_t cell = cs.x;
+    const int k = cs.y;
+    if (k < 0 || k >= P || cell < 0 || cell >= ncells) {
+        atomicOr(err, ERR_CONN);
+        return;
+    }
+    const int k1 = (k + 1 == P) ? 0 : k + 1;
+    const int loc[4] = {k, k1, k1 + P, k + P};
+    int32_t nid[4];
+    double x[4][3], sn[4];
+#pragma unroll
+    for (int n = 0; n < 4; ++n) {
+        nid[n] = __ldg(conn + cell * N + loc[n]);
+        sn[n] = __ldg(surface + nid[n]);
+#pragma unroll
+        for (int r = 0; r < 3; ++r) x[n][r] = __ldg(coords + 3 * (int64_t)nid[n] + r);
+    }
+    const double z0 = x[0][2];
+    const double g = 0.5773502691896257645;  // 1/sqrt(3)
+    double Rf[4][2] = {};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const double xi = (q & 1) ? g : -g, et = (q & 2) ? g : -g;
+        double phi[4], dxi[4], det[4];
+#pragma unroll
+        for (int n = 0; n < 4; ++n) {
+            const double sx = (n == 1 || n == 2) ? 1.0 : -1.0, sy = (n >= 2) ? 1.0 : -1.0;
+            phi[n] = 0.25 * (1.0 + sx * xi) * (1.0 + sy * et);
+            dxi[n] = 0.25 * sx * (1.0 + sy * et);
+            det[n] = 0.25 * (1.0 + sx * xi) * sy;
+        }
+        double t0[3] = {0, 0, 0}, t1[3] = {0, 0, 0};
+        double zq = 0.0, sq = 0.0;
+#pragma unroll
+        for (int n = 0; n < 4; ++n) {
+#pragma unroll
+            for (int r = 0; r < 3; ++r) {
+                const double xl = x[n][r] - x[0][r];  // face-local (reading Z17)
+                t0[r] = fma(xl, dxi[n], t0[r]);
+                t1[r] = fma(xl, det[n], t1[r]);
+            }
+            zq = fma(x[n][2] - z0, phi[n], zq);
+            sq = fma(sn[n], phi[n], sq);
+        }
+        zq += z0;  // sum_n phi_n = 1
+        const double n0 = t0[1] * t1[2] - t0[2] * t1[1];
+        const double n1 = t0[2] * t1[0] - t0[0] * t1[2];
+        const double psi = rho_i_g * (sq - zq) - rho_w_g * fmax(z_sl - zq, 0.0);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            Rf[i][0] = fma(-psi * n0, phi[i], Rf[i][0]);
+            Rf[i][1] = fma(-psi * n1, phi[i], Rf[i][1]);
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        atomicAdd(R + 2 * (int64_t)nid[i], Rf[i][0]);
+        atomicAdd(R + 2 * (int64_t)nid[i] + 1, Rf[i][1]);
+    }
+}
+
+// ---------------------------------------------------------------------------
 // G5: assembly.  R part: thread <-> (cell, node).  CSR part: thread <-> (cell, row).
 // ---------------------------------------------------------------------------
 template <int N>

@@ -79,4 +79,36 @@ int stokesfo_mesh_halo_list(int64_t n_mine, const int64_t *gids_mine, int64_t n_
     return STOKESFO_OK;
 }
 
+int stokesfo_mesh_lateral_faces(int32_t npoly, int64_t nf, const int32_t *polys, int32_t L, int64_t *nfaces,
+                                int32_t *faces) {
+    if ((npoly != 3 && npoly != 4) || nf < 0 || L < 1 || !nfaces || (nf > 0 && !polys)) return STOKESFO_EINVAL;
+    if (nf * (int64_t)L > INT32_MAX) return STOKESFO_EINVAL;
+    // undirected edge key (min, max) of every polygon side; a boundary side is
+    // one whose key occurs once.  Sort the keys, then look each side up.
+    std::vector<std::pair<int64_t, int64_t>> keys;
+    keys.reserve((size_t)(nf * npoly));
+    auto key = [&](int64_t f, int m) {
+        const int64_t a = polys[f * npoly + m], b = polys[f * npoly + (m + 1) % npoly];
+        return std::make_pair(std::min(a, b), std::max(a, b));
+    };
+    for (int64_t f = 0; f < nf; ++f)
+        for (int m = 0; m < npoly; ++m) keys.push_back(key(f, m));
+    std::sort(keys.begin(), keys.end());
+    int64_t n = 0;
+    for (int64_t f = 0; f < nf; ++f)
+        for (int m = 0; m < npoly; ++m) {
+            const auto kk = key(f, m);
+            const auto r = std::equal_range(keys.begin(), keys.end(), kk);
+            if (r.second - r.first != 1) continue;
+            if (faces)
+                for (int32_t l = 0; l < L; ++l) {  // (f, side, layer) order; cell = f L + l (reading Z10)
+                    faces[2 * (n + l) + 0] = (int32_t)(f * L + l);
+                    faces[2 * (n + l) + 1] = m;
+                }
+            n += L;
+        }
+    *nfaces = n;
+    return STOKESFO_OK;
+}
+
 }  // extern "C"

@@ -55,7 +55,8 @@ EXPORTS = [
     "stokesfo_albany_scratch_size", "stokesfo_albany_setup", "stokesfo_albany_evaluators",
     "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp", "stokesfo_basal_friction",
     "stokesfo_set_remote", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
-    "stokesfo_newton_work_size", "stokesfo_newton_solve",
+    "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
+    "stokesfo_mesh_lateral_faces",
 ]
 
 
@@ -89,6 +90,9 @@ def _lib():
             L.stokesfo_jvp.argtypes = [P, P, P, P, P]
         if hasattr(L, "stokesfo_basal_friction"):
             L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
+        if hasattr(L, "stokesfo_lateral_pressure"):
+            L.stokesfo_lateral_pressure.argtypes = [P, P, I64, P, D, D, D, P]
+            L.stokesfo_mesh_lateral_faces.argtypes = [I32, I64, P, I32, ctypes.POINTER(I64), P]
         if hasattr(L, "stokesfo_newton_solve"):
             L.stokesfo_newton_work_size.argtypes = [P, I64, ctypes.POINTER(ctypes.c_size_t)]
             L.stokesfo_newton_solve.argtypes = [P, P, I64, P, P, P, ctypes.POINTER(NewtonOpts), P, P,
@@ -248,6 +252,18 @@ class StokesFO:
         _check(_lib().stokesfo_basal_friction(self._h, _ptr(basal_cells), int(basal_cells.numel()), _ptr(beta),
                                               _ptr(U), _ptr(R), _ptr(J_face)), "basal_friction")
 
+    def lateral_pressure(self, faces, surface, R, rho_i_g=8.927, rho_w_g=10.05, sea_level=0.0):
+        """R -= lateral (calving-front) pressure term on faces (int32 cuda [nfaces][2] = (cell, side))."""
+        import torch
+        _dev(faces, torch.int32, None, "faces")
+        if faces.dim() != 2 or faces.shape[1] != 2:
+            raise ValueError("faces must have shape [nfaces][2]")
+        _dev(surface, torch.float64, (self.num_nodes,), "surface")
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_lateral_pressure(self._h, _ptr(faces), int(faces.shape[0]), _ptr(surface),
+                                                float(rho_i_g), float(rho_w_g), float(sea_level), _ptr(R)),
+               "lateral_pressure")
+
     def newton_solve(self, basal_cells, beta, U, max_newton=8, max_cg=500, max_ls=20, rtol_newton=1e-10,
                      atol_newton=0.0, rtol_cg=1e-6, ls_c=1e-4):
         """Damped Newton-Krylov solve of R_visc(U) + R_basal(U) = 0 in place on U
@@ -370,6 +386,18 @@ def mesh_extrude(xy, polys, b, H, L: int):
     _check(_lib().stokesfo_mesh_extrude(npoly, nv, _ptr(xy), nf, _ptr(polys), _ptr(b), _ptr(H), L,
                                         _ptr(conn), _ptr(coords)), "mesh_extrude")
     return conn, coords
+
+
+def mesh_lateral_faces(polys, L: int):
+    """(cell, side) of every lateral face over the footprint boundary, ordered by (f, side, layer)."""
+    polys = np.ascontiguousarray(polys, dtype=np.int32)
+    nf, npoly = polys.shape
+    n = ctypes.c_int64(0)
+    _check(_lib().stokesfo_mesh_lateral_faces(npoly, nf, _ptr(polys), L, ctypes.byref(n), None), "mesh_lateral_faces")
+    faces = np.empty((n.value, 2), dtype=np.int32)
+    _check(_lib().stokesfo_mesh_lateral_faces(npoly, nf, _ptr(polys), L, ctypes.byref(n), _ptr(faces)),
+           "mesh_lateral_faces")
+    return faces
 
 
 def mesh_partition_columns(nf: int, nparts: int):

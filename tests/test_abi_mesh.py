@@ -121,3 +121,24 @@ def test_create_rejects_bad_descriptors_without_gpu():
     n = ctypes.c_size_t()
     assert lib.stokesfo_workspace_size(ctypes.byref(desc(geometry_mode=1)), ctypes.byref(n)) == 0
     assert n.value == 256 + ((10 * 32 + 255) // 256) * 256      # header + double4 coordinates
+
+
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_lateral_faces_bit_exact_vs_oracle(elem):
+    """NEXT-4 (reading Z19): the library's boundary-side set equals the oracle's set algebra."""
+    from oracle import lateral as LT
+    fp = synth.tiny_footprint(n=7, jitter=0.2, seed=4)
+    if elem == "wedge6":
+        fp = synth.split_to_triangles(fp)
+    for L in (1, 4):
+        got = S.mesh_lateral_faces(fp.polys, L)
+        assert np.array_equal(got, LT.lateral_faces(fp.polys, L))
+
+
+def test_lateral_faces_antarctica_vs_oracle():
+    """C4 footprint (ragged, masked margin with embayments): same set, bit-exact."""
+    from oracle import lateral as LT
+    fp = synth.antarctica_footprint(h=16.0)
+    got = S.mesh_lateral_faces(fp.polys, 2)
+    assert got.shape[0] > 0
+    assert np.array_equal(got, LT.lateral_faces(fp.polys, 2))

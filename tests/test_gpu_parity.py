@@ -330,3 +330,31 @@ def test_basal_friction_parity(torch, elem):
     sc = np.abs(Jr).reshape(cells.size, -1).max(1)
     assert (np.abs(Jg - Jr).reshape(cells.size, -1).max(1) <= TOL * sc).all()
     assert np.abs(R.cpu().numpy() - Rr).max() <= TOL * np.abs(Rr).max()
+
+
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_lateral_pressure_parity(torch, elem):
+    """NEXT-4 (reading Z19): GPU lateral (calving-front) pressure term vs the numpy
+    oracle on every footprint-boundary face; sea level cuts through the faces of
+    some columns (above-, below- and straddling-water faces all occur)."""
+    from oracle import lateral as LT
+    L = 5
+    ctx, orc = _setup(torch, elem, n=8, L=L)
+    faces = LT.lateral_faces(M.tiny(elem, n=8, L=L)[0].polys, L)
+    z = orc["coords"][:, 2]
+    zsl = 0.5 * (z.min() + z.max())
+    assert (z < zsl).any() and (z > zsl).any()
+    R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+    ctx.lateral_pressure(_t(torch, faces), _t(torch, orc["s"]), R, rho_i_g=8.927, rho_w_g=10.05, sea_level=zsl)
+    ctx.sync()
+    Rr, F = LT.lateral_pressure(ctx.N, orc["conn"], orc["coords"], faces, orc["s"],
+                                8.927, 10.05, zsl)
+    assert np.abs(Rr).max() > 0
+    assert np.abs(R.cpu().numpy() - Rr).max() <= TOL * np.abs(Rr).max()
+    # a side index outside [0, P) raises the sticky EMESH flag
+    bad = faces[:1].copy()
+    bad[0, 1] = ctx.N // 2
+    ctx.lateral_pressure(_t(torch, bad), _t(torch, orc["s"]), R)
+    from paper_conf_sc_antepara0cw24_b200.stokesfo import StokesFOError
+    with pytest.raises(StokesFOError):
+        ctx.sync()
