@@ -35,7 +35,8 @@ WORKLOADS = {
 }
 
 
-def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored", op: str = "jacobian") -> int:
+def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored", op: str = "jacobian",
+                     nnz: int = 0) -> int:
     """Algorithmic (compulsory) HBM bytes of one stokesfo_jacobian launch with
     assembled R.
     stored:     per cell conn 4N + GradBF 24NQ + wMeasure 8Q + k_c 8 + J_cell 8(2N)^2;
@@ -46,10 +47,16 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
     Q = N
     J = 8 * (2 * N) ** 2 if op == "jacobian" else 0
     xy = (16 + 32) if op == "jvp" else 0  # X gather, Y read+write
+    if op == "jac_csr":
+        # NEXT-2 fused CSR: no J_cell; per cell the slot row 8N, per node the
+        # rowptr pair 16, and every CSR value read + written once (16 nnz)
+        J = 8 * N
+        xy = 16
+    vals = 16 * nnz if op == "jac_csr" else 0
     if geometry == "on_the_fly":
-        return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32 + xy)
+        return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32 + xy) + vals
     per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + J
-    return cells * per_cell + nodes * (16 + 8 + 32 + xy)
+    return cells * per_cell + nodes * (16 + 8 + 32 + xy) + vals
 
 
 def load_peaks():
@@ -201,7 +208,7 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly"])
-    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp"],
+    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jac_csr"],
                     help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
                          "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
     ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
@@ -252,6 +259,12 @@ def main():
     Xd = torch.from_numpy(np.random.default_rng(5).normal(0, 10.0, (NN, 2))).to(dev) if args.op == "jvp" else None
     Yd = torch.zeros((NN, 2), dtype=torch.float64, device=dev) if args.op == "jvp" else None
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
+    nnz, vals = 0, None
+    if args.op == "jac_csr":   # NEXT-2: pattern + slot table once per mesh (untimed)
+        _, colidx = ctx.csr_pattern()
+        ctx.csr_slots()
+        nnz = int(colidx.numel())
+        vals = torch.zeros(nnz, dtype=torch.float64, device=dev)
     halo = None
     p2p = None
     halo_mode = "none"
@@ -280,10 +293,14 @@ def main():
         else:
             Rc = R
             Rc.zero_()
+        if vals is not None:
+            vals.zero_()
         if i is not None:
             k0[i].record(stream)
         if args.op == "jacobian":
             ctx.jacobian(U, J, R=Rc)
+        elif args.op == "jac_csr":
+            ctx.jacobian_csr(U, vals, R=Rc)
         elif args.op == "jvp":
             ctx.jvp(U, Xd, Yd, R=Rc)
         else:
@@ -352,8 +369,12 @@ def main():
                     stream.wait_event(ev_d2h[b])        # R[b] of step t-2 has been downloaded
                 Rc = Rb[b]
                 Rc.zero_()
+            if vals is not None:
+                vals.zero_()
             if args.op == "jacobian":
                 ctx.jacobian(Ub[b], J, R=Rc)
+            elif args.op == "jac_csr":
+                ctx.jacobian_csr(Ub[b], vals, R=Rc)
             elif args.op == "jvp":
                 ctx.jvp(Ub[b], Xd, Yd, R=Rc)
             else:
@@ -417,7 +438,7 @@ def main():
 
     if rank == 0:
         peak, peak_src = load_peaks()
-        bpl = bytes_per_launch(elem, C, NN, args.geometry, args.op)
+        bpl = bytes_per_launch(elem, C, NN, args.geometry, args.op, nnz)
         achieved = bpl / (kern_ms_max * 1e-3) / 1e9
         traffic = None
         tpath = os.path.join(ROOT, "profiles", "traffic.json")
@@ -429,9 +450,11 @@ def main():
                 traffic = tr[key]["dram_bytes_per_launch"]
         l2_bytes = 126 * 2 ** 20
         line = {
-            "metric": METRIC if args.op == "jacobian" else (
-                "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s" if args.op == "resid"
-                else "Stokes-FO matrix-free J(U)X + residual (stokesfo_jvp) cells/s and achieved HBM GB/s"),
+            "metric": {"jacobian": METRIC,
+                       "resid": "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s",
+                       "jvp": "Stokes-FO matrix-free J(U)X + residual (stokesfo_jvp) cells/s and achieved HBM GB/s",
+                       "jac_csr": "Stokes-FO residual + Jacobian assembled into global CSR (stokesfo_jacobian_csr) "
+                                  "cells/s and achieved HBM GB/s"}[args.op],
             "value": total_cells / (ms_step * 1e-3),
             "unit": "cells/s",
             "n_gpus": world,
@@ -453,9 +476,9 @@ def main():
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel": ("eval_otf_kernel" if args.geometry == "on_the_fly" else "eval_kernel")
                          + ("<Hex8," if elem == "hex8" else "<Wedge6,")
-                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>"}[args.op]
+                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>"}[args.op]
                          + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
-                            "jvp": " (stokesfo_jvp)"}[args.op],
+                            "jvp": " (stokesfo_jvp)", "jac_csr": " (stokesfo_jacobian_csr)"}[args.op],
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src},
             "achieved_hbm_gbs": achieved,
             "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),
@@ -464,6 +487,8 @@ def main():
         }
         if check is not None:
             line["halo_check_max_rel_err"] = check
+        if nnz:
+            line["config"]["csr_nnz"] = nnz
         if e2e:
             line["e2e"] = {"value": total_cells / (e2e_ms * 1e-3), "unit": "cells/s",
                            "h2d_bytes_per_step": e2e[1], "d2h_bytes_per_step": e2e[2],

@@ -25,7 +25,7 @@ struct stokesfo_ctx {
     char *recs;            // device records (full or light)
     double4 *xyz4;         // node coordinates (on-the-fly geometry mode)
     int mode;              // stokesfo_geometry_mode_t
-    int grid_resid, grid_jac, grid_jvp;
+    int grid_resid, grid_jac, grid_jvp, grid_csr;
     int rec_bytes;
     int nstage_resid, nstage_jac;  // TMA record ring depth of the eval kernels
     const int32_t *rem = nullptr;     // fused halo over peer memory (stokesfo_set_remote)
@@ -34,6 +34,8 @@ struct stokesfo_ctx {
     const int64_t *rowptr = nullptr;  // CSR pattern (set by stokesfo_csr_pattern)
     const int32_t *colidx = nullptr;
     int64_t csr_rows = 0;
+    int64_t csr_maxdeg = 0;            // max neighbour nodes of a node (slots are uint8)
+    const uint64_t *slots = nullptr;   // per-cell CSR slots (set by stokesfo_csr_slots)
 };
 
 namespace {
@@ -113,6 +115,8 @@ int create_impl(stokesfo_ctx *c) {
         if (st) return st;
         st = configure_otf<E, M_JVP>(&c->grid_jvp);
         if (st) return st;
+        st = configure_otf<E, M_CSR>(&c->grid_csr);
+        if (st) return st;
     } else {
         // ring depth: default per element, STOKESFO_STAGES_{RESID,JAC} override (2 or 3)
         c->nstage_resid = default_stages<E, false>();
@@ -126,6 +130,8 @@ int create_impl(stokesfo_ctx *c) {
                                 : configure_eval<E, M_JAC, 2>(&c->grid_jac);
         if (st) return st;
         st = configure_eval<E, M_JVP, 2>(&c->grid_jvp);
+        if (st) return st;
+        st = configure_eval<E, M_CSR, 2>(&c->grid_csr);
         if (st) return st;
     }
     if (cudaMemsetAsync(c->err, 0, sizeof(int), c->stream) != cudaSuccess) return cuda_status();
@@ -150,7 +156,7 @@ int create_impl(stokesfo_ctx *c) {
 
 template <class E, int MODE>
 int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R, double *J_cell,
-              const double *X = nullptr, double *Y = nullptr) {
+              const double *X = nullptr, double *Y = nullptr, double *csr_vals = nullptr) {
     if (c->ntiles == 0) return STOKESFO_OK;
     EvalArgs a;
     a.recs = c->recs;
@@ -175,12 +181,17 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.rem = c->rem;
     a.remtab = c->remtab;
     a.peers = c->peers;
-    const int g = MODE == M_JAC ? c->grid_jac : (MODE == M_JVP ? c->grid_jvp : c->grid_resid);
+    a.rowptr = c->rowptr;
+    a.slots = c->slots;
+    a.csr_vals = csr_vals;
+    const int g = MODE == M_JAC ? c->grid_jac
+                : MODE == M_JVP ? c->grid_jvp
+                : MODE == M_CSR ? c->grid_csr : c->grid_resid;
     const int grid = (int)std::min<int64_t>(g, c->ntiles);
-    const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_JVP ? 2 : c->nstage_resid);
+    const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_RESID ? c->nstage_resid : 2);
     if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY)
         eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
-    else if (ns == 3)
+    else if (MODE != M_CSR && ns == 3)
         eval_kernel<E, MODE, 3><<<grid, 32, EvalSmem<E, MODE, 3>::BYTES, c->stream>>>(a);
     else
         eval_kernel<E, MODE, 2><<<grid, 32, EvalSmem<E, MODE, 2>::BYTES, c->stream>>>(a);
@@ -296,6 +307,40 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
 #undef CALL
 }
 
+int stokesfo_jacobian_csr(stokesfo_ctx *c, const double *U, double *csr_vals, double *R) {
+    if (!c) return STOKESFO_EINVAL;
+    if (c->d.num_cells == 0) return STOKESFO_OK;
+    if (!c->slots || !c->rowptr) return STOKESFO_EINVAL;  // needs stokesfo_csr_slots
+    if (!U || !csr_vals || !aligned(U, 16) || !aligned(csr_vals, 16) || (R && !aligned(R, 16)))
+        return STOKESFO_EINVAL;
+#define CALL(E) eval_impl<E, M_CSR>(c, U, nullptr, nullptr, R, nullptr, nullptr, nullptr, csr_vals)
+    return DISPATCH(c, CALL);
+#undef CALL
+}
+
+int stokesfo_csr_slots_size(stokesfo_ctx *c, size_t *bytes) {
+    if (!c || !bytes) return STOKESFO_EINVAL;
+    *bytes = (size_t)(c->d.num_cells * c->N * 8);
+    return STOKESFO_OK;
+}
+
+int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots) {
+    if (!c || !slots || !aligned(slots, 16)) return STOKESFO_EINVAL;
+    if (!c->rowptr || !c->colidx) return STOKESFO_EINVAL;  // needs the stokesfo_csr_pattern fill
+    if (c->csr_maxdeg > 256) return STOKESFO_EUNSUPPORTED;
+    const int64_t work = c->d.num_cells * c->N;
+    if (work > 0) {
+        const int bs = 256;
+        const unsigned g = (unsigned)((work + bs - 1) / bs);
+        if (c->N == 8)
+            csr_slots_kernel<8><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.conn, c->rowptr, c->colidx, slots, c->err);
+        else
+            csr_slots_kernel<6><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.conn, c->rowptr, c->colidx, slots, c->err);
+    }
+    c->slots = slots;
+    return cuda_status();
+}
+
 int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, double *R) {
     if (!c) return STOKESFO_EINVAL;
     if (c->d.num_cells == 0) return STOKESFO_OK;
@@ -359,7 +404,12 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
         if (!c->rowptr || !c->colidx) return STOKESFO_EINVAL;
         const int64_t work = C * 2 * c->N;
         const unsigned g = (unsigned)((work + bs - 1) / bs);
-        if (c->N == 8)
+        if (c->slots) {  // slot table attached: no per-entry search
+            if (c->N == 8)
+                scatter_csr_slots_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->slots, csr_vals);
+            else
+                scatter_csr_slots_kernel<6><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->slots, csr_vals);
+        } else if (c->N == 8)
             scatter_csr_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->colidx, csr_vals, c->err);
         else
             scatter_csr_kernel<6><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->colidx, csr_vals, c->err);
@@ -742,7 +792,10 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
         rp[2 * v + 2] = rp[2 * v + 1] + deg;
     }
     *nnz = rp[2 * NN];
+    int64_t maxdeg = 0;
+    for (int64_t v = 0; v < NN; ++v) maxdeg = std::max(maxdeg, nstart[v + 1] - nstart[v]);
     if (!rowptr || !colidx) return STOKESFO_OK;
+    if (!aligned(rowptr, 16)) return STOKESFO_EINVAL;  // (rowptr[2v], rowptr[2v+1]) pairs are loaded as 16 B
     if (!aligned(rowptr, 8) || !aligned(colidx, 4)) return STOKESFO_EINVAL;
     std::vector<int32_t> ci((size_t)*nnz);
     for (int64_t v = 0; v < NN; ++v)
@@ -762,6 +815,8 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
     c->rowptr = rowptr;
     c->colidx = colidx;
     c->csr_rows = 2 * NN;
+    c->csr_maxdeg = maxdeg;
+    c->slots = nullptr;  // a new pattern invalidates an attached slot table
     return STOKESFO_OK;
 }
 

@@ -263,6 +263,11 @@ struct EvalArgs {
     const int32_t *rem;
     const int32_t *remtab;
     double *const *peers;
+    // NEXT-2 fused CSR assembly (M_CSR): J contributions go straight into
+    // csr_vals[rowptr[2 g_i + a] + 2 slot[c][i][j] + b] (no element matrices)
+    const int64_t *rowptr;    // [2 nodes + 1]
+    const uint64_t *slots;    // [C][N] rows of N uint8 slots (8-byte pitch)
+    double *csr_vals;         // [nnz] (+=)
 };
 
 constexpr int REM_MAX = 7;                 // remote copies of one node (<= 8 parts meet at a vertex)
@@ -290,7 +295,12 @@ __device__ __forceinline__ void scatter_node(const EvalArgs &a, int32_t node, do
 }
 
 // Evaluation modes of the fused kernels
-enum { M_RESID = 0, M_JAC = 1, M_JVP = 2 };
+enum { M_RESID = 0, M_JAC = 1, M_JVP = 2, M_CSR = 3 };
+// modes that form the tangent blocks (element matrices or CSR contributions)
+template <int MODE>
+__host__ __device__ constexpr bool forms_jac() {
+    return MODE == M_JAC || MODE == M_CSR;
+}
 // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 beta12, wmu2, gamma, wf0, wf1
 // (+ for M_JVP: dbeta00 dbeta01 dbeta02 dbeta11 dbeta12, gamma * tau)
 constexpr int NQS = 9;
@@ -373,7 +383,7 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
                                                 double &R0, double &R1, double (&Jb)[E::N / 2 + 1][2][2], double &dR0,
                                                 double &dR1, PF pf) {
     constexpr int N = E::N, Q = E::Q, K = N / 2;
-    constexpr bool JAC = MODE == M_JAC;
+    constexpr bool JAC = forms_jac<MODE>();
     R0 = 0.0;
     R1 = 0.0;
     dR0 = 0.0;
@@ -473,6 +483,54 @@ __device__ __forceinline__ void store_J(double *J_cell, int64_t cell0, int nvali
     bulk_commit();
 }
 
+// NEXT-2 fused assembly: lane (c, i) adds its tangent blocks into the CSR
+// values through the per-cell slot table -- direct blocks (i, i+k), k = 0..K,
+// and, by symmetry, the transposed blocks (i+k, i) for 0 < k < K (the same
+// split as stage_J).  Row bases rp = (rowptr[2 g_i], rowptr[2 g_i + 1]) and
+// slot rows of the partner nodes come from their lanes by shuffle.  Every lane
+// of the warp must call this (shuffles); `live` gates the atomics.
+template <class E>
+__device__ __forceinline__ void csr_scatter(double *vals, int c, int i, bool live, uint64_t srow, longlong2 rp,
+                                            const double (&Jb)[E::N / 2 + 1][2][2]) {
+    constexpr int N = E::N, K = N / 2;
+    const int cc = c < E::TC ? c : 0;
+#pragma unroll
+    for (int k = 0; k <= K; ++k) {
+        const int j = (i + k) % N;
+        const int src = E::lane_of(cc, j);
+        const uint64_t srow_j = __shfl_sync(0xffffffffu, srow, src);
+        const long long rj0 = __shfl_sync(0xffffffffu, rp.x, src);
+        const long long rj1 = __shfl_sync(0xffffffffu, rp.y, src);
+        if (live) {
+            const int sij = (int)((srow >> (8 * j)) & 0xff);
+            double *p0 = vals + rp.x + 2 * sij, *p1 = vals + rp.y + 2 * sij;
+            atomicAdd(p0, Jb[k][0][0]);
+            atomicAdd(p0 + 1, Jb[k][0][1]);
+            atomicAdd(p1, Jb[k][1][0]);
+            atomicAdd(p1 + 1, Jb[k][1][1]);
+            if (k > 0 && k < K) {  // J[(j,a),(i,b)] = J[(i,b),(j,a)]
+                const int sji = (int)((srow_j >> (8 * i)) & 0xff);
+                double *q0 = vals + rj0 + 2 * sji, *q1 = vals + rj1 + 2 * sji;
+                atomicAdd(q0, Jb[k][0][0]);
+                atomicAdd(q0 + 1, Jb[k][1][0]);
+                atomicAdd(q1, Jb[k][0][1]);
+                atomicAdd(q1 + 1, Jb[k][1][1]);
+            }
+        }
+    }
+}
+
+// slot row and CSR row bases of lane (cell, node i), loaded ahead of use
+__device__ __forceinline__ void csr_row_load(const EvalArgs &a, int64_t cell, int32_t g, bool live, uint64_t &srow,
+                                             longlong2 &rp, int N, int i) {
+    srow = 0;
+    rp = make_longlong2(0, 0);
+    if (live) {
+        srow = __ldg(a.slots + cell * N + i);
+        rp = __ldg(reinterpret_cast<const longlong2 *>(a.rowptr) + g);
+    }
+}
+
 template <class E>
 __device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
 #pragma unroll
@@ -487,7 +545,7 @@ __device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
 // Jacobian accumulators, 16 for the residual-only kernels: <= 128 registers).
 template <class E, int MODE>
 constexpr int warps_per_sm() {
-    return MODE == M_JAC ? 12 : 16;
+    return forms_jac<MODE>() ? 12 : 16;
 }
 
 // ---- G3/G4 with stored geometry (the §8(a2) precompute streamed per tile) ----
@@ -552,7 +610,7 @@ __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
 template <class E, int MODE, int NSTAGE>
 __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
-    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP;
+    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
     static_assert(N == Q, "lane mappings assume N == Q");
     using R = Rec<E>;
     using S = EvalSmem<E, MODE, NSTAGE>;
@@ -653,10 +711,14 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
         };
         double R0 = 0.0, R1 = 0.0, dR0 = 0.0, dR1 = 0.0;
         double Jb[N / 2 + 1][2][2];
+        uint64_t srow = 0;
+        longlong2 rp = make_longlong2(0, 0);
+        if (CSR) csr_row_load(a, cell0 + c, gnode, act && c < nvalid, srow, rp, N, s);
         if (act) node_accumulate<E, MODE>(rg, qs, c, s, bfi, R0, R1, Jb, dR0, dR1, prefetch);
         else prefetch();
         __syncwarp();  // every lane is done with this stage's record and qs
 
+        if (CSR) csr_scatter<E>(a.csr_vals, c, s, act && c < nvalid, srow, rp, Jb);
         if (JAC) {
             if (act) stage_J<E>(reinterpret_cast<double *>(stage), c, s, Jb);
             fence_proxy_async_smem();
@@ -731,7 +793,7 @@ template <class E, int MODE>
 __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_otf_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "lane mappings assume N == Q");
-    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP;
+    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
     using S = OtfSmem<E, MODE>;
     extern __shared__ __align__(128) char smem[];
     double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
@@ -860,9 +922,13 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_otf_kernel
         };
         double R0 = 0.0, R1 = 0.0, dR0 = 0.0, dR1 = 0.0;
         double Jb[N / 2 + 1][2][2];
+        uint64_t srow = 0;
+        longlong2 rp = make_longlong2(0, 0);
+        if (CSR) csr_row_load(a, cell0 + c, gnode, act && c < nvalid, srow, rp, N, s);
         if (act) node_accumulate<E, MODE>(rg, qs, c, s, bfi, R0, R1, Jb, dR0, dR1, prefetch);
         else prefetch();
         __syncwarp();  // G and qs are consumed
+        if (CSR) csr_scatter<E>(a.csr_vals, c, s, act && c < nvalid, srow, rp, Jb);
 
         if (JAC) {
             if (act) stage_J<E>(rg, c, s, Jb);
@@ -1110,6 +1176,56 @@ __global__ void scatter_csr_kernel(int64_t ncells, const int32_t *__restrict__ c
             atomicAdd(vals + lo, Jc[cell * ND * ND + r * ND + s]);
         else
             atomicOr(err, ERR_CSR);
+    }
+}
+
+// NEXT-2: per-cell CSR slots (thread <-> (cell, i)): slot[c][i][j] = index of
+// node g_j in the sorted neighbour list of g_i (binary search in row 2 g_i,
+// once per mesh), packed as N bytes of one uint64 per (cell, i).
+template <int N>
+__global__ void csr_slots_kernel(int64_t ncells, const int32_t *__restrict__ conn,
+                                 const int64_t *__restrict__ rowptr, const int32_t *__restrict__ colidx,
+                                 uint64_t *__restrict__ slots, int *__restrict__ err) {
+    const int64_t gid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (gid >= ncells * N) return;
+    const int64_t cell = gid / N;
+    const int64_t row = 2 * (int64_t)conn[gid];
+    const int64_t lo0 = rowptr[row], hi0 = rowptr[row + 1];
+    uint64_t w = 0;
+    for (int j = 0; j < N; ++j) {
+        const int32_t col = 2 * conn[cell * N + j];
+        int64_t lo = lo0, hi = hi0;
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (colidx[mid] < col) lo = mid + 1; else hi = mid;
+        }
+        const int64_t sl = (lo - lo0) >> 1;
+        if (lo < hi0 && colidx[lo] == col && sl < 256) w |= (uint64_t)sl << (8 * j);
+        else atomicOr(err, ERR_CSR);
+    }
+    slots[gid] = w;
+}
+
+// CSR assembly of element matrices through the slot table (thread <-> (cell, row)).
+template <int N>
+__global__ void scatter_csr_slots_kernel(int64_t ncells, const int32_t *__restrict__ conn,
+                                         const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
+                                         const uint64_t *__restrict__ slots, double *__restrict__ vals) {
+    constexpr int ND = 2 * N;
+    const int64_t gid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (gid >= ncells * ND) return;
+    const int64_t cell = gid / ND;
+    const int r = (int)(gid % ND);
+    const int i = r >> 1;
+    const uint64_t w = __ldg(slots + cell * N + i);
+    double *base = vals + __ldg(rowptr + 2 * (int64_t)conn[cell * N + i] + (r & 1));
+    const double2 *Jr = reinterpret_cast<const double2 *>(Jc + (cell * ND + r) * ND);
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+        const double2 v = __ldcs(Jr + j);  // streamed once
+        double *p = base + 2 * (int)((w >> (8 * j)) & 0xff);
+        atomicAdd(p, v.x);
+        atomicAdd(p + 1, v.y);
     }
 }
 

@@ -109,8 +109,17 @@ def main():
             emit("scatter_assemble:CSR", ms, nb, C, "cells",
                  {"nnz": nnz, "atomics_per_s": C * (2 * N) ** 2 / (ms * 1e-3),
                   "pattern_host_s": t_pat})
+            t0 = time.perf_counter()
+            ctx.csr_slots()
+            ctx.sync()
+            t_slots = time.perf_counter() - t0
+            ms = timed(lambda: ctx.scatter_assemble(J_cell=J, csr_vals=vals), stream, pre=vals.zero_)
+            ctx.sync()
+            nb = C * (4 * N + 8 * (2 * N) ** 2 + 8 * N) + 2 * NN * 8 + nnz * 16
+            emit("scatter_assemble:CSR(slots)", ms, nb, C, "cells",
+                 {"nnz": nnz, "atomics_per_s": C * (2 * N) ** 2 / (ms * 1e-3), "slots_setup_s": t_slots})
             del vals, rowptr, colidx
-            ctx.rowptr = ctx.colidx = None
+            ctx.rowptr = ctx.colidx = ctx.slots = None
         del J, Rc
         torch.cuda.empty_cache()
     if "basal" in ops:

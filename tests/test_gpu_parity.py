@@ -358,3 +358,47 @@ def test_lateral_pressure_parity(torch, elem):
     from paper_conf_sc_antepara0cw24_b200.stokesfo import StokesFOError
     with pytest.raises(StokesFOError):
         ctx.sync()
+
+
+@pytest.mark.parametrize("geometry", GEOMS)
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_csr_slots_and_fused_assembly(torch, elem, geometry):
+    """NEXT-2: per-cell CSR slots bit-exact vs the oracle's pattern (searchsorted),
+    slot-based scatter_assemble and the fused jacobian_csr (no element matrices)
+    vs the oracle's CSR scatter of its element Jacobians; ragged last tile."""
+    ctx, orc = _setup(torch, elem, n=5, L=3, drop=3, geometry=geometry)
+    C, N = ctx.num_cells, ctx.N
+    rowptr, colidx = ctx.csr_pattern()
+    rp2, ci2 = O.csr_pattern(orc["conn"], ctx.num_nodes)
+    slots = ctx.csr_slots().cpu().numpy().view(np.uint8).reshape(C, N, 8)[:, :, :N]
+    conn = orc["conn"]
+    want = np.zeros((C, N, N), dtype=np.uint8)
+    for c in range(C):
+        for i in range(N):
+            row = 2 * conn[c, i]
+            cols = ci2[rp2[row]:rp2[row + 1]]
+            for j in range(N):
+                k = int(np.searchsorted(cols, 2 * conn[c, j]))
+                assert cols[k] == 2 * conn[c, j]
+                want[c, i, j] = k // 2
+    assert np.array_equal(slots, want)
+    ref = O.evaluate(orc["e"], conn, orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"], mode="jac")
+    v2, miss = O.scatter_csr(orc["e"], conn, ref["J_cell"], rp2, ci2)
+    cell_scale = np.abs(ref["J_cell"]).reshape(C, -1).max(1)[:, None, None] * np.ones_like(ref["J_cell"])
+    a2, _ = O.scatter_csr(orc["e"], conn, cell_scale, rp2, ci2)
+    assert miss == 0
+    U = _t(torch, orc["U"])
+    # slot-based assembly of element matrices
+    J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
+    ctx.jacobian(U, J)
+    vals = torch.zeros(colidx.numel(), dtype=torch.float64, device="cuda")
+    ctx.scatter_assemble(J_cell=J, csr_vals=vals)
+    ctx.sync()
+    assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2).all()
+    # fused: residual + Jacobian straight into CSR
+    vals.zero_()
+    R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+    ctx.jacobian_csr(U, vals, R=R)
+    ctx.sync()
+    assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2).all()
+    _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
