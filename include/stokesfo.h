@@ -174,6 +174,28 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R,
  * dev [nnz] int32.  Synchronises the stream (host-side construction). */
 int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t *colidx);
 
+/* NEXT-2 per-cell CSR slots: slot[c][i][j] (uint8, j = 0..N-1, byte j of the
+ * uint64 slots[c*N + i]) = index of node conn[c][j] in the sorted neighbour-node
+ * list of node conn[c][i], so that J_cell[c][(i,a)][(j,b)] lands at
+ * csr_vals[rowptr[2 conn[c][i] + a] + 2 slot + b].  Requires an earlier
+ * stokesfo_csr_pattern fill (rowptr 16-B aligned); computed on the device once
+ * (binary searches in colidx) into caller-owned slots: dev uint64 [C][N]
+ * (stokesfo_csr_slots_size bytes, 16-B aligned, must stay valid).  Attaches
+ * the table to the ctx: stokesfo_scatter_assemble then uses it instead of
+ * per-entry searches, and stokesfo_jacobian_csr becomes available.  A node
+ * with more than 256 neighbour nodes returns EUNSUPPORTED; a missing entry
+ * raises the sticky EMESH flag.  A new stokesfo_csr_pattern fill detaches it. */
+int stokesfo_csr_slots_size(stokesfo_ctx *c, size_t *bytes);
+int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots);
+
+/* NEXT-2 fused: residual + forward-AD Jacobian assembled straight into the
+ * global CSR matrix in one pass (no element matrices in HBM; Albany's
+ * ScatterResidual into a CrsMatrix): csr_vals[...] += every
+ * cell's J contributions (red.global.add.f64 through the slot table), R += the
+ * residual (optional).  Requires stokesfo_csr_slots.  csr_vals: dev [nnz]
+ * (+=); U, R: dev [num_nodes][2].  Summation order is unspecified (atomics). */
+int stokesfo_jacobian_csr(stokesfo_ctx *c, const double *U, double *csr_vals, double *R);
+
 /* Export the precomputed geometry in the canonical layout:
  * grad_bf dev [C][N][Q][3], w_measure dev [C][Q] (either may be NULL). */
 int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure);

@@ -36,6 +36,10 @@ struct stokesfo_ctx {
     int64_t csr_rows = 0;
     int64_t csr_maxdeg = 0;            // max neighbour nodes of a node (slots are uint8)
     const uint64_t *slots = nullptr;   // per-cell CSR slots (set by stokesfo_csr_slots)
+    const int64_t *inc_ptr = nullptr;  // node -> (cell N + i) incidence on the device (in the slots buffer)
+    const int32_t *inc = nullptr;
+    std::vector<int64_t> inc_ptr_h;    // host incidence from the last csr_pattern fill (until csr_slots)
+    std::vector<int32_t> inc_h;
 };
 
 namespace {
@@ -318,9 +322,15 @@ int stokesfo_jacobian_csr(stokesfo_ctx *c, const double *U, double *csr_vals, do
 #undef CALL
 }
 
+// slots buffer: [slots C N uint64][inc_ptr (nodes+1) int64][inc C N int32]
+static int64_t slots_off_incptr(const stokesfo_ctx *c) { return round_up(c->d.num_cells * c->N * 8, 16); }
+static int64_t slots_off_inc(const stokesfo_ctx *c) {
+    return slots_off_incptr(c) + round_up((c->d.num_nodes + 1) * 8, 16);
+}
+
 int stokesfo_csr_slots_size(stokesfo_ctx *c, size_t *bytes) {
     if (!c || !bytes) return STOKESFO_EINVAL;
-    *bytes = (size_t)(c->d.num_cells * c->N * 8);
+    *bytes = (size_t)(slots_off_inc(c) + round_up(c->d.num_cells * c->N * 4, 16));
     return STOKESFO_OK;
 }
 
@@ -338,6 +348,22 @@ int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots) {
             csr_slots_kernel<6><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.conn, c->rowptr, c->colidx, slots, c->err);
     }
     c->slots = slots;
+    // node -> (cell, i) incidence for the atomic-free assembly kernel
+    char *base = reinterpret_cast<char *>(slots);
+    int64_t *ip = reinterpret_cast<int64_t *>(base + slots_off_incptr(c));
+    int32_t *in = reinterpret_cast<int32_t *>(base + slots_off_inc(c));
+    if ((int64_t)c->inc_ptr_h.size() == c->d.num_nodes + 1 && (int64_t)c->inc_h.size() == work) {
+        if (cudaMemcpyAsync(ip, c->inc_ptr_h.data(), c->inc_ptr_h.size() * 8, cudaMemcpyHostToDevice, c->stream) !=
+                cudaSuccess ||
+            (work > 0 &&
+             cudaMemcpyAsync(in, c->inc_h.data(), c->inc_h.size() * 4, cudaMemcpyHostToDevice, c->stream) != cudaSuccess) ||
+            cudaStreamSynchronize(c->stream) != cudaSuccess)
+            return cuda_status();
+        c->inc_ptr = ip;
+        c->inc = in;
+        std::vector<int64_t>().swap(c->inc_ptr_h);
+        std::vector<int32_t>().swap(c->inc_h);
+    }
     return cuda_status();
 }
 
@@ -393,6 +419,8 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
     const int64_t C = c->d.num_cells;
     const int bs = 256;
+    // STOKESFO_CSR_ATOMIC=1: slot-based atomic kernel instead of the pull kernel (A/B)
+    static const bool pull = !(getenv("STOKESFO_CSR_ATOMIC") && atoi(getenv("STOKESFO_CSR_ATOMIC")) == 1);
     if (R_cell && R && C > 0) {
         const int64_t work = C * c->N;
         const unsigned g = (unsigned)((work + bs - 1) / bs);
@@ -404,7 +432,16 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
         if (!c->rowptr || !c->colidx) return STOKESFO_EINVAL;
         const int64_t work = C * 2 * c->N;
         const unsigned g = (unsigned)((work + bs - 1) / bs);
-        if (c->slots) {  // slot table attached: no per-entry search
+        if (c->slots && c->inc && c->csr_maxdeg <= CSR_GATHER_MAXDEG && pull) {  // atomic-free, deterministic
+            const int64_t NN = c->d.num_nodes;
+            const unsigned gg = (unsigned)((NN + CSR_GATHER_WARPS - 1) / CSR_GATHER_WARPS);
+            if (c->N == 8)
+                csr_gather_kernel<8><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr,
+                                                                                 c->inc, c->slots, csr_vals);
+            else
+                csr_gather_kernel<6><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr,
+                                                                                 c->inc, c->slots, csr_vals);
+        } else if (c->slots) {  // slot table attached: no per-entry search
             if (c->N == 8)
                 scatter_csr_slots_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->slots, csr_vals);
             else
@@ -765,10 +802,11 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
     std::vector<int64_t> nc(NN + 1, 0);
     for (int64_t i = 0; i < C * N; ++i) nc[conn[i] + 1]++;
     for (int64_t v = 0; v < NN; ++v) nc[v + 1] += nc[v];
-    std::vector<int32_t> ncell(C * N);
+    if (C * N > INT32_MAX) return STOKESFO_EUNSUPPORTED;
+    std::vector<int32_t> ncell(C * N);  // node -> cell N + local index, ascending cell order
     {
         std::vector<int64_t> pos(nc.begin(), nc.end() - 1);
-        for (int64_t i = 0; i < C * N; ++i) ncell[pos[conn[i]]++] = (int32_t)(i / N);
+        for (int64_t i = 0; i < C * N; ++i) ncell[pos[conn[i]]++] = (int32_t)i;
     }
     // node -> sorted unique neighbour nodes
     std::vector<int64_t> rp(2 * NN + 1, 0);
@@ -778,7 +816,7 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
     for (int64_t v = 0; v < NN; ++v) {
         nb.clear();
         for (int64_t k = nc[v]; k < nc[v + 1]; ++k) {
-            const int64_t cell = ncell[k];
+            const int64_t cell = ncell[k] / N;
             for (int n = 0; n < N; ++n) nb.push_back(conn[cell * N + n]);
         }
         std::sort(nb.begin(), nb.end());
@@ -817,6 +855,10 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
     c->csr_rows = 2 * NN;
     c->csr_maxdeg = maxdeg;
     c->slots = nullptr;  // a new pattern invalidates an attached slot table
+    c->inc_ptr = nullptr;
+    c->inc = nullptr;
+    c->inc_ptr_h = std::move(nc);
+    c->inc_h = std::move(ncell);
     return STOKESFO_OK;
 }
 

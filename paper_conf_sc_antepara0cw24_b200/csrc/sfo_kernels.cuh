@@ -1229,6 +1229,54 @@ __global__ void scatter_csr_slots_kernel(int64_t ncells, const int32_t *__restri
     }
 }
 
+// Deterministic, atomic-free CSR assembly of element matrices ("pull"): one
+// warp per node v owns CSR rows 2v and 2v+1 (contiguous in vals), accumulates
+// the two rows of every incident cell's J (node -> (cell, local i) incidence,
+// ascending cell order) in a shared-memory row buffer through the slot table,
+// then adds the buffer to vals with coalesced stores.  Every J_cell element is
+// read once (by the warp of its row's node); no two warps touch the same entry.
+constexpr int CSR_GATHER_MAXDEG = 64;   // neighbour nodes per node (else the atomic kernel)
+constexpr int CSR_GATHER_WARPS = 8;
+template <int N>
+__global__ void __launch_bounds__(32 * CSR_GATHER_WARPS)
+    csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
+                      const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
+                      const uint64_t *__restrict__ slots, double *__restrict__ vals) {
+    constexpr int ND = 2 * N, NE = 2 * ND;  // entries of one node's two rows in one cell
+    constexpr int BATCH = 8;
+    __shared__ double buf[CSR_GATHER_WARPS][4 * CSR_GATHER_MAXDEG];
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    const int64_t v = blockIdx.x * (int64_t)CSR_GATHER_WARPS + w;
+    if (v >= nnodes) return;  // uniform per warp
+    double *b = buf[w];
+    const int64_t r0 = __ldg(rowptr + 2 * v);
+    const int len = (int)(__ldg(rowptr + 2 * v + 2) - r0);  // both rows: 4 deg entries
+    const int half = len >> 1;
+    for (int p = l; p < len; p += 32) b[p] = 0.0;
+    const int a = l / ND, col = l % ND, j = col >> 1, bb = col & 1;
+    const int64_t k0 = __ldg(inc_ptr + v), k1 = __ldg(inc_ptr + v + 1);
+    __syncwarp();
+    for (int64_t k = k0; k < k1; k += BATCH) {
+        const int cnt = (k1 - k < BATCH) ? (int)(k1 - k) : BATCH;
+        int32_t ci[BATCH];
+        double x[BATCH];
+        uint64_t sl[BATCH];
+#pragma unroll
+        for (int t = 0; t < BATCH; ++t) {  // independent loads of up to BATCH cells
+            ci[t] = t < cnt ? __ldg(inc + k + t) : 0;
+            const int64_t cell = ci[t] / N;
+            const int i = ci[t] - (int)(cell * N);
+            x[t] = (t < cnt && l < NE) ? __ldcs(Jc + (cell * ND + 2 * i + a) * ND + col) : 0.0;
+            sl[t] = t < cnt ? __ldg(slots + ci[t]) : 0;
+        }
+#pragma unroll
+        for (int t = 0; t < BATCH; ++t)
+            if (t < cnt && l < NE) b[a * half + 2 * (int)((sl[t] >> (8 * j)) & 0xff) + bb] += x[t];
+    }
+    __syncwarp();
+    for (int p = l; p < len; p += 32) vals[r0 + p] += b[p];
+}
+
 // ---------------------------------------------------------------------------
 // G7: halo pack / unpack-add.
 // ---------------------------------------------------------------------------

@@ -56,7 +56,7 @@ EXPORTS = [
     "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp", "stokesfo_basal_friction",
     "stokesfo_set_remote", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
     "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
-    "stokesfo_mesh_lateral_faces",
+    "stokesfo_mesh_lateral_faces", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
 ]
 
 
@@ -93,6 +93,10 @@ def _lib():
         if hasattr(L, "stokesfo_lateral_pressure"):
             L.stokesfo_lateral_pressure.argtypes = [P, P, I64, P, D, D, D, P]
             L.stokesfo_mesh_lateral_faces.argtypes = [I32, I64, P, I32, ctypes.POINTER(I64), P]
+        if hasattr(L, "stokesfo_jacobian_csr"):
+            L.stokesfo_csr_slots_size.argtypes = [P, ctypes.POINTER(ctypes.c_size_t)]
+            L.stokesfo_csr_slots.argtypes = [P, P]
+            L.stokesfo_jacobian_csr.argtypes = [P, P, P, P]
         if hasattr(L, "stokesfo_newton_solve"):
             L.stokesfo_newton_work_size.argtypes = [P, I64, ctypes.POINTER(ctypes.c_size_t)]
             L.stokesfo_newton_solve.argtypes = [P, P, I64, P, P, P, ctypes.POINTER(NewtonOpts), P, P,
@@ -298,6 +302,23 @@ class StokesFO:
                "csr_pattern")
         self.colidx = self.colidx[:int(nnz.value)]
         return self.rowptr, self.colidx
+
+    def csr_slots(self):
+        """Per-cell CSR slot table (stokesfo_csr_slots); needs csr_pattern() first."""
+        import torch
+        n = ctypes.c_size_t(0)
+        _check(_lib().stokesfo_csr_slots_size(self._h, ctypes.byref(n)), "csr_slots_size")
+        self.slots = torch.empty(max(int(n.value) // 8, 2), dtype=torch.int64, device=self.device)
+        _check(_lib().stokesfo_csr_slots(self._h, _ptr(self.slots)), "csr_slots")
+        return self.slots[:int(n.value) // 8]
+
+    def jacobian_csr(self, U, csr_vals, R=None):
+        """csr_vals += assembled Jacobian (fused, no element matrices); optionally R += residual."""
+        import torch
+        _dev(U, torch.float64, (self.num_nodes, 2), "U")
+        _dev(csr_vals, torch.float64, None, "csr_vals")
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_jacobian_csr(self._h, _ptr(U), _ptr(csr_vals), _ptr(R)), "jacobian_csr")
 
     def scatter_assemble(self, R_cell=None, R=None, J_cell=None, csr_vals=None):
         _check(_lib().stokesfo_scatter_assemble(self._h, _ptr(R_cell), _ptr(R), _ptr(J_cell), _ptr(csr_vals)),

@@ -116,7 +116,8 @@ def main():
             ms = timed(lambda: ctx.scatter_assemble(J_cell=J, csr_vals=vals), stream, pre=vals.zero_)
             ctx.sync()
             nb = C * (4 * N + 8 * (2 * N) ** 2 + 8 * N) + 2 * NN * 8 + nnz * 16
-            emit("scatter_assemble:CSR(slots)", ms, nb, C, "cells",
+            emit("scatter_assemble:CSR(slots, atomics)" if os.environ.get("STOKESFO_CSR_ATOMIC") == "1"
+                 else "scatter_assemble:CSR(slots, pull: warp per node, no atomics)", ms, nb, C, "cells",
                  {"nnz": nnz, "atomics_per_s": C * (2 * N) ** 2 / (ms * 1e-3), "slots_setup_s": t_slots})
             del vals, rowptr, colidx
             ctx.rowptr = ctx.colidx = ctx.slots = None

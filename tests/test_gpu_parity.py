@@ -395,6 +395,11 @@ def test_csr_slots_and_fused_assembly(torch, elem, geometry):
     ctx.scatter_assemble(J_cell=J, csr_vals=vals)
     ctx.sync()
     assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2).all()
+    # the slot-based assembly is atomic-free (one warp owns a node's two rows): bitwise reproducible
+    vals2 = torch.zeros_like(vals)
+    ctx.scatter_assemble(J_cell=J, csr_vals=vals2)
+    ctx.sync()
+    assert torch.equal(vals, vals2)
     # fused: residual + Jacobian straight into CSR
     vals.zero_()
     R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
