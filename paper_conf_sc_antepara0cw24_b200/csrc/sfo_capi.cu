@@ -434,7 +434,8 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
         const unsigned g = (unsigned)((work + bs - 1) / bs);
         if (c->slots && c->inc && c->csr_maxdeg <= CSR_GATHER_MAXDEG && pull) {  // atomic-free, deterministic
             const int64_t NN = c->d.num_nodes;
-            const unsigned gg = (unsigned)((NN + CSR_GATHER_WARPS - 1) / CSR_GATHER_WARPS);
+            const int64_t per_block = (int64_t)CSR_GATHER_WARPS * CSR_GATHER_NPW;
+            const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
             if (c->N == 8)
                 csr_gather_kernel<8><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr,
                                                                                  c->inc, c->slots, csr_vals);

@@ -1229,52 +1229,87 @@ __global__ void scatter_csr_slots_kernel(int64_t ncells, const int32_t *__restri
     }
 }
 
-// Deterministic, atomic-free CSR assembly of element matrices ("pull"): one
-// warp per node v owns CSR rows 2v and 2v+1 (contiguous in vals), accumulates
-// the two rows of every incident cell's J (node -> (cell, local i) incidence,
-// ascending cell order) in a shared-memory row buffer through the slot table,
-// then adds the buffer to vals with coalesced stores.  Every J_cell element is
-// read once (by the warp of its row's node); no two warps touch the same entry.
+// Deterministic, atomic-free CSR assembly of element matrices ("pull"): a
+// warp owns the CSR rows 2v, 2v+1 (contiguous in vals) of NPW nodes v at once,
+// accumulates the two rows of every incident cell's J (node -> (cell, local i)
+// incidence, ascending cell order) in a shared-memory row buffer through the
+// slot table, then adds the buffer to vals with coalesced stores.  Every
+// J_cell element is read once (by the warp of its row's node); no two warps
+// touch the same entry.  The NPW nodes' loads (incidence, up to 8 cells' J
+// rows and slot rows each) are all issued before any is consumed: the kernel
+// is a chain of dependent gathers, so memory-level parallelism per warp is
+// what sets its speed.
 constexpr int CSR_GATHER_MAXDEG = 64;   // neighbour nodes per node (else the atomic kernel)
 constexpr int CSR_GATHER_WARPS = 8;
+constexpr int CSR_GATHER_NPW = 2;       // nodes per warp
 template <int N>
-__global__ void __launch_bounds__(32 * CSR_GATHER_WARPS)
+__global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
     csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
                       const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
                       const uint64_t *__restrict__ slots, double *__restrict__ vals) {
     constexpr int ND = 2 * N, NE = 2 * ND;  // entries of one node's two rows in one cell
-    constexpr int BATCH = 8;
-    __shared__ double buf[CSR_GATHER_WARPS][4 * CSR_GATHER_MAXDEG];
+    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW;
+    __shared__ double buf[CSR_GATHER_WARPS][NPW][4 * CSR_GATHER_MAXDEG];
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
-    const int64_t v = blockIdx.x * (int64_t)CSR_GATHER_WARPS + w;
-    if (v >= nnodes) return;  // uniform per warp
-    double *b = buf[w];
-    const int64_t r0 = __ldg(rowptr + 2 * v);
-    const int len = (int)(__ldg(rowptr + 2 * v + 2) - r0);  // both rows: 4 deg entries
-    const int half = len >> 1;
-    for (int p = l; p < len; p += 32) b[p] = 0.0;
-    const int a = l / ND, col = l % ND, j = col >> 1, bb = col & 1;
-    const int64_t k0 = __ldg(inc_ptr + v), k1 = __ldg(inc_ptr + v + 1);
-    __syncwarp();
-    for (int64_t k = k0; k < k1; k += BATCH) {
-        const int cnt = (k1 - k < BATCH) ? (int)(k1 - k) : BATCH;
-        int32_t ci[BATCH];
-        double x[BATCH];
-        uint64_t sl[BATCH];
+    const int64_t v0 = (blockIdx.x * (int64_t)CSR_GATHER_WARPS + w) * NPW;
+    if (v0 >= nnodes) return;  // uniform per warp
+    int64_t r0[NPW], k0[NPW];
+    int len[NPW], cnt[NPW];
 #pragma unroll
-        for (int t = 0; t < BATCH; ++t) {  // independent loads of up to BATCH cells
-            ci[t] = t < cnt ? __ldg(inc + k + t) : 0;
-            const int64_t cell = ci[t] / N;
-            const int i = ci[t] - (int)(cell * N);
-            x[t] = (t < cnt && l < NE) ? __ldcs(Jc + (cell * ND + 2 * i + a) * ND + col) : 0.0;
-            sl[t] = t < cnt ? __ldg(slots + ci[t]) : 0;
+    for (int n = 0; n < NPW; ++n) {
+        const bool ok = v0 + n < nnodes;
+        const int64_t v = ok ? v0 + n : v0;
+        r0[n] = __ldg(rowptr + 2 * v);
+        len[n] = ok ? (int)(__ldg(rowptr + 2 * v + 2) - r0[n]) : 0;  // both rows: 4 deg entries
+        k0[n] = __ldg(inc_ptr + v);
+        cnt[n] = ok ? (int)(__ldg(inc_ptr + v + 1) - k0[n]) : 0;
+    }
+    // incidence: lane n LPN + t holds entry t (< BATCH) of node n
+    const int ln = l / LPN, lt = l % LPN;
+    int32_t my = 0;
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+        if (ln == n && lt < cnt[n] && lt < BATCH) my = __ldg(inc + k0[n] + lt);
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+        for (int p = l; p < len[n]; p += 32) buf[w][n][p] = 0.0;
+    const int a = l / ND, col = l % ND, j = col >> 1, bb = col & 1;
+    double x[NPW][BATCH];
+    int sl[NPW][BATCH];  // this lane's slot byte (column node j) of each incident cell
+    const uint8_t *sb = reinterpret_cast<const uint8_t *>(slots);
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+#pragma unroll
+        for (int t = 0; t < BATCH; ++t) {
+            const int32_t ci = __shfl_sync(0xffffffffu, my, n * LPN + t);
+            const bool live = t < cnt[n];
+            const int64_t cell = ci / N;
+            const int i = ci - (int)(cell * N);
+            x[n][t] = (live && l < NE) ? __ldcs(Jc + (cell * ND + 2 * i + a) * ND + col) : 0.0;
+            sl[n][t] = live ? (int)__ldg(sb + 8 * (int64_t)ci + j) : 0;
         }
+    __syncwarp();
+#pragma unroll
+    for (int n = 0; n < NPW; ++n) {
+        const int half = len[n] >> 1;
 #pragma unroll
         for (int t = 0; t < BATCH; ++t)
-            if (t < cnt && l < NE) b[a * half + 2 * (int)((sl[t] >> (8 * j)) & 0xff) + bb] += x[t];
+            if (t < cnt[n] && l < NE) buf[w][n][a * half + 2 * sl[n][t] + bb] += x[n][t];
+        // rare: more than BATCH incident cells (not on extruded hex8 / wedge6 meshes)
+        for (int64_t k = k0[n] + BATCH; k < k0[n] + cnt[n]; ++k) {
+            const int32_t ci = __ldg(inc + k);
+            const int64_t cell = ci / N;
+            const int i = ci - (int)(cell * N);
+            if (l < NE) {
+                const uint64_t s = __ldg(slots + ci);
+                buf[w][n][a * half + 2 * (int)((s >> (8 * j)) & 0xff) + bb] += __ldcs(Jc + (cell * ND + 2 * i + a) * ND + col);
+            }
+        }
     }
     __syncwarp();
-    for (int p = l; p < len; p += 32) vals[r0 + p] += b[p];
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+        for (int p = l; p < len[n]; p += 32) vals[r0[n] + p] += buf[w][n][p];
 }
 
 // ---------------------------------------------------------------------------

@@ -310,7 +310,8 @@ class StokesFO:
         _check(_lib().stokesfo_csr_slots_size(self._h, ctypes.byref(n)), "csr_slots_size")
         self.slots = torch.empty(max(int(n.value) // 8, 2), dtype=torch.int64, device=self.device)
         _check(_lib().stokesfo_csr_slots(self._h, _ptr(self.slots)), "csr_slots")
-        return self.slots[:int(n.value) // 8]
+        C, N = self.num_cells, self.N
+        return self.slots[:C * N]
 
     def jacobian_csr(self, U, csr_vals, R=None):
         """csr_vals += assembled Jacobian (fused, no element matrices); optionally R += residual."""
