@@ -1247,9 +1247,11 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
     csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
                       const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
                       const uint64_t *__restrict__ slots, double *__restrict__ vals) {
-    constexpr int ND = 2 * N, NE = 2 * ND;  // entries of one node's two rows in one cell
-    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW;
-    __shared__ double buf[CSR_GATHER_WARPS][NPW][4 * CSR_GATHER_MAXDEG];
+    constexpr int ND = 2 * N;
+    constexpr int LC = 2 * N;            // lanes per cell: each loads one (j, b = 0..1) pair of one row
+    constexpr int CPI = 32 / LC;         // cells per load instruction (2 for hex8 and wedge6)
+    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW, NI = BATCH / CPI;
+    __shared__ __align__(16) double buf[CSR_GATHER_WARPS][NPW][4 * CSR_GATHER_MAXDEG];
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
     const int64_t v0 = (blockIdx.x * (int64_t)CSR_GATHER_WARPS + w) * NPW;
     if (v0 >= nnodes) return;  // uniform per warp
@@ -1264,6 +1266,11 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
         k0[n] = __ldg(inc_ptr + v);
         cnt[n] = ok ? (int)(__ldg(inc_ptr + v + 1) - k0[n]) : 0;
     }
+    // pull the rows' vals lines into L2 now: the final read-modify-write then hits L2
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+        for (int p = 16 * l; p < len[n]; p += 16 * 32)
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(vals + r0[n] + p));
     // incidence: lane n LPN + t holds entry t (< BATCH) of node n
     const int ln = l / LPN, lt = l % LPN;
     int32_t my = 0;
@@ -1272,44 +1279,69 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
         if (ln == n && lt < cnt[n] && lt < BATCH) my = __ldg(inc + k0[n] + lt);
 #pragma unroll
     for (int n = 0; n < NPW; ++n)
-        for (int p = l; p < len[n]; p += 32) buf[w][n][p] = 0.0;
-    const int a = l / ND, col = l % ND, j = col >> 1, bb = col & 1;
-    double x[NPW][BATCH];
-    int sl[NPW][BATCH];  // this lane's slot byte (column node j) of each incident cell
+        for (int p = 2 * l; p < len[n]; p += 64) *reinterpret_cast<double2 *>(&buf[w][n][p]) = make_double2(0.0, 0.0);
+    // lane l <-> (cell u = l / LC of the pair, row a, column node j); columns (j, 0..1) as one double2
+    const int u = l / LC, a = (l % LC) / N, j = l % N;
+    const bool lane_ok = l < CPI * LC;
+    double2 x[NPW][NI];
+    int sl[NPW][NI];  // this lane's slot byte (column node j) of its incident cell
     const uint8_t *sb = reinterpret_cast<const uint8_t *>(slots);
 #pragma unroll
     for (int n = 0; n < NPW; ++n)
 #pragma unroll
-        for (int t = 0; t < BATCH; ++t) {
-            const int32_t ci = __shfl_sync(0xffffffffu, my, n * LPN + t);
-            const bool live = t < cnt[n];
+        for (int t = 0; t < NI; ++t) {
+            const int e = CPI * t + (u < CPI ? u : 0);  // incidence entry of this lane
+            const int32_t ci = __shfl_sync(0xffffffffu, my, n * LPN + e);
+            const bool live = lane_ok && e < cnt[n];
             const int64_t cell = ci / N;
             const int i = ci - (int)(cell * N);
-            x[n][t] = (live && l < NE) ? __ldcs(Jc + (cell * ND + 2 * i + a) * ND + col) : 0.0;
-            sl[n][t] = live ? (int)__ldg(sb + 8 * (int64_t)ci + j) : 0;
+            x[n][t] = live ? __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j)
+                           : make_double2(0.0, 0.0);
+            sl[n][t] = live ? (int)__ldg(sb + 8 * (int64_t)ci + j) : -1;
         }
     __syncwarp();
 #pragma unroll
     for (int n = 0; n < NPW; ++n) {
         const int half = len[n] >> 1;
+        // cells u = 0 and u = 1 of a pair may hit the same entries: add them in turn
 #pragma unroll
-        for (int t = 0; t < BATCH; ++t)
-            if (t < cnt[n] && l < NE) buf[w][n][a * half + 2 * sl[n][t] + bb] += x[n][t];
+        for (int t = 0; t < NI; ++t)
+#pragma unroll
+            for (int uu = 0; uu < CPI; ++uu) {
+                if (u == uu && sl[n][t] >= 0) {
+                    double2 *p = reinterpret_cast<double2 *>(&buf[w][n][a * half + 2 * sl[n][t]]);
+                    double2 b = *p;
+                    b.x += x[n][t].x;
+                    b.y += x[n][t].y;
+                    *p = b;
+                }
+                __syncwarp();
+            }
         // rare: more than BATCH incident cells (not on extruded hex8 / wedge6 meshes)
         for (int64_t k = k0[n] + BATCH; k < k0[n] + cnt[n]; ++k) {
             const int32_t ci = __ldg(inc + k);
             const int64_t cell = ci / N;
             const int i = ci - (int)(cell * N);
-            if (l < NE) {
-                const uint64_t s = __ldg(slots + ci);
-                buf[w][n][a * half + 2 * (int)((s >> (8 * j)) & 0xff) + bb] += __ldcs(Jc + (cell * ND + 2 * i + a) * ND + col);
+            if (l < LC) {
+                const int s = (int)__ldg(sb + 8 * (int64_t)ci + j);
+                const double2 y = __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j);
+                buf[w][n][a * half + 2 * s] += y.x;
+                buf[w][n][a * half + 2 * s + 1] += y.y;
             }
+            __syncwarp();
         }
     }
     __syncwarp();
 #pragma unroll
     for (int n = 0; n < NPW; ++n)
-        for (int p = l; p < len[n]; p += 32) vals[r0[n] + p] += buf[w][n][p];
+        for (int p = 2 * l; p < len[n]; p += 64) {
+            double2 *o = reinterpret_cast<double2 *>(vals + r0[n] + p);
+            const double2 b = *reinterpret_cast<const double2 *>(&buf[w][n][p]);
+            double2 c = *o;
+            c.x += b.x;
+            c.y += b.y;
+            *o = c;
+        }
 }
 
 // ---------------------------------------------------------------------------
