@@ -305,7 +305,7 @@ __host__ __device__ constexpr bool forms_jac() {
 // (+ for M_JVP: dbeta00 dbeta01 dbeta02 dbeta11 dbeta12, gamma * tau)
 constexpr int NQS = 9;
 template <int MODE>
-constexpr int nqs() {
+__host__ __device__ constexpr int nqs() {
     return MODE == M_JVP ? 15 : 9;
 }
 
@@ -316,14 +316,26 @@ __device__ __forceinline__ int qsi(int f, int c, int q) {
     return E::qsi(f, c, q);
 }
 
+// Per-QP scalars in shared memory: fields [0, SPLIT) in the common region `lo`,
+// fields [SPLIT, nqs) in `hi` (the unused tail of the current stage buffer,
+// when it has room: one shared-memory region less per warp -> one more
+// resident warp per SM for hex8 JAC; see EvalSmem).
+template <class E, int SPLIT>
+struct QsView {
+    double *lo, *hi;
+    __device__ __forceinline__ double &operator()(int f, int c, int q) const {
+        return f < SPLIT ? lo[E::qsi(f, c, q)] : hi[E::qsi(f - SPLIT, c, q)];
+    }
+};
+
 // ---- shared device pieces ---------------------------------------------------
 
 // Per-QP tail: given Ugrad and grad s_h at (cell c, qp q), evaluate the
 // effective strain rate (Z2), Glen viscosity at n = 3 (Z1, Z3) and the per-QP
 // scalars the per-node phase needs.  beta = B g so that sigma = 2 mu beta gives
 // strs00..strs12 of Fig. 2.
-template <class E, int MODE = M_RESID>
-__device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, int q, int nvalid, int64_t cell0,
+template <class E, int MODE = M_RESID, class QS>
+__device__ __forceinline__ void qp_tail(const EvalArgs &a, const QS &qs, int c, int q, int nvalid, int64_t cell0,
                                         bool have_s, double kc, double wm, double ux, double uy, double uz, double vx,
                                         double vy, double vz, double gs0, double gs1, const double *dg = nullptr) {
     constexpr int Q = E::Q;
@@ -333,14 +345,14 @@ __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, in
     const double r = rcbrt(e2 + a.delta);  // (e2 + delta)^(-1/3)
     const double mu = kc * r;
     const double wmu2 = 2.0 * wm * mu;
-    qs[qsi<E>(0, c, q)] = 2.0 * ux + vy;   // beta_(0,0) = strs00 / (2 mu)
-    qs[qsi<E>(1, c, q)] = 0.5 * uyvx;      // beta_(0,1) = beta_(1,0) = strs01 / (2 mu)
-    qs[qsi<E>(2, c, q)] = 0.5 * uz;        // beta_(0,2) = strs02 / (2 mu)
-    qs[qsi<E>(3, c, q)] = ux + 2.0 * vy;   // beta_(1,1) = strs11 / (2 mu)
-    qs[qsi<E>(4, c, q)] = 0.5 * vz;        // beta_(1,2) = strs12 / (2 mu)
-    qs[qsi<E>(5, c, q)] = wmu2;
+    qs(0, c, q) = 2.0 * ux + vy;   // beta_(0,0) = strs00 / (2 mu)
+    qs(1, c, q) = 0.5 * uyvx;      // beta_(0,1) = beta_(1,0) = strs01 / (2 mu)
+    qs(2, c, q) = 0.5 * uz;        // beta_(0,2) = strs02 / (2 mu)
+    qs(3, c, q) = ux + 2.0 * vy;   // beta_(1,1) = strs11 / (2 mu)
+    qs(4, c, q) = 0.5 * vz;        // beta_(1,2) = strs12 / (2 mu)
+    qs(5, c, q) = wmu2;
     // gamma = wM 2 mu p / (e2 + delta) = wmu2 p r^3  (d mu / d e2, reading Z5)
-    qs[qsi<E>(6, c, q)] = wmu2 * P_EXP * (r * r * r);
+    qs(6, c, q) = wmu2 * P_EXP * (r * r * r);
     double wf0 = 0.0, wf1 = 0.0;
     if (a.force_qp) {
         if (c < nvalid) {
@@ -352,20 +364,20 @@ __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, in
         wf0 = wm * a.rho_g * gs0;
         wf1 = wm * a.rho_g * gs1;
     }
-    qs[qsi<E>(7, c, q)] = wf0;
-    qs[qsi<E>(8, c, q)] = wf1;
+    qs(7, c, q) = wf0;
+    qs(8, c, q) = wf1;
     if (MODE == M_JVP) {
         // directional derivative along X: dg = grad of X at the QP; d beta = B dg;
         // tau = (B g) . dg = d(eps_e^2); d sigma = 2 mu (d beta + p tau beta / (e2 + delta))
         const double dux = dg[0], duy = dg[1], duz = dg[2], dvx = dg[3], dvy = dg[4], dvz = dg[5];
         const double b00 = 2.0 * ux + vy, b01 = 0.5 * uyvx, b02 = 0.5 * uz, b11 = ux + 2.0 * vy, b12 = 0.5 * vz;
         const double tau = b00 * dux + b01 * (duy + dvx) + b02 * duz + b11 * dvy + b12 * dvz;
-        qs[qsi<E>(9, c, q)] = 2.0 * dux + dvy;
-        qs[qsi<E>(10, c, q)] = 0.5 * (duy + dvx);
-        qs[qsi<E>(11, c, q)] = 0.5 * duz;
-        qs[qsi<E>(12, c, q)] = dux + 2.0 * dvy;
-        qs[qsi<E>(13, c, q)] = 0.5 * dvz;
-        qs[qsi<E>(14, c, q)] = wmu2 * P_EXP * (r * r * r) * tau;
+        qs(9, c, q) = 2.0 * dux + dvy;
+        qs(10, c, q) = 0.5 * (duy + dvx);
+        qs(11, c, q) = 0.5 * duz;
+        qs(12, c, q) = dux + 2.0 * dvy;
+        qs(13, c, q) = 0.5 * dvz;
+        qs(14, c, q) = wmu2 * P_EXP * (r * r * r) * tau;
     }
     if (a.mu_qp && c < nvalid) a.mu_qp[(cell0 + c) * Q + q] = mu;
 }
@@ -378,8 +390,8 @@ __device__ __forceinline__ void qp_tail(const EvalArgs &a, double *qs, int c, in
 // M_ab = wM 2 mu (B-block (a,b) applied to G_i) + gamma h_(i,a) beta_(b,.)
 // is the exact forward derivative of the chain (seed-sparse Sacado lanes).
 // pf() is called once at q = Q/2 (prefetch hook).
-template <class E, int MODE, class PF>
-__device__ __forceinline__ void node_accumulate(const double *rg, const double *qs, int c2, int i, const double *bfi,
+template <class E, int MODE, class PF, class QS>
+__device__ __forceinline__ void node_accumulate(const double *rg, const QS &qs, int c2, int i, const double *bfi,
                                                 double &R0, double &R1, double (&Jb)[E::N / 2 + 1][2][2], double &dR0,
                                                 double &dR1, PF pf) {
     constexpr int N = E::N, Q = E::Q, K = N / 2;
@@ -395,11 +407,11 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
         if (q == Q / 2) pf();
-        const double b00 = qs[qsi<E>(0, c2, q)], b01 = qs[qsi<E>(1, c2, q)], b02 = qs[qsi<E>(2, c2, q)];
-        const double b11 = qs[qsi<E>(3, c2, q)], b12 = qs[qsi<E>(4, c2, q)];
+        const double b00 = qs(0, c2, q), b01 = qs(1, c2, q), b02 = qs(2, c2, q);
+        const double b11 = qs(3, c2, q), b12 = qs(4, c2, q);
         const double b10 = b01;
-        const double wmu2 = qs[qsi<E>(5, c2, q)];
-        const double wf0 = qs[qsi<E>(7, c2, q)], wf1 = qs[qsi<E>(8, c2, q)];
+        const double wmu2 = qs(5, c2, q);
+        const double wf0 = qs(7, c2, q), wf1 = qs(8, c2, q);
         const double gi0 = rg[gidx<E>(i, q, 0, c2)];
         const double gi1 = rg[gidx<E>(i, q, 1, c2)];
         const double gi2 = rg[gidx<E>(i, q, 2, c2)];
@@ -410,16 +422,16 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const double *
         R1 = fma(wf1, bfi[q], fma(wmu2, h1, R1));
         if (MODE == M_JVP) {
             // dR_(i,a) += wmu2 G_i . dbeta_a + gamma tau h_(i,a)
-            const double d00 = qs[qsi<E>(9, c2, q)], d01 = qs[qsi<E>(10, c2, q)], d02 = qs[qsi<E>(11, c2, q)];
-            const double d11 = qs[qsi<E>(12, c2, q)], d12 = qs[qsi<E>(13, c2, q)];
-            const double gt = qs[qsi<E>(14, c2, q)];
+            const double d00 = qs(9, c2, q), d01 = qs(10, c2, q), d02 = qs(11, c2, q);
+            const double d11 = qs(12, c2, q), d12 = qs(13, c2, q);
+            const double gt = qs(14, c2, q);
             const double e0 = fma(gi2, d02, fma(gi1, d01, gi0 * d00));
             const double e1 = fma(gi2, d12, fma(gi1, d11, gi0 * d01));
             dR0 = fma(gt, h0, fma(wmu2, e0, dR0));
             dR1 = fma(gt, h1, fma(wmu2, e1, dR1));
         }
         if (JAC) {
-            const double gam = qs[qsi<E>(6, c2, q)];
+            const double gam = qs(6, c2, q);
             const double gh0 = gam * h0, gh1 = gam * h1;
             const double w0 = wmu2 * gi0, w1 = wmu2 * gi1, w2 = wmu2 * gi2;
             const double m00x = fma(2.0, w0, gh0 * b00), m00y = fma(0.5, w1, gh0 * b01),
@@ -564,8 +576,14 @@ struct EvalSmem {
     static constexpr int IN_BYTES = X_OFF + (MODE == M_JVP ? TC * E::UPITCH * 16 : 0);
     static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
-    static constexpr int OFF_QS = NSTAGE * STAGE;            // double [nqs][TC][Q]
-    static constexpr int OFF_BAR = (int)round_up(OFF_QS + nqs<MODE>() * TC * Q * 8, 8);
+    // per-QP scalar fields that fit in the stage's tail past the inputs (free until the J staging)
+    static constexpr int TAIL_OFF = (int)round_up(IN_BYTES, 16);
+    static constexpr int FIELD = TC * Q * 8;
+    static constexpr int TAIL_FIT = (STAGE - TAIL_OFF) / FIELD;
+    static constexpr int TAIL_FIELDS = TAIL_FIT < 3 ? TAIL_FIT : 3;
+    static constexpr int SPLIT = nqs<MODE>() - TAIL_FIELDS;   // fields [0, SPLIT) in the common region
+    static constexpr int OFF_QS = NSTAGE * STAGE;            // double [SPLIT][TC][Q]
+    static constexpr int OFF_BAR = (int)round_up(OFF_QS + SPLIT * FIELD, 8);
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
     static_assert(U_OFF % 16 == 0 && X_OFF % 16 == 0 && STAGE % 128 == 0 && OFF_QS % 16 == 0, "alignment");
 };
@@ -615,7 +633,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
     using R = Rec<E>;
     using S = EvalSmem<E, MODE, NSTAGE>;
     extern __shared__ __align__(128) char smem[];
-    double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
+    double *qs_lo = reinterpret_cast<double *>(smem + S::OFF_QS);
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
     const int l = threadIdx.x;
     const bool act = l < TC * N;
@@ -654,6 +672,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
         const double2 *Us = reinterpret_cast<const double2 *>(stage + S::U_OFF);
         const double *ss = reinterpret_cast<const double *>(stage + S::S_OFF);
         const double2 *Xs = reinterpret_cast<const double2 *>(stage + S::X_OFF);
+        const QsView<E, S::SPLIT> qs{qs_lo, reinterpret_cast<double *>(stage + S::TAIL_OFF)};
         const int64_t cell0 = tile * TC;
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
 
@@ -797,7 +816,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_otf_kernel
     using S = OtfSmem<E, MODE>;
     extern __shared__ __align__(128) char smem[];
     double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
-    double *qs = reinterpret_cast<double *>(smem + S::OFF_QS);
+    const QsView<E, nqs<MODE>()> qs{reinterpret_cast<double *>(smem + S::OFF_QS), nullptr};
     double *dphi = reinterpret_cast<double *>(smem + S::OFF_DPHI);
     const int l = threadIdx.x;
     const bool act = l < TC * N;
