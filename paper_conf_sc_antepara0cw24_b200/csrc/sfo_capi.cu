@@ -87,16 +87,25 @@ int configure_otf(int *grid) {
     return STOKESFO_OK;
 }
 
+// Launch shape of eval_kernel: WPC independent warps per CTA, each with its own
+// shared-memory slice (WPC = 1: exactly S::BYTES).
+template <class E, int MODE, int NS>
+constexpr int eval_smem_bytes() {
+    using S = EvalSmem<E, MODE, NS>;
+    return warps_per_cta<E, MODE>() == 1 ? S::BYTES : warps_per_cta<E, MODE>() * S::SLICE;
+}
+
 template <class E, int MODE, int NS>
 int configure_eval(int *grid) {
-    using S = EvalSmem<E, MODE, NS>;
     auto fn = eval_kernel<E, MODE, NS>;
-    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES) != cudaSuccess)
+    constexpr int bytes = eval_smem_bytes<E, MODE, NS>();
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
         return cuda_status();
     int dev = 0, sms = 0, per_sm = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, S::BYTES) != cudaSuccess)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32 * warps_per_cta<E, MODE>(), bytes) !=
+        cudaSuccess)
         return cuda_status();
     *grid = std::max(1, sms * std::max(1, per_sm));
     return STOKESFO_OK;
@@ -191,14 +200,16 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     const int g = MODE == M_JAC ? c->grid_jac
                 : MODE == M_JVP ? c->grid_jvp
                 : MODE == M_CSR ? c->grid_csr : c->grid_resid;
-    const int grid = (int)std::min<int64_t>(g, c->ntiles);
+    const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
+    constexpr int WPC = warps_per_cta<E, MODE>();  // eval_kernel only (the on-the-fly kernel: 1)
+    const int grid = (int)std::min<int64_t>(g, otf ? c->ntiles : (c->ntiles + WPC - 1) / WPC);
     const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_RESID ? c->nstage_resid : 2);
-    if (c->mode == STOKESFO_GEOMETRY_ON_THE_FLY)
+    if (otf)
         eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
     else if (MODE != M_CSR && ns == 3)
-        eval_kernel<E, MODE, 3><<<grid, 32, EvalSmem<E, MODE, 3>::BYTES, c->stream>>>(a);
+        eval_kernel<E, MODE, 3><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 3>(), c->stream>>>(a);
     else
-        eval_kernel<E, MODE, 2><<<grid, 32, EvalSmem<E, MODE, 2>::BYTES, c->stream>>>(a);
+        eval_kernel<E, MODE, 2><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 2>(), c->stream>>>(a);
     return cuda_status();
 }
 

@@ -555,9 +555,20 @@ __device__ __forceinline__ void basis_row(int i, double (&bfi)[E::Q]) {
 
 // Resident 1-warp CTAs per SM the register budget is sized for (12 with the
 // Jacobian accumulators, 16 for the residual-only kernels: <= 128 registers).
+#ifndef SFO_WEDGE_JAC_WARPS
+#define SFO_WEDGE_JAC_WARPS 16
+#endif
 template <class E, int MODE>
-constexpr int warps_per_sm() {
-    return forms_jac<MODE>() ? 12 : 16;
+__host__ __device__ constexpr int warps_per_sm() {
+    // wedge6 JAC: 16 (128 registers, 2-warp CTAs so that 16 x 13.7 KB of shared
+    // memory fits next to the per-CTA driver reserve)
+    return forms_jac<MODE>() ? (E::N == 6 && MODE == M_JAC ? SFO_WEDGE_JAC_WARPS : 12) : 16;
+}
+// Independent persistent warps per CTA (each warp runs its own tile loop and
+// record ring in its own shared-memory slice; only __syncwarp is used).
+template <class E, int MODE>
+__host__ __device__ constexpr int warps_per_cta() {
+    return (E::N == 6 && MODE == M_JAC && SFO_WEDGE_JAC_WARPS > 12) ? 2 : 1;
 }
 
 // ---- G3/G4 with stored geometry (the §8(a2) precompute streamed per tile) ----
@@ -585,6 +596,7 @@ struct EvalSmem {
     static constexpr int OFF_QS = NSTAGE * STAGE;            // double [SPLIT][TC][Q]
     static constexpr int OFF_BAR = (int)round_up(OFF_QS + SPLIT * FIELD, 8);
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
+    static constexpr int SLICE = (int)round_up(BYTES, 128);  // per-warp slice in multi-warp CTAs
     static_assert(U_OFF % 16 == 0 && X_OFF % 16 == 0 && STAGE % 128 == 0 && OFF_QS % 16 == 0, "alignment");
 };
 
@@ -603,7 +615,7 @@ __device__ __forceinline__ Gathered gather_load(const char *stage, const double 
                                                 bool have_s, const double *X) {
     using R = Rec<E>;
     Gathered v{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
-    const int l = threadIdx.x;
+    const int l = threadIdx.x & 31;
     if (l < E::TC * E::N) {
         const int c = E::lane_cell(l), n = E::lane_sub(l);
         const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[R::conn(n, c)];
@@ -616,7 +628,7 @@ __device__ __forceinline__ Gathered gather_load(const char *stage, const double 
 template <class E, int MODE>
 __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
     using S = EvalSmem<E, MODE>;
-    const int l = threadIdx.x;
+    const int l = threadIdx.x & 31;
     if (l < E::TC * E::N) {
         const int e = E::lane_cell(l) * E::UPITCH + E::lane_sub(l);  // [cell][node]
         reinterpret_cast<double2 *>(stage + S::U_OFF)[e] = v.u;
@@ -626,16 +638,22 @@ __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
 }
 
 template <class E, int MODE, int NSTAGE>
-__global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(EvalArgs a) {
+__global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E, MODE>() / warps_per_cta<E, MODE>()))
+    eval_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
     static_assert(N == Q, "lane mappings assume N == Q");
     using R = Rec<E>;
     using S = EvalSmem<E, MODE, NSTAGE>;
-    extern __shared__ __align__(128) char smem[];
+    constexpr int WPC = warps_per_cta<E, MODE>();
+    extern __shared__ __align__(128) char smem_all[];
+    // this warp's virtual CTA: index vb of vg, its own shared-memory slice
+    char *smem = smem_all + (threadIdx.x >> 5) * S::SLICE;
+    const int64_t vb = (int64_t)blockIdx.x * WPC + (threadIdx.x >> 5);
+    const int64_t vg = (int64_t)gridDim.x * WPC;
     double *qs_lo = reinterpret_cast<double *>(smem + S::OFF_QS);
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
-    const int l = threadIdx.x;
+    const int l = threadIdx.x & 31;
     const bool act = l < TC * N;
     const int c = act ? E::lane_cell(l) : TC, s = act ? E::lane_sub(l) : 0;  // (cell, node-or-qp)
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
@@ -646,7 +664,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
         for (int k = 0; k < NSTAGE; ++k) mbar_init(&bar[k], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         for (int k = 0; k < NSTAGE; ++k) {
-            const int64_t tile = blockIdx.x + (int64_t)k * gridDim.x;
+            const int64_t tile = vb + (int64_t)k * vg;
             if (tile < a.ntiles) {
                 mbar_arrive_expect_tx(&bar[k], R::BYTES);
                 bulk_g2s(smem + k * S::STAGE, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[k], pol_stream);
@@ -654,7 +672,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
         }
     }
     __syncwarp();
-    if ((int64_t)blockIdx.x < a.ntiles) {
+    if (vb < a.ntiles) {
         mbar_wait(&bar[0], 0);
         gather_store<E, MODE>(smem, gather_load<E, MODE>(smem, a.U, a.surface, have_s, a.X));
     }
@@ -662,7 +680,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
     basis_row<E>(act ? s : 0, bfi);
 
     int it = 0;
-    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+    for (int64_t tile = vb; tile < a.ntiles; tile += vg, ++it) {
         const int st = it % NSTAGE;
         char *stage = smem + st * S::STAGE;
         const int32_t *rconn = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF);
@@ -708,7 +726,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
 
         // ---- per-node phase (+ gather of the next tile at q = Q/2) ----
         const int32_t gnode = act ? rconn[R::conn(s, c)] : 0;
-        const int64_t ntile = tile + gridDim.x;
+        const int64_t ntile = tile + vg;
         const int nst = (it + 1) % NSTAGE;
         Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
         auto prefetch = [&]() {
@@ -720,7 +738,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
             // its J bulk store was issued (its SMEM read has long completed)
             if (NSTAGE >= 3 && l == 0 && it >= 1) {
                 const int ps = (it - 1) % NSTAGE;
-                const int64_t rt = tile + (int64_t)(NSTAGE - 1) * gridDim.x;
+                const int64_t rt = tile + (int64_t)(NSTAGE - 1) * vg;
                 if (JAC) bulk_wait_read0();
                 if (rt < a.ntiles) {
                     mbar_arrive_expect_tx(&bar[ps], R::BYTES);
@@ -748,7 +766,7 @@ __global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_kernel(Eva
             }
         }
         if (l == 0 && NSTAGE < 3) {
-            const int64_t nt = tile + (int64_t)NSTAGE * gridDim.x;
+            const int64_t nt = tile + (int64_t)NSTAGE * vg;
             if (nt < a.ntiles) {
                 mbar_arrive_expect_tx(&bar[st], R::BYTES);
                 bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
@@ -809,7 +827,7 @@ __device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live,
 }
 
 template <class E, int MODE>
-__global__ void __launch_bounds__(32, (warps_per_sm<E, MODE>())) eval_otf_kernel(EvalArgs a) {
+__global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "lane mappings assume N == Q");
     constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
