@@ -317,6 +317,27 @@ def main():
         step()
     ctx.sync()
 
+    # live context for the peak: a plain device-to-device copy on this box right now
+    live_copy = None
+    if rank == 0:
+        try:
+            nb = 1 << 31
+            src = torch.empty(nb // 8, dtype=torch.float64, device=dev)
+            dst = torch.empty_like(src)
+            for _ in range(2):
+                dst.copy_(src)
+            c0 = torch.cuda.Event(enable_timing=True)
+            c1 = torch.cuda.Event(enable_timing=True)
+            c0.record(stream)
+            for _ in range(5):
+                dst.copy_(src)
+            c1.record(stream)
+            torch.cuda.synchronize(dev)
+            live_copy = 2 * nb * 5 / (c0.elapsed_time(c1) * 1e-3) / 1e9
+            del src, dst
+        except Exception:
+            live_copy = None
+
     clocks = ClockSampler(local)
     if world > 1:
         dist.barrier()
@@ -479,7 +500,10 @@ def main():
                          + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>"}[args.op]
                          + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
                             "jvp": " (stokesfo_jvp)", "jac_csr": " (stokesfo_jacobian_csr)"}[args.op],
-                         "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src},
+                         "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src,
+                         "live_copy_gbs": live_copy,
+                         "note": "live_copy_gbs: torch device-to-device copy of 2 GiB on this box before the timed "
+                                 "region (context for box-to-box variance; not the denominator)"},
             "achieved_hbm_gbs": achieved,
             "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),
             "halo": halo_mode,
