@@ -28,16 +28,9 @@ struct Hex8 {
     // lanes over (c,q)) and the per-node loads (fixed q, lanes over (c,j)) hit 16
     // distinct bank pairs per half-warp
     __host__ __device__ static constexpr int slot(int c, int n, int q) { return c * N + (n + q) % N; }
-    // gathered U/s per (cell, node) and per-QP scalars (f, cell, qp) in shared memory.
-    // Odd cell pitches (9 x 16 B for U, 9 x 8 B for s and the scalars): the
-    // per-QP phase's U/s reads and the per-node phase's scalar reads are
-    // broadcasts within a quarter-warp (one cell), and the odd pitch puts the 4
-    // cells of a warp in distinct banks (a pitch of 8 put them all in the same
-    // banks: 4 wavefronts per 128-bit read instead of 1).
-    static constexpr int UPITCH = 9;
-    static constexpr int QPITCH = Q + 1;
-    static constexpr int QS_FIELD = TC * QPITCH;  // doubles per scalar field
-    __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * TC + c) * QPITCH + q; }
+    // gathered U/s per (cell, node) and per-QP scalars (f, cell, qp) in shared memory
+    static constexpr int UPITCH = N;
+    __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * TC + c) * Q + q; }
 };
 struct Wedge6 {
     static constexpr int N = 6, Q = 6, TC = 5, ELEM = 1;  // 30 active lanes
@@ -53,7 +46,6 @@ struct Wedge6 {
     // odd 16-B cell pitch for the gathered U rows; per-QP scalars qp-major
     // (lanes (c, q) of the per-QP phase then write consecutive addresses)
     static constexpr int UPITCH = 7;
-    static constexpr int QS_FIELD = TC * Q;
     __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * Q + q) * TC + c; }
 };
 

@@ -589,7 +589,7 @@ struct EvalSmem {
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
     // per-QP scalar fields that fit in the stage's tail past the inputs (free until the J staging)
     static constexpr int TAIL_OFF = (int)round_up(IN_BYTES, 16);
-    static constexpr int FIELD = E::QS_FIELD * 8;
+    static constexpr int FIELD = TC * Q * 8;
     static constexpr int TAIL_FIT = (STAGE - TAIL_OFF) / FIELD;
     static constexpr int TAIL_FIELDS = TAIL_FIT < 3 ? TAIL_FIT : 3;
     static constexpr int SPLIT = nqs<MODE>() - TAIL_FIELDS;   // fields [0, SPLIT) in the common region
@@ -804,8 +804,8 @@ struct OtfSmem {
     static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * DPITCH * 8, 128);  // GradBF [Q][3][SLAB]
     static constexpr int OFF_QS = OFF_G + Q * 3 * SLAB * 8;                  // double [NQS][TC][Q]
     static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;   // J staging overlays G + qs
-    static_assert(J_BYTES <= OFF_QS + nqs<MODE>() * E::QS_FIELD * 8 - OFF_G, "J staging must fit over G + qs");
-    static constexpr int BYTES = OFF_QS + nqs<MODE>() * E::QS_FIELD * 8;
+    static_assert(J_BYTES <= OFF_QS + nqs<MODE>() * TC * Q * 8 - OFF_G, "J staging must fit over G + qs");
+    static constexpr int BYTES = OFF_QS + nqs<MODE>() * TC * Q * 8;
     static_assert(IN_X % 16 == 0 && IN_BYTES % 128 == 0 && OFF_G % 128 == 0 && OFF_QS % 16 == 0, "alignment");
 };
 
