@@ -161,6 +161,14 @@ int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t
 int stokesfo_lateral_pressure(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
                               double rho_i_g, double rho_w_g, double sea_level, double *R);
 
+/* Attach the lateral pressure term (same arguments as stokesfo_lateral_pressure,
+ * minus R) to the ctx so that stokesfo_newton_solve solves
+ * F = R_visc + R_basal + R_lateral = 0 (the term is U-independent: it enters F,
+ * not J).  The arrays stay caller-owned and must outlive the solve;
+ * nfaces = 0 detaches. */
+int stokesfo_set_lateral(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
+                         double rho_i_g, double rho_w_g, double sea_level);
+
 /* Assembly: R[2 conn[c][n] + a] += R_cell[c][n][a] (if R_cell and R are non-NULL)
  * and csr_vals[pos(row, col)] += J_cell[c][k][l] (if J_cell and csr_vals are
  * non-NULL; requires an earlier stokesfo_csr_pattern call with non-NULL rowptr
@@ -242,7 +250,8 @@ int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid
 
 /* ---------------- NEXT-3: damped Newton-Krylov driver ---------------------- */
 
-/* Solves F(U) = R_visc(U) + R_basal(U) = 0 (damped Newton, Jacobian at
+/* Solves F(U) = R_visc(U) + R_basal(U) [+ R_lateral, see stokesfo_set_lateral] = 0
+ * (damped Newton, Jacobian at
  * every nonlinear step): per step, J dU = -F by Jacobi-preconditioned CG on the
  * matrix-free operator stokesfo_jvp + basal face term (J is SPD once basal
  * friction removes the rigid null space; Jacobi diagonal from stokesfo_jacobian

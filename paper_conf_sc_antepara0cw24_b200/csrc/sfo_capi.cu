@@ -40,6 +40,11 @@ struct stokesfo_ctx {
     const int32_t *inc = nullptr;
     std::vector<int64_t> inc_ptr_h;    // host incidence from the last csr_pattern fill (until csr_slots)
     std::vector<int32_t> inc_h;
+    // lateral pressure term attached for the Newton driver (stokesfo_set_lateral)
+    const int32_t *lat_faces = nullptr;
+    int64_t lat_n = 0;
+    const double *lat_surface = nullptr;
+    double lat_rho_i_g = 0.0, lat_rho_w_g = 0.0, lat_sea = 0.0;
 };
 
 namespace {
@@ -422,6 +427,19 @@ int stokesfo_lateral_pressure(stokesfo_ctx *c, const int32_t *faces, int64_t nfa
     return cuda_status();
 }
 
+int stokesfo_set_lateral(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
+                         double rho_i_g, double rho_w_g, double sea_level) {
+    if (!c || nfaces < 0) return STOKESFO_EINVAL;
+    if (nfaces > 0 && (!faces || !surface || !aligned(faces, 8))) return STOKESFO_EINVAL;
+    c->lat_faces = nfaces > 0 ? faces : nullptr;
+    c->lat_n = nfaces > 0 ? nfaces : 0;
+    c->lat_surface = surface;
+    c->lat_rho_i_g = rho_i_g;
+    c->lat_rho_w_g = rho_w_g;
+    c->lat_sea = sea_level;
+    return STOKESFO_OK;
+}
+
 int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, const double *J_cell,
                               double *csr_vals) {
     if (!c) return STOKESFO_EINVAL;
@@ -715,10 +733,13 @@ int stokesfo_newton_solve(stokesfo_ctx *c, const int32_t *basal_cells, int64_t n
         if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_status();
         return STOKESFO_OK;
     };
-    auto eval_F = [&](const double *u, double *F) -> int {  // F = R_visc(u) + R_basal(u)
+    auto eval_F = [&](const double *u, double *F) -> int {  // F = R_visc(u) + R_basal(u) + R_lateral
         if (cudaMemsetAsync(F, 0, vb, st) != cudaSuccess) return cuda_status();
         int r = stokesfo_viscosity_resid(c, u, nullptr, nullptr, F);
         if (r == STOKESFO_OK && nbasal > 0) r = stokesfo_basal_friction(c, basal_cells, nbasal, beta, u, F, nullptr);
+        if (r == STOKESFO_OK && c->lat_n > 0)
+            r = stokesfo_lateral_pressure(c, c->lat_faces, c->lat_n, c->lat_surface, c->lat_rho_i_g, c->lat_rho_w_g,
+                                          c->lat_sea, F);
         return r;
     };
     auto apply_A = [&](const double *v, double *Av) -> int {  // Av = J(U) v + J_basal v

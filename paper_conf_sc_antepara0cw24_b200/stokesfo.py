@@ -56,7 +56,7 @@ EXPORTS = [
     "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp", "stokesfo_basal_friction",
     "stokesfo_set_remote", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
     "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
-    "stokesfo_mesh_lateral_faces", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
+    "stokesfo_mesh_lateral_faces", "stokesfo_set_lateral", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
 ]
 
 
@@ -93,6 +93,7 @@ def _lib():
         if hasattr(L, "stokesfo_lateral_pressure"):
             L.stokesfo_lateral_pressure.argtypes = [P, P, I64, P, D, D, D, P]
             L.stokesfo_mesh_lateral_faces.argtypes = [I32, I64, P, I32, ctypes.POINTER(I64), P]
+            L.stokesfo_set_lateral.argtypes = [P, P, I64, P, D, D, D]
         if hasattr(L, "stokesfo_jacobian_csr"):
             L.stokesfo_csr_slots_size.argtypes = [P, ctypes.POINTER(ctypes.c_size_t)]
             L.stokesfo_csr_slots.argtypes = [P, P]
@@ -267,6 +268,19 @@ class StokesFO:
         _check(_lib().stokesfo_lateral_pressure(self._h, _ptr(faces), int(faces.shape[0]), _ptr(surface),
                                                 float(rho_i_g), float(rho_w_g), float(sea_level), _ptr(R)),
                "lateral_pressure")
+
+    def set_lateral(self, faces, surface, rho_i_g=8.927, rho_w_g=10.05, sea_level=0.0):
+        """Attach the lateral pressure term to newton_solve's F (faces=None detaches)."""
+        import torch
+        if faces is None:
+            self._lateral_keep = None
+            _check(_lib().stokesfo_set_lateral(self._h, None, 0, None, 0.0, 0.0, 0.0), "set_lateral")
+            return
+        _dev(faces, torch.int32, None, "faces")
+        _dev(surface, torch.float64, (self.num_nodes,), "surface")
+        self._lateral_keep = (faces, surface)
+        _check(_lib().stokesfo_set_lateral(self._h, _ptr(faces), int(faces.shape[0]), _ptr(surface), float(rho_i_g),
+                                           float(rho_w_g), float(sea_level)), "set_lateral")
 
     def newton_solve(self, basal_cells, beta, U, max_newton=8, max_cg=500, max_ls=20, rtol_newton=1e-10,
                      atol_newton=0.0, rtol_cg=1e-6, ls_c=1e-4):

@@ -7,12 +7,13 @@ import pytest
 
 import oracle as O
 from oracle import basal as B
+from oracle import lateral as LT
 from tests import _meshes as M
 
 pytestmark = pytest.mark.gpu
 
 
-def _oracle_newton(elem, conn, coords, G, wm, s, kc, cells, beta, U0, iters=12):
+def _oracle_newton(elem, conn, coords, G, wm, s, kc, cells, beta, U0, iters=12, lateral=None):
     e = O.ELEM[elem]
     N = conn.shape[1]
     nb = N // 2
@@ -23,7 +24,10 @@ def _oracle_newton(elem, conn, coords, G, wm, s, kc, cells, beta, U0, iters=12):
     def F_J(U, need_J=True):
         out = O.evaluate(e, conn, G, wm, U, surface=s, kc=kc, mode="jac" if need_J else "resid")
         Rb, Jb, _ = B.basal_friction(nb, conn, coords, cells, beta, U)
-        F = (O.scatter(e, conn, out["R_cell"], nn) + Rb).reshape(-1)
+        F = O.scatter(e, conn, out["R_cell"], nn) + Rb
+        if lateral is not None:   # (faces, rho_i_g, rho_w_g, sea level): U-independent, F only
+            F = F + LT.lateral_pressure(N, conn, coords, lateral[0], s, *lateral[1:])[0]
+        F = F.reshape(-1)
         if not need_J:
             return F, None
         J = np.zeros((2 * nn, 2 * nn))
@@ -48,8 +52,9 @@ def _oracle_newton(elem, conn, coords, G, wm, s, kc, cells, beta, U0, iters=12):
     return U, np.linalg.norm(F_J(U, need_J=False)[0])
 
 
+@pytest.mark.parametrize("lateral", [False, True])
 @pytest.mark.parametrize("elem", ["hex8", "wedge6"])
-def test_newton_krylov_matches_oracle_newton(elem):
+def test_newton_krylov_matches_oracle_newton(elem, lateral):
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
@@ -62,9 +67,15 @@ def test_newton_krylov_matches_oracle_newton(elem):
     G, wm, _ = O.geometry(e, conn, coords)
     cells = np.arange(0, conn.shape[0], L, dtype=np.int32)
     beta = np.full(coords.shape[0], 5.0)
-    Uo, nFo = _oracle_newton(elem, conn, coords, G, wm, s, kc, cells, beta, U0)
+    lat = None
+    if lateral:   # NEXT-4 lateral (ocean) pressure on every footprint-boundary face (reading Z19)
+        z = coords[:, 2]
+        lat = (LT.lateral_faces(fp.polys, L), 8.927, 10.05, 0.5 * (z.min() + z.max()))
+    Uo, nFo = _oracle_newton(elem, conn, coords, G, wm, s, kc, cells, beta, U0, lateral=lat)
     ctx = StokesFO(elem, torch.from_numpy(conn).cuda(), torch.from_numpy(coords).cuda(),
                    surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda())
+    if lat is not None:
+        ctx.set_lateral(torch.from_numpy(lat[0]).cuda(), torch.from_numpy(s).cuda(), *lat[1:])
     Ud = torch.from_numpy(U0).cuda()
     h = ctx.newton_solve(torch.from_numpy(cells).cuda(), torch.from_numpy(beta).cuda(), Ud, max_newton=12,
                          max_cg=2000, rtol_newton=1e-11, rtol_cg=1e-10)
