@@ -328,6 +328,27 @@ struct QsView {
     }
 };
 
+// Per-QP scalars kept in registers (the residual-only and J.v modes of the
+// stored-geometry kernel, which exchange per-node partial sums instead).
+struct RegQs {
+    double *v;
+    __device__ __forceinline__ double &operator()(int f, int, int) const { return v[f]; }
+};
+
+// Partial-sum exchange of the residual / J.v modes: lane (c, q) writes, for
+// every node n of its cell, P[c][n][q] = (G_n(q) . sigma_a(q) + wf_a(q) phi_n(q))_a
+// (double2, a = 0, 1); lane (c, i) then sums P[c][i][(k + i) mod Q] over k.
+// Row pitch 8 double2, cell pitch chosen with the bank model (writes and
+// rotated reads conflict-free for hex8; 24 / 28 wavefronts for wedge6).
+template <class E>
+__host__ __device__ constexpr int psum_idx(int c, int n, int q) {
+    return c * (E::N == 8 ? 64 : 53) + n * 8 + q;
+}
+template <class E>
+constexpr int psum_bytes() {
+    return (E::N == 8 ? E::TC * 64 : (E::TC - 1) * 53 + E::N * 8) * 16;
+}
+
 // ---- shared device pieces ---------------------------------------------------
 
 // Per-QP tail: given Ugrad and grad s_h at (cell c, qp q), evaluate the
@@ -592,11 +613,14 @@ struct EvalSmem {
     static constexpr int FIELD = TC * Q * 8;
     static constexpr int TAIL_FIT = (STAGE - TAIL_OFF) / FIELD;
     static constexpr int TAIL_FIELDS = TAIL_FIT < 3 ? TAIL_FIT : 3;
-    static constexpr int SPLIT = nqs<MODE>() - TAIL_FIELDS;   // fields [0, SPLIT) in the common region
+    // residual-only and J.v modes keep the per-QP scalars in registers (partial-sum exchange)
+    static constexpr bool PSUM = MODE == M_RESID || MODE == M_JVP;
+    static constexpr int SPLIT = PSUM ? 0 : nqs<MODE>() - TAIL_FIELDS;   // fields [0, SPLIT) in the common region
     static constexpr int OFF_QS = NSTAGE * STAGE;            // double [SPLIT][TC][Q]
     static constexpr int OFF_BAR = (int)round_up(OFF_QS + SPLIT * FIELD, 8);
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
     static constexpr int SLICE = (int)round_up(BYTES, 128);  // per-warp slice in multi-warp CTAs
+    static_assert(!PSUM || Rec<E>::G_OFF + psum_bytes<E>() <= Rec<E>::BYTES, "partial sums overlay GradBF");
     static_assert(U_OFF % 16 == 0 && X_OFF % 16 == 0 && STAGE % 128 == 0 && OFF_QS % 16 == 0, "alignment");
 };
 
@@ -678,6 +702,13 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
     }
     double bfi[Q];
     basis_row<E>(act ? s : 0, bfi);
+    double bq[N];  // phi_n at this lane's QP, every n (partial-sum modes)
+    {
+        double x, y, z, w, dx, dy, dz;
+        qp_coords<E>(act ? s : 0, x, y, z, w);
+#pragma unroll
+        for (int n = 0; n < N; ++n) basis<E>(n, x, y, z, bq[n], dx, dy, dz);
+    }
 
     int it = 0;
     for (int64_t tile = vb; tile < a.ntiles; tile += vg, ++it) {
@@ -697,6 +728,8 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
         __syncwarp();  // this tile's gathered U, s (stored by every lane) are visible
 
         // ---- per-QP phase: lane <-> (cell c, qp s) ----
+        double gq[S::PSUM ? N : 1][3];  // G_n(q) kept for the partial sums (PSUM modes)
+        double qv[S::PSUM ? 15 : 1];
         if (act) {
             const int q = s;
             double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
@@ -706,6 +739,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
                 const double g0 = rg[gidx<E>(n, q, 0, c)];
                 const double g1 = rg[gidx<E>(n, q, 1, c)];
                 const double g2 = rg[gidx<E>(n, q, 2, c)];
+                if constexpr (S::PSUM) {
+                    gq[n][0] = g0;
+                    gq[n][1] = g1;
+                    gq[n][2] = g2;
+                }
                 const double2 uv = Us[c * E::UPITCH + n];
                 ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
                 vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
@@ -719,8 +757,12 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
                     dg[3] = fma(xv.y, g0, dg[3]); dg[4] = fma(xv.y, g1, dg[4]); dg[5] = fma(xv.y, g2, dg[5]);
                 }
             }
-            qp_tail<E, MODE>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy, vz,
-                             gs0, gs1, dg);
+            if constexpr (S::PSUM)
+                qp_tail<E, MODE>(a, RegQs{qv}, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx,
+                                 vy, vz, gs0, gs1, dg);
+            else
+                qp_tail<E, MODE>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy,
+                                 vz, gs0, gs1, dg);
         }
         __syncwarp();
 
@@ -751,8 +793,58 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
         uint64_t srow = 0;
         longlong2 rp = make_longlong2(0, 0);
         if (CSR) csr_row_load(a, cell0 + c, gnode, act && c < nvalid, srow, rp, N, s);
-        if (act) node_accumulate<E, MODE>(rg, qs, c, s, bfi, R0, R1, Jb, dR0, dR1, prefetch);
-        else prefetch();
+        if constexpr (S::PSUM) {
+            // partial sums over the GradBF region of this stage (its reads are done: __syncwarp above)
+            double2 *P = reinterpret_cast<double2 *>(stage + R::G_OFF);
+            if (act) {
+                const double w = qv[5];
+                const double s00 = w * qv[0], s01 = w * qv[1], s02 = w * qv[2], s11 = w * qv[3], s12 = w * qv[4];
+#pragma unroll
+                for (int n = 0; n < N; ++n) {
+                    const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
+                    P[psum_idx<E>(c, n, s)] = make_double2(fma(qv[7], bq[n], fma(g2, s02, fma(g1, s01, g0 * s00))),
+                                                           fma(qv[8], bq[n], fma(g2, s12, fma(g1, s11, g0 * s01))));
+                }
+            }
+            __syncwarp();
+            prefetch();
+            if (act) {
+#pragma unroll
+                for (int k = 0; k < Q; ++k) {
+                    const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
+                    R0 += v.x;
+                    R1 += v.y;
+                }
+            }
+            if (JVP) {
+                __syncwarp();
+                if (act) {
+                    // d sigma_a = wmu2 d beta_a + gamma tau beta_a
+                    const double w = qv[5], gt = qv[14];
+                    const double d00 = fma(w, qv[9], gt * qv[0]), d01 = fma(w, qv[10], gt * qv[1]);
+                    const double d02 = fma(w, qv[11], gt * qv[2]), d11 = fma(w, qv[12], gt * qv[3]);
+                    const double d12 = fma(w, qv[13], gt * qv[4]);
+#pragma unroll
+                    for (int n = 0; n < N; ++n) {
+                        const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
+                        P[psum_idx<E>(c, n, s)] = make_double2(fma(g2, d02, fma(g1, d01, g0 * d00)),
+                                                               fma(g2, d12, fma(g1, d11, g0 * d01)));
+                    }
+                }
+                __syncwarp();
+                if (act) {
+#pragma unroll
+                    for (int k = 0; k < Q; ++k) {
+                        const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
+                        dR0 += v.x;
+                        dR1 += v.y;
+                    }
+                }
+            }
+        } else {
+            if (act) node_accumulate<E, MODE>(rg, qs, c, s, bfi, R0, R1, Jb, dR0, dR1, prefetch);
+            else prefetch();
+        }
         __syncwarp();  // every lane is done with this stage's record and qs
 
         if (CSR) csr_scatter<E>(a.csr_vals, c, s, act && c < nvalid, srow, rp, Jb);
