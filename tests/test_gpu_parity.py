@@ -133,7 +133,9 @@ def test_jacobian_residual_equals_viscosity_resid(torch, geometry):
     ctx.jacobian(U, J, R_cell=R1)
     ctx.viscosity_resid(U, R_cell=R2)
     ctx.sync()
-    assert torch.equal(R1, R2)
+    # same residual up to reassociation (reading Z12): the stored-geometry residual-only
+    # kernel sums per-QP partial contributions G_n . (wmu2 beta) in a rotated order
+    assert _cell_rel(R1.cpu().numpy(), R2.cpu().numpy()) <= 1e-13
 
 
 @pytest.mark.parametrize("geometry", GEOMS)
