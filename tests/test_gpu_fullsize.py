@@ -54,3 +54,102 @@ def test_fullsize_sampled_parity(cfg, geometry):
     np.add.at(Aref, conn[rows].reshape(-1), np.abs(Rc).reshape(-1, 2))
     Rg = R[torch.from_numpy(nodes).cuda()].cpu().numpy()
     assert (np.abs(Rg - Rref[nodes]) <= TOL * Aref[nodes] + 1e-300).all()
+
+
+def _sample_nodes_expect(e, conn, coords, U, s, kc, nodes, need_j):
+    """Oracle residual (and element Jacobians) of every cell incident to the sampled nodes."""
+    hit = np.isin(conn, nodes)
+    rows = np.nonzero(hit.any(1))[0]
+    G, wm, _ = O.geometry(e, conn[rows], coords)
+    out = O.evaluate(e, conn[rows], G, wm, U, surface=s, kc=kc[rows], mode="jac" if need_j else "resid")
+    return rows, out
+
+
+@pytest.mark.parametrize("cfg", ["C4", "C5"])
+def test_fullsize_residual_only_sampled(cfg):
+    """stokesfo_viscosity_resid (partial-sum kernel) at full size, sampled assembled nodes."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO
+    fp, L, elem = synth.make_config(cfg)
+    conn, coords = O.extrude(fp.xy, fp.polys, fp.b, fp.H, L)
+    U = synth.velocity_balance(fp, L, seed=12)
+    s = synth.surface_nodal(fp, L)
+    kc = synth.flow_factor(fp, L)
+    ctx = StokesFO(elem, torch.from_numpy(conn).cuda(), torch.from_numpy(coords).cuda(),
+                   surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda())
+    R = torch.zeros((coords.shape[0], 2), dtype=torch.float64, device="cuda")
+    ctx.viscosity_resid(torch.from_numpy(U).cuda(), R=R)
+    ctx.sync()
+    rng = np.random.default_rng(7)
+    nodes = np.unique(np.concatenate([rng.integers(0, coords.shape[0], 300), [coords.shape[0] - 1]]))
+    e = O.ELEM[elem]
+    rows, out = _sample_nodes_expect(e, conn, coords, U, s, kc, nodes, False)
+    Rref = np.zeros((coords.shape[0], 2))
+    Aref = np.zeros((coords.shape[0], 2))
+    np.add.at(Rref, conn[rows].reshape(-1), out["R_cell"].reshape(-1, 2))
+    np.add.at(Aref, conn[rows].reshape(-1), np.abs(out["R_cell"]).reshape(-1, 2))
+    Rg = R[torch.from_numpy(nodes).cuda()].cpu().numpy()
+    assert (np.abs(Rg - Rref[nodes]) <= TOL * Aref[nodes] + 1e-300).all()
+
+
+@pytest.mark.parametrize("cfg", ["C3", "C5"])
+def test_fullsize_csr_assembly_sampled_rows(cfg):
+    """NEXT-2 at full size: CSR pattern rows (bit-exact vs the incident cells' node sets),
+    pull assembly of stokesfo_jacobian's element matrices and the fused jacobian_csr,
+    on sampled rows recomputed by the oracle."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO
+    fp, L, elem = synth.make_config(cfg)
+    conn, coords = O.extrude(fp.xy, fp.polys, fp.b, fp.H, L)
+    U = synth.velocity_balance(fp, L, seed=11 if cfg == "C3" else 12)
+    s = synth.surface_nodal(fp, L)
+    kc = synth.flow_factor(fp, L)
+    C, N = conn.shape
+    ctx = StokesFO(elem, torch.from_numpy(conn).cuda(), torch.from_numpy(coords).cuda(),
+                   surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda())
+    rowptr, colidx = ctx.csr_pattern()
+    ctx.csr_slots()
+    Ud = torch.from_numpy(U).cuda()
+    rng = np.random.default_rng(11)
+    nodes = np.unique(np.concatenate([rng.integers(0, coords.shape[0], 120), [0, coords.shape[0] - 1]]))
+    e = O.ELEM[elem]
+    rows, out = _sample_nodes_expect(e, conn, coords, U, s, kc, nodes, True)
+    rp = rowptr.cpu().numpy()
+    want = {}
+    for v in nodes:
+        nb = np.unique(conn[np.nonzero((conn == v).any(1))[0]])
+        cols = np.stack([2 * nb, 2 * nb + 1], 1).reshape(-1)
+        for a in range(2):
+            got = colidx[int(rp[2 * v + a]):int(rp[2 * v + a + 1])].cpu().numpy()
+            assert np.array_equal(got, cols)
+            want[(v, a)] = (cols, np.zeros(cols.size), np.zeros(cols.size))
+    for r, c in enumerate(rows):
+        for i in range(N):
+            v = conn[c, i]
+            for a in range(2):
+                if (v, a) not in want:
+                    continue
+                cols, val, absv = want[(v, a)]
+                pos = np.searchsorted(cols, (2 * conn[c][:, None] + np.arange(2)).reshape(-1))
+                np.add.at(val, pos, out["J_cell"][r, 2 * i + a])
+                np.add.at(absv, pos, np.abs(out["J_cell"][r, 2 * i + a]))
+    nnz = colidx.numel()
+    for fused in (False, True):
+        vals = torch.zeros(nnz, dtype=torch.float64, device="cuda")
+        if fused:
+            ctx.jacobian_csr(Ud, vals)
+        else:
+            J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
+            ctx.jacobian(Ud, J)
+            ctx.scatter_assemble(J_cell=J, csr_vals=vals)
+            del J
+        ctx.sync()
+        for (v, a), (cols, val, absv) in want.items():
+            got = vals[int(rp[2 * v + a]):int(rp[2 * v + a + 1])].cpu().numpy()
+            assert (np.abs(got - val) <= TOL * absv + 1e-300).all(), (fused, v, a)
+        del vals
+        torch.cuda.empty_cache()
