@@ -1,17 +1,22 @@
-"""Small runs of every eval kernel variant for compute-sanitizer (memcheck /
-racecheck / synccheck / initcheck): hex8 + wedge6, stored + on-the-fly,
-residual + Jacobian, ragged tiles, plus the NEXT-1 chain and assembly kernels."""
+"""Runs of every kernel variant for compute-sanitizer (memcheck / racecheck /
+synccheck / initcheck): hex8 + wedge6, stored + on-the-fly geometry, residual
+(partial-sum exchange), Jacobian, J.v, fused CSR, slot table + pull assembly,
+ragged tiles, side sets, the NEXT-1 chain and a short Newton solve.  A second,
+larger mesh (more tiles than resident warps) exercises the persistent tile
+loop: record ring refills, next-tile gathers and the partial-sum overlay of a
+stage that is refilled right after."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
-import oracle as O
+from oracle import lateral as LT
 from tests import _meshes as M
 from paper_conf_sc_antepara0cw24_b200 import StokesFO
 
-for elem in ("hex8", "wedge6"):
-    fp, conn, coords = M.tiny(elem, n=5, L=3)
-    conn = conn[:conn.shape[0] - 3]
-    U, s, kc = M.fields(fp, 3)
+
+def run(elem, n, L, drop, full):
+    fp, conn, coords = M.tiny(elem, n=n, L=L)
+    conn = conn[:conn.shape[0] - drop]
+    U, s, kc = M.fields(fp, L)
     kc = kc[:conn.shape[0]]
     C, N = conn.shape
     for geo in ("stored", "on_the_fly"):
@@ -21,21 +26,44 @@ for elem in ("hex8", "wedge6"):
         J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
         Rc = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
         R = torch.zeros((coords.shape[0], 2), dtype=torch.float64, device="cuda")
+        Y = torch.zeros_like(R)
         mu = torch.empty((C, N), dtype=torch.float64, device="cuda")
         ctx.jacobian(Ud, J, R_cell=Rc, R=R)
         ctx.viscosity_resid(Ud, mu_qp=mu, R_cell=Rc, R=R)
-        ctx.gather(Ud)
-        G, wm = ctx.geometry()
+        ctx.jvp(Ud, Ud, Y, R=R)
         rp, ci = ctx.csr_pattern()
+        ctx.csr_slots()
         vals = torch.zeros(ci.numel(), dtype=torch.float64, device="cuda")
+        ctx.jacobian_csr(Ud, vals, R=R)
         ctx.scatter_assemble(R_cell=Rc, R=R, J_cell=J, csr_vals=vals)
         ctx.sync()
-    for derivs in (False, True):
-        S = ctx.albany_scratch(derivs)
-        ctx.albany_setup(derivs, S)
-        ctx.albany_evaluators(derivs, Ud, S)
-        for v in ("baseline", "optimized"):
-            ctx.albany_resid(derivs, v, S)
-        ctx.albany_extract(derivs, S, R_cell=Rc, J_cell=J if derivs else None)
-    ctx.sync()
+        if not full:
+            continue
+        ctx.gather(Ud)
+        G, wm = ctx.geometry()
+        cells = torch.arange(0, C, L, dtype=torch.int32, device="cuda")
+        beta = torch.full((coords.shape[0],), 2.0, dtype=torch.float64, device="cuda")
+        ctx.basal_friction(cells, beta, Ud, R, J_face=torch.empty((cells.numel(), N, N), dtype=torch.float64,
+                                                                    device="cuda"))
+        faces = torch.from_numpy(LT.lateral_faces(fp.polys, L)).cuda()
+        sd = torch.from_numpy(s).cuda()
+        ctx.lateral_pressure(faces, sd, R)
+        ctx.sync()
+        if geo == "stored":
+            ctx.set_lateral(faces, sd)
+            Un = torch.ones_like(Ud)
+            ctx.newton_solve(cells, beta, Un, max_newton=2, max_cg=20)
+            for derivs in (False, True):
+                S = ctx.albany_scratch(derivs)
+                ctx.albany_setup(derivs, S)
+                ctx.albany_evaluators(derivs, Ud, S)
+                for v in ("baseline", "optimized"):
+                    ctx.albany_resid(derivs, v, S)
+                ctx.albany_extract(derivs, S, R_cell=Rc, J_cell=J if derivs else None)
+            ctx.sync()
+
+
+for elem in ("hex8", "wedge6"):
+    run(elem, 5, 3, 3, True)          # every kernel, ragged last tile
+    run(elem, 48, 8, 1, False)        # more tiles than resident warps: the persistent pipelines
 print("sanitize workload done")
