@@ -15,6 +15,7 @@ Prints ONE JSON line on rank 0 (the driver's bench contract, DESIGN.md
 from __future__ import annotations
 
 import argparse
+import datetime
 import json
 import os
 import subprocess
@@ -69,8 +70,10 @@ def load_peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+    """nvidia-smi clocks / power / throttle reasons sampled every 20 ms; only the
+    samples whose nvidia-smi timestamp falls inside the timed region (host wall
+    clock, set by mark_start / mark_stop) are reported."""
+    Q = ("timestamp,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
@@ -78,20 +81,27 @@ class ClockSampler:
         self.idx = gpu_index
         self.proc = None
         self.file = None
+        self.t0 = self.t1 = None
 
     def start(self):
         try:
             self.file = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
             self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "20"],
                                          stdout=self.file, stderr=subprocess.DEVNULL)
         except Exception:
             self.proc = None
 
+    def mark_start(self):
+        self.t0 = time.time()
+
+    def mark_stop(self):
+        self.t1 = time.time()
+
     def stop(self):
         if self.proc is None:
             return None
-        time.sleep(0.15)
+        time.sleep(0.1)
         self.proc.terminate()
         try:
             self.proc.wait(timeout=5)
@@ -101,21 +111,26 @@ class ClockSampler:
         self.file.seek(0)
         rows = [r.split(", ") for r in self.file.read().strip().splitlines() if r.strip()]
         os.unlink(self.file.name)
-        sm, mx, reasons = [], 0.0, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        parsed = []
         for r in rows:
             try:
-                sm.append(float(r[1]))
-                mx = max(mx, float(r[2]))
-                for n, v in zip(names, r[5:9]):
-                    if v.strip().lower().startswith("active"):
-                        reasons.add(n)
+                ts = datetime.datetime.strptime(r[0].strip(), "%Y/%m/%d %H:%M:%S.%f").timestamp()
+                rs = {n for n, v in zip(names, r[5:9]) if v.strip().lower().startswith("active")}
+                parsed.append((ts, float(r[1]), float(r[2]), float(r[3]), rs))
             except Exception:
                 continue
-        if not sm:
+        if not parsed:
             return None
-        sm.sort()
-        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+        win = [p for p in parsed if self.t0 is not None and self.t0 <= p[0] <= (self.t1 or p[0])]
+        if not win:   # timed region shorter than the sampling period: the first sample after its start
+            after = [p for p in parsed if self.t0 is not None and p[0] >= self.t0]
+            win = after[:1] or parsed[-1:]
+        sm = sorted(p[1] for p in win)
+        pw = sorted(p[3] for p in win)
+        return {"sm_mhz": sm[len(sm) // 2], "sm_min_mhz": sm[0], "sm_max_mhz": max(p[2] for p in parsed),
+                "power_w": pw[len(pw) // 2], "reasons": sorted(set().union(*(p[4] for p in win))),
+                "samples": len(win), "window": "nvidia-smi every 20 ms, samples inside the timed region"}
 
 
 def dist_env():
@@ -346,11 +361,13 @@ def main():
     time.sleep(0.3)
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
+    clocks.mark_start()
     t0.record(stream)
     for i in range(args.steps):
         step(i)
     t1.record(stream)
     torch.cuda.synchronize(dev)
+    clocks.mark_stop()
     if world > 1:
         dist.barrier()
     clk = clocks.stop()

@@ -295,19 +295,14 @@ __device__ __forceinline__ void scatter_node(const EvalArgs &a, int32_t node, do
 }
 
 // Half-block split of the k = N/2 tangent block between the two lanes that
-// both own it (A/B switch; 1 = on)
+// both own it, and diagonal 2x2 blocks formed as symmetric (3 entries): the
+// tangent then forms each of the N(N+1)/2 distinct blocks of a cell once
+// (A/B switches; 1 = on)
 #ifndef SFO_KSPLIT
 #define SFO_KSPLIT 1
 #endif
-
-// Diagonal 2x2 tangent blocks formed as symmetric (3 entries; A/B switch)
 #ifndef SFO_DIAGSYM
 #define SFO_DIAGSYM 1
-#endif
-
-// Element Jacobians stored from registers (1) or staged + TMA bulk store (0)
-#ifndef SFO_JDIRECT
-#define SFO_JDIRECT 0
 #endif
 
 // Evaluation modes of the fused kernels
@@ -568,30 +563,6 @@ __device__ __forceinline__ void store_J(double *J_cell, int64_t cell0, int nvali
     bulk_commit();
 }
 
-// SFO_JDIRECT: lane (c, i) writes its rows' blocks (the same set as stage_J)
-// straight from registers to the global J image with 16-B stores (L2
-// evict_first); no shared-memory staging, no bulk store.  The stage buffer then
-// only holds the inputs, which frees shared memory for one more resident warp.
-__device__ __forceinline__ void st_global_v2(double *p, double x, double y, uint64_t pol) {
-    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(p), "d"(x), "d"(y),
-                 "l"(pol)
-                 : "memory");
-}
-template <class E>
-__device__ __forceinline__ void put_J_global(double *Jc, int i, const double (&Jb)[E::N / 2 + 1][2][2], uint64_t pol) {
-    constexpr int N = E::N, K = N / 2, LD = 2 * N;
-#pragma unroll
-    for (int k = 0; k <= K; ++k) {
-        const int j = (i + k) % N;
-        st_global_v2(Jc + (2 * i + 0) * LD + 2 * j, Jb[k][0][0], Jb[k][0][1], pol);
-        st_global_v2(Jc + (2 * i + 1) * LD + 2 * j, Jb[k][1][0], Jb[k][1][1], pol);
-        if (k > 0 && k < K) {
-            st_global_v2(Jc + (2 * j + 0) * LD + 2 * i, Jb[k][0][0], Jb[k][1][0], pol);
-            st_global_v2(Jc + (2 * j + 1) * LD + 2 * i, Jb[k][0][1], Jb[k][1][1], pol);
-        }
-    }
-}
-
 // NEXT-2 fused assembly: lane (c, i) adds its tangent blocks into the CSR
 // values through the per-cell slot table -- direct blocks (i, i+k), k = 0..K,
 // and, by symmetry, the transposed blocks (i+k, i) for 0 < k < K (the same
@@ -659,10 +630,7 @@ template <class E, int MODE>
 __host__ __device__ constexpr int warps_per_sm() {
     // wedge6 JAC: 16 (128 registers, 2-warp CTAs so that 16 x 13.7 KB of shared
     // memory fits next to the per-CTA driver reserve)
-    // hex8 JAC with direct J stores: 16.4 KB shared per warp -> 13 (<= 152 registers)
-    return forms_jac<MODE>() ? (E::N == 6 && MODE == M_JAC ? SFO_WEDGE_JAC_WARPS
-                                                           : (MODE == M_JAC && SFO_JDIRECT ? 13 : 12))
-                             : 16;
+    return forms_jac<MODE>() ? (E::N == 6 && MODE == M_JAC ? SFO_WEDGE_JAC_WARPS : 12) : 16;
 }
 // Independent persistent warps per CTA (each warp runs its own tile loop and
 // record ring in its own shared-memory slice; only __syncwarp is used).
@@ -685,16 +653,12 @@ struct EvalSmem {
     static constexpr int S_OFF = U_OFF + TC * E::UPITCH * 16;  // double  [TC][UPITCH]
     static constexpr int X_OFF = (int)round_up(S_OFF + TC * E::UPITCH * 8, 16);  // double2 [TC][UPITCH] (M_JVP)
     static constexpr int IN_BYTES = X_OFF + (MODE == M_JVP ? TC * E::UPITCH * 16 : 0);
-    // JAC with direct J stores: no staging; per-QP scalar fields overlay the
-    // tile's gathered U/s (consumed by the per-QP phase before it writes them)
-    static constexpr bool JDIRECT = MODE == M_JAC && SFO_JDIRECT;
-    static constexpr int J_BYTES = (MODE == M_JAC && !JDIRECT) ? TC * E::JPITCH * 8 : 0;
+    static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;
     static constexpr int STAGE = (int)round_up(IN_BYTES > J_BYTES ? IN_BYTES : J_BYTES, 128);
+    // per-QP scalar fields that fit in the stage's tail past the inputs (free until the J staging)
+    static constexpr int TAIL_OFF = (int)round_up(IN_BYTES, 16);
     static constexpr int FIELD = TC * Q * 8;
-    // per-QP scalar fields that fit in the stage's tail past the inputs (free until the J staging),
-    // or (JDIRECT) over the gathered U/s
-    static constexpr int TAIL_OFF = JDIRECT ? U_OFF : (int)round_up(IN_BYTES, 16);
-    static constexpr int TAIL_FIT = JDIRECT ? (IN_BYTES - U_OFF) / FIELD : (STAGE - TAIL_OFF) / FIELD;
+    static constexpr int TAIL_FIT = (STAGE - TAIL_OFF) / FIELD;
     static constexpr int TAIL_FIELDS = TAIL_FIT < 3 ? TAIL_FIT : 3;
     // residual-only and J.v modes keep the per-QP scalars in registers (partial-sum exchange)
     static constexpr bool PSUM = MODE == M_RESID || MODE == M_JVP;
@@ -765,8 +729,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
     const int c = act ? E::lane_cell(l) : TC, s = act ? E::lane_sub(l) : 0;  // (cell, node-or-qp)
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
 
-    const uint64_t pol_stream = policy_evict_first();  // every lane (direct J stores)
+    uint64_t pol_stream = 0;
     if (l == 0) {
+        pol_stream = policy_evict_first();
         for (int k = 0; k < NSTAGE; ++k) mbar_init(&bar[k], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         for (int k = 0; k < NSTAGE; ++k) {
@@ -812,10 +777,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
         // ---- per-QP phase: lane <-> (cell c, qp s) ----
         double gq[S::PSUM ? N : 1][3];  // G_n(q) kept for the partial sums (PSUM modes)
         double qv[S::PSUM ? 15 : 1];
-        double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
-        double dg[6] = {0, 0, 0, 0, 0, 0};
-        const int q = s;
         if (act) {
+            const int q = s;
+            double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+            double dg[6] = {0, 0, 0, 0, 0, 0};
 #pragma unroll
             for (int n = 0; n < N; ++n) {
                 const double g0 = rg[gidx<E>(n, q, 0, c)];
@@ -839,9 +804,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
                     dg[3] = fma(xv.y, g0, dg[3]); dg[4] = fma(xv.y, g1, dg[4]); dg[5] = fma(xv.y, g2, dg[5]);
                 }
             }
-        }
-        if (S::JDIRECT) __syncwarp();  // U/s read by every lane before the qs fields overwrite them
-        if (act) {
             if constexpr (S::PSUM)
                 qp_tail<E, MODE>(a, RegQs{qv}, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx,
                                  vy, vz, gs0, gs1, dg);
@@ -934,19 +896,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
         __syncwarp();  // every lane is done with this stage's record and qs
 
         if (CSR) csr_scatter<E>(a.csr_vals, c, s, act && c < nvalid, srow, rp, Jb);
-        auto refill = [&]() {
-            if (l == 0 && NSTAGE < 3) {
-                const int64_t nt = tile + (int64_t)NSTAGE * vg;
-                if (nt < a.ntiles) {
-                    mbar_arrive_expect_tx(&bar[st], R::BYTES);
-                    bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
-                }
-            }
-        };
-        if (JAC && S::JDIRECT) {
-            refill();  // the record's reads are done (__syncwarp above); J goes out from registers
-            if (act && c < nvalid) put_J_global<E>(a.J_cell + (cell0 + c) * (4 * N * N), s, Jb, pol_stream);
-        } else if (JAC) {
+        if (JAC) {
             if (act) stage_J<E>(reinterpret_cast<double *>(stage), c, s, Jb);
             fence_proxy_async_smem();
             __syncwarp();
@@ -955,7 +905,13 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
                 if (NSTAGE < 3) bulk_wait_read0();  // staging read -> the buffer may take the next record
             }
         }
-        if (!(JAC && S::JDIRECT)) refill();
+        if (l == 0 && NSTAGE < 3) {
+            const int64_t nt = tile + (int64_t)NSTAGE * vg;
+            if (nt < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[st], R::BYTES);
+                bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
+            }
+        }
         if (act && c < nvalid) {
             if (a.R) scatter_node(a, gnode, R0, R1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
