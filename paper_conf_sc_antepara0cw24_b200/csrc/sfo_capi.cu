@@ -45,6 +45,10 @@ struct stokesfo_ctx {
     int64_t lat_n = 0;
     const double *lat_surface = nullptr;
     double lat_rho_i_g = 0.0, lat_rho_w_g = 0.0, lat_sea = 0.0;
+    // wedge6 element-Jacobian tensor map (TMA 2-D store of a padded tile), re-encoded when J_cell moves
+    CUtensorMap jmap;
+    const double *jmap_ptr = nullptr;
+    bool jmap_ok = false;
 };
 
 namespace {
@@ -172,6 +176,48 @@ int create_impl(stokesfo_ctx *c) {
     return cuda_status();
 }
 
+// cuTensorMapEncodeTiled from the driver (no -lcuda link: fetched once through the runtime)
+typedef CUresult (*encode_tiled_fn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                    const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+encode_tiled_fn tensor_map_encoder() {
+    static encode_tiled_fn fn = [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            p = nullptr;
+        cudaGetLastError();
+        return reinterpret_cast<encode_tiled_fn>(p);
+    }();
+    return fn;
+}
+
+// J_cell as a 2-D tensor [C][NN] doubles, box (JPITCH x TC): one TMA store per
+// tile writes the TC cells of a padded (odd-pitch) staging image; the padding
+// columns and rows past C are outside the tensor.  STOKESFO_JMAP=0 disables it
+// (per-cell 1-D bulk copies).
+template <class E>
+bool wedge_jmap(stokesfo_ctx *c, const double *J_cell) {
+    constexpr int NN = 4 * E::N * E::N;
+    if (E::JPITCH == NN || J_cell == nullptr) return false;
+    if (const char *e = getenv("STOKESFO_JMAP"))
+        if (atoi(e) == 0) return false;
+    if (c->jmap_ptr == J_cell) return c->jmap_ok;
+    c->jmap_ptr = J_cell;
+    c->jmap_ok = false;
+    encode_tiled_fn enc = tensor_map_encoder();
+    if (!enc || c->d.num_cells > 0x7fffffff) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)NN, (cuuint64_t)c->d.num_cells};
+    const cuuint64_t strides[1] = {(cuuint64_t)NN * 8};
+    const cuuint32_t box[2] = {(cuuint32_t)E::JPITCH, (cuuint32_t)E::TC};
+    const cuuint32_t estr[2] = {1, 1};
+    c->jmap_ok = enc(&c->jmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double *>(J_cell), dims, strides, box,
+                     estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    return c->jmap_ok;
+}
+
 template <class E, int MODE>
 int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R, double *J_cell,
               const double *X = nullptr, double *Y = nullptr, double *csr_vals = nullptr) {
@@ -206,15 +252,17 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
                 : MODE == M_JVP ? c->grid_jvp
                 : MODE == M_CSR ? c->grid_csr : c->grid_resid;
     const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
+    a.use_jmap = (!otf && MODE == M_JAC && wedge_jmap<E>(c, J_cell)) ? 1 : 0;
+    const CUtensorMap jm = a.use_jmap ? c->jmap : CUtensorMap{};
     constexpr int WPC = warps_per_cta<E, MODE>();  // eval_kernel only (the on-the-fly kernel: 1)
     const int grid = (int)std::min<int64_t>(g, otf ? c->ntiles : (c->ntiles + WPC - 1) / WPC);
     const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_RESID ? c->nstage_resid : 2);
     if (otf)
         eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
     else if (MODE != M_CSR && ns == 3)
-        eval_kernel<E, MODE, 3><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 3>(), c->stream>>>(a);
+        eval_kernel<E, MODE, 3><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 3>(), c->stream>>>(a, jm);
     else
-        eval_kernel<E, MODE, 2><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 2>(), c->stream>>>(a);
+        eval_kernel<E, MODE, 2><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 2>(), c->stream>>>(a, jm);
     return cuda_status();
 }
 

@@ -5,6 +5,7 @@
 // here from the basis formulas, not shared.
 #pragma once
 #include <cstdint>
+#include <cuda.h>  // CUtensorMap (type only; the encoder is fetched through cudaGetDriverEntryPoint)
 #include <cuda_runtime.h>
 
 namespace sfo {
@@ -121,6 +122,14 @@ __device__ __forceinline__ void bulk_s2g(void *dst, const void *src, uint32_t by
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(dst),
                  "r"(smem_u32(src)), "r"(bytes), "l"(pol)
                  : "memory");
+}
+// shared -> global 2-D tensor store (TMA; bulk-group completion); out-of-bound box elements are skipped
+__device__ __forceinline__ void tensor_s2g_2d(const CUtensorMap *map, int x, int y, const void *src, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%1, %2}], [%3], %4;" ::"l"(
+            reinterpret_cast<uint64_t>(map)),
+        "r"(x), "r"(y), "r"(smem_u32(src)), "l"(pol)
+        : "memory");
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }

@@ -268,6 +268,7 @@ struct EvalArgs {
     const int64_t *rowptr;    // [2 nodes + 1]
     const uint64_t *slots;    // [C][N] rows of N uint8 slots (8-byte pitch)
     double *csr_vals;         // [nnz] (+=)
+    int use_jmap;             // wedge6 M_JAC: J tile stored through the kernel's tensor-map parameter
 };
 
 constexpr int REM_MAX = 7;                 // remote copies of one node (<= 8 parts meet at a vertex)
@@ -549,13 +550,20 @@ __device__ __forceinline__ void stage_J(double *base, int c2, int i, const doubl
     }
 }
 
-// One lane issues the TMA bulk store(s) of a staged tile of element Jacobians
-// (one copy when the staging pitch is the global image, else one per cell).
+// One lane issues the TMA store(s) of a staged tile of element Jacobians: one
+// 1-D bulk copy when the staging pitch is the global image (hex8); for the
+// padded wedge6 staging (pitch JPITCH > NN) one 2-D tensor store through the
+// tensor map J viewed as [C][NN] doubles with a (JPITCH x TC) box -- the box's
+// padding columns and the rows past C fall outside the tensor and are not
+// written -- or, without a map, one bulk copy per cell.
 template <class E>
-__device__ __forceinline__ void store_J(double *J_cell, int64_t cell0, int nvalid, const char *stage, uint64_t pol) {
+__device__ __forceinline__ void store_J(double *J_cell, int64_t cell0, int nvalid, const char *stage, uint64_t pol,
+                                        const CUtensorMap *jmap = nullptr) {
     constexpr int NN = 4 * E::N * E::N;
     if (E::JPITCH == NN) {
         bulk_s2g(J_cell + cell0 * NN, stage, (uint32_t)(nvalid * NN * 8), pol);
+    } else if (jmap) {
+        tensor_s2g_2d(jmap, 0, (int)cell0, stage, pol);
     } else {
         for (int c = 0; c < nvalid; ++c)
             bulk_s2g(J_cell + (cell0 + c) * NN, stage + c * E::JPITCH * 8, (uint32_t)(NN * 8), pol);
@@ -710,7 +718,7 @@ __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
 
 template <class E, int MODE, int NSTAGE>
 __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E, MODE>() / warps_per_cta<E, MODE>()))
-    eval_kernel(EvalArgs a) {
+    eval_kernel(EvalArgs a, const __grid_constant__ CUtensorMap jmap) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
     static_assert(N == Q, "lane mappings assume N == Q");
@@ -901,7 +909,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
             fence_proxy_async_smem();
             __syncwarp();
             if (l == 0) {
-                store_J<E>(a.J_cell, cell0, nvalid, stage, pol_stream);
+                store_J<E>(a.J_cell, cell0, nvalid, stage, pol_stream, a.use_jmap ? &jmap : nullptr);
                 if (NSTAGE < 3) bulk_wait_read0();  // staging read -> the buffer may take the next record
             }
         }
