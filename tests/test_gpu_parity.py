@@ -409,3 +409,28 @@ def test_csr_slots_and_fused_assembly(torch, elem, geometry):
     ctx.sync()
     assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2).all()
     _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
+
+
+@pytest.mark.parametrize("drop", [0, 11])
+def test_wedge_tensor_map_store(torch, drop, monkeypatch):
+    """wedge6 J tiles leave the kernel as ONE 2-D TMA tensor store of the padded
+    (146-double pitch) staging image per tile (csrc/sfo_kernels.cuh store_J): the
+    result must be bitwise the per-cell bulk-copy path's (STOKESFO_JMAP=0), and
+    neither the padding columns nor the box rows past the last cell may land in
+    memory: a sentinel after J[C-1] (ragged last tile for drop=11) stays intact."""
+    ctx, orc = _setup(torch, "wedge6", drop=drop)
+    C, N = ctx.num_cells, ctx.N
+    U = _t(torch, orc["U"])
+    outs = []
+    for jmap in ("1", "0"):
+        monkeypatch.setenv("STOKESFO_JMAP", jmap)
+        buf = torch.full((C + 3, 2 * N, 2 * N), 7.0, dtype=torch.float64, device="cuda")
+        ctx.jacobian(U, buf[:C])
+        ctx.sync()
+        outs.append(buf.cpu().numpy())
+    a, b = outs
+    assert (a[C:] == 7.0).all() and (b[C:] == 7.0).all()
+    assert np.array_equal(a[:C], b[:C])
+    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
+                     mode="jac")
+    assert _cell_rel(a[:C], ref["J_cell"]) <= TOL
