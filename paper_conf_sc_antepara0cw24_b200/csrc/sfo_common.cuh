@@ -33,9 +33,19 @@ struct Hex8 {
     static constexpr int UPITCH = N;
     __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * TC + c) * Q + q; }
 };
+#ifndef SFO_WEDGE_SLAB32
+#define SFO_WEDGE_SLAB32 1
+#endif
 struct Wedge6 {
     static constexpr int N = 6, Q = 6, TC = 5, ELEM = 1;  // 30 active lanes
+#if SFO_WEDGE_SLAB32
+    // 32-double slabs (2 padding slots per (qp, dir): +288 B per 5-cell record) with the q-rotated slot map
+    // (c + 5n + 5q) mod 32: per-QP-phase GradBF loads conflict-free (36 vs 57 wavefronts per tile in the bank
+    // model), per-node loads 162 (same), and the slot arithmetic is a power-of-two mask
+    static constexpr int SLAB = 32;
+#else
     static constexpr int SLAB = 30;
+#endif
     static constexpr int JPITCH = 4 * N * N + 2;  // odd 16-B pitch: conflict-free staging, per-cell bulk stores
     // lane l <-> (cell l % 5, node-or-qp l / 5) (node-major), slot (29c + 25n) mod 30:
     // chosen by a search over affine slot maps with the shared-memory bank model
@@ -43,7 +53,11 @@ struct Wedge6 {
     __host__ __device__ static constexpr int lane_cell(int l) { return l % TC; }
     __host__ __device__ static constexpr int lane_sub(int l) { return l / TC; }
     __host__ __device__ static constexpr int lane_of(int c, int sub) { return sub * TC + c; }
+#if SFO_WEDGE_SLAB32
+    __host__ __device__ static constexpr int slot(int c, int n, int q) { return (c + 5 * n + 5 * q) & 31; }
+#else
     __host__ __device__ static constexpr int slot(int c, int n, int) { return (29 * c + 25 * n) % 30; }
+#endif
     // odd 16-B cell pitch for the gathered U rows; per-QP scalars qp-major
     // (lanes (c, q) of the per-QP phase then write consecutive addresses)
     static constexpr int UPITCH = 7;
