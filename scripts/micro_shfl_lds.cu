@@ -7,7 +7,8 @@
 #include <cstdio>
 #include <cuda_runtime.h>
 
-template <int MODE>  // 0 = LDS only, 1 = SHFL only, 2 = both
+template <int MODE>  // 0 = LDS only, 1 = SHFL only, 2 = both, 3 = LDS.128 with lane pairs on one 16-B chunk,
+                     // 4 = LDS.128 all lanes distinct
 __global__ void loop(double *out, int iters) {
     __shared__ double sm[32 * 16 + 32];
     const int l = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -19,8 +20,16 @@ __global__ void loop(double *out, int iters) {
     for (int it = 0; it < iters; ++it) {
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
-            if (MODE != 1) acc[k] += base[(l + k + it) & 31];                  // conflict-free LDS.64
-            if (MODE != 0) acc[k] += __shfl_sync(0xffffffffu, v, (l + k) & 31);  // SHFL x2 (double)
+            if (MODE == 0 || MODE == 2) acc[k] += base[(l + k + it) & 31];      // conflict-free LDS.64
+            if (MODE == 1 || MODE == 2) acc[k] += __shfl_sync(0xffffffffu, v, (l + k) & 31);  // SHFL x2
+            if (MODE == 3) {  // lanes 2m, 2m+1 read chunk m: 16 distinct 16-B chunks per warp
+                const double2 t = reinterpret_cast<const double2 *>(sm)[((l >> 1) + k + it) & 15];
+                acc[k] += t.x * t.y;
+            }
+            if (MODE == 4) {  // 32 distinct 16-B chunks
+                const double2 t = reinterpret_cast<const double2 *>(sm)[(l + k + it) & 31];
+                acc[k] += t.x * t.y;
+            }
         }
         v += 1.0;
     }
@@ -39,14 +48,16 @@ int main() {
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
     const int iters = 1 << 16;
-    const char *names[3] = {"lds64", "shfl64", "both"};
+    const char *names[5] = {"lds64", "shfl64", "both", "lds128_pairs", "lds128_distinct"};
     for (int rep = 0; rep < 2; ++rep)
-        for (int m = 0; m < 3; ++m) {
+        for (int m = 0; m < 5; ++m) {
             cudaEventRecord(e0);
             const dim3 g(sms * 4), b(256);
             if (m == 0) loop<0><<<g, b>>>(out, iters);
             if (m == 1) loop<1><<<g, b>>>(out, iters);
             if (m == 2) loop<2><<<g, b>>>(out, iters);
+            if (m == 3) loop<3><<<g, b>>>(out, iters);
+            if (m == 4) loop<4><<<g, b>>>(out, iters);
             cudaEventRecord(e1);
             cudaEventSynchronize(e1);
             float ms;
