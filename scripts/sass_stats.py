@@ -17,4 +17,4 @@ for fn in re.split(r"\n\s+Function : ", txt)[1:]:
     ins = [l for l in fn.split("\n") if re.match(r"\s+/\*[0-9a-f]{4}\*/", l)]
     c = lambda k: sum(1 for l in ins if re.search(k, l))
     print(f"{name[:56]:56s} n={len(ins):5d} DFMA={c(r'DFMA'):4d} DMUL={c(r'DMUL'):4d} DADD={c(r'DADD'):4d} "
-          f"LDS={c(r'LDS'):4d} STS={c(r'STS'):4d} SEL={c(r' F?SEL'):4d} SHFL={c(r'SHFL'):3d}")
+          f"LDS={c(r"LDS"):4d} LDS128={c(r"LDS\.128"):3d} STS={c(r'STS'):4d} SEL={c(r' F?SEL'):4d} SHFL={c(r'SHFL'):3d}")
