@@ -45,7 +45,8 @@ def run(elem, n, L, drop, full):
         beta = torch.full((coords.shape[0],), 2.0, dtype=torch.float64, device="cuda")
         ctx.basal_friction(cells, beta, Ud, R, J_face=torch.empty((cells.numel(), N, N), dtype=torch.float64,
                                                                     device="cuda"))
-        faces = torch.from_numpy(LT.lateral_faces(fp.polys, L)).cuda()
+        lf = LT.lateral_faces(fp.polys, L)
+        faces = torch.from_numpy(np.ascontiguousarray(lf[lf[:, 0] < C])).cuda()  # faces of dropped cells: EMESH
         sd = torch.from_numpy(s).cuda()
         ctx.lateral_pressure(faces, sd, R)
         ctx.sync()
