@@ -486,13 +486,13 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const QS &qs, 
                 }
                 if (SFO_KSPLIT && k == K) {
                     // block (i, i+K) is also block (i+K, i)^T of the partner lane: each lane of
-                    // the pair forms half of it (lanes i < K row a = 0, lanes i >= K column
-                    // b = 1 of their own block), completed by ksplit_exchange
+                    // the pair forms half of it (lanes i < K column b = 0: (0,0), (1,0); lanes
+                    // i >= K row a = 1 of their own block: (1,1), (1,0)), so only the first
+                    // operand differs between the two (m00 / m11); ksplit_exchange completes it
                     const bool lo = i < K;
-                    const double ax = lo ? m00x : m01x, ay = lo ? m00y : m01y, az = lo ? m00z : m01z;
-                    const double bx = lo ? m01x : m11x, by = lo ? m01y : m11y, bz = lo ? m01z : m11z;
+                    const double ax = lo ? m00x : m11x, ay = lo ? m00y : m11y, az = lo ? m00z : m11z;
                     Jb[k][0][0] = fma(az, gj2, fma(ay, gj1, fma(ax, gj0, Jb[k][0][0])));
-                    Jb[k][0][1] = fma(bz, gj2, fma(by, gj1, fma(bx, gj0, Jb[k][0][1])));
+                    Jb[k][0][1] = fma(m10z, gj2, fma(m10y, gj1, fma(m10x, gj0, Jb[k][0][1])));
                     continue;
                 }
                 // explicit 3-deep DFMA chains into the accumulators (no DMUL/DADD)
@@ -509,9 +509,9 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const QS &qs, 
 }
 
 // Completes block k = K after node_accumulate's split (SFO_KSPLIT): lane i < K
-// holds P00, P01 of P = J[(i,.),(i+K,.)], its partner lane i+K holds P10, P11
-// (column b = 1 of its own block P^T).  One exchange of two doubles; every lane
-// of the warp must call this.
+// holds P00, P10 of P = J[(i,.),(i+K,.)], its partner lane i+K holds P11, P01
+// (entries (1,1), (1,0) of its own block P^T).  One exchange of two doubles;
+// every lane of the warp must call this.
 template <class E>
 __device__ __forceinline__ void ksplit_exchange(double (&Jb)[E::N / 2 + 1][2][2], int c, int i, bool act) {
     constexpr int N = E::N, K = N / 2;
@@ -519,14 +519,16 @@ __device__ __forceinline__ void ksplit_exchange(double (&Jb)[E::N / 2 + 1][2][2]
     const int src = act ? E::lane_of(c, (i + K) % N) : (int)(threadIdx.x & 31);
     const double e0 = Jb[K][0][0], e1 = Jb[K][0][1];
     const double f0 = __shfl_sync(0xffffffffu, e0, src), f1 = __shfl_sync(0xffffffffu, e1, src);
-    if (i < K) {
-        Jb[K][1][0] = f0;
-        Jb[K][1][1] = f1;
-    } else {  // own block = P^T = [[P00, P10], [P01, P11]]
+    if (i < K) {  // e = (P00, P10), f = (P11, P01)
+        Jb[K][0][0] = e0;
+        Jb[K][0][1] = f1;
+        Jb[K][1][0] = e1;
+        Jb[K][1][1] = f0;
+    } else {  // e = (P11, P01), f = (P00, P10); own block = P^T = [[P00, P10], [P01, P11]]
         Jb[K][0][0] = f0;
-        Jb[K][0][1] = e0;
-        Jb[K][1][0] = f1;
-        Jb[K][1][1] = e1;
+        Jb[K][0][1] = f1;
+        Jb[K][1][0] = e1;
+        Jb[K][1][1] = e0;
     }
 }
 
