@@ -154,3 +154,50 @@ def test_fullsize_csr_assembly_sampled_rows(cfg):
             assert (np.abs(got - val) <= TOL * absv + 1e-300).all(), (fused, v, a)
         del vals
         torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("cfg", ["C4", "C5"])
+def test_fullsize_jvp_sampled(cfg):
+    """NEXT-3 at full size, in the launch bench.py --op jvp times (Y += J(U) X with
+    R += R(U) in the same pass): Y and R at sampled nodes equal the oracle's element
+    AD Jacobians of every incident cell applied to X, and the oracle residual."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_antepara0cw24_b200 import StokesFO
+    fp, L, elem = synth.make_config(cfg)
+    conn, coords = O.extrude(fp.xy, fp.polys, fp.b, fp.H, L)
+    U = synth.velocity_balance(fp, L, seed=12)
+    s = synth.surface_nodal(fp, L)
+    kc = synth.flow_factor(fp, L)
+    C, N = conn.shape
+    nn = coords.shape[0]
+    X = np.random.default_rng(5).normal(0, 10.0, (nn, 2))
+    ctx = StokesFO(elem, torch.from_numpy(conn).cuda(), torch.from_numpy(coords).cuda(),
+                   surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda())
+    Y = torch.zeros((nn, 2), dtype=torch.float64, device="cuda")
+    R = torch.zeros((nn, 2), dtype=torch.float64, device="cuda")
+    ctx.jvp(torch.from_numpy(U).cuda(), torch.from_numpy(X).cuda(), Y, R=R)
+    ctx.sync()
+    rng = np.random.default_rng(13)
+    nodes = np.unique(np.concatenate([rng.integers(0, nn, 150), [0, nn - 1]]))
+    e = O.ELEM[elem]
+    rows, out = _sample_nodes_expect(e, conn, coords, U, s, kc, nodes, True)
+    nr = len(rows)
+    Xc = X[conn[rows]].reshape(nr, 2 * N)
+    JX = np.einsum("ckl,cl->ck", out["J_cell"], Xc).reshape(nr, N, 2)
+    # per-entry bound as in test_jvp_matrix_free_parity: 1e-12 of max|J_c| |X_c| per contributing cell
+    scale_c = (np.abs(out["J_cell"]).reshape(nr, -1).max(1) * np.abs(Xc).sum(1))[:, None, None] * np.ones((nr, N, 2))
+    Yref = np.zeros((nn, 2))
+    Yscale = np.zeros((nn, 2))
+    Rref = np.zeros((nn, 2))
+    Aref = np.zeros((nn, 2))
+    np.add.at(Yref, conn[rows].reshape(-1), JX.reshape(-1, 2))
+    np.add.at(Yscale, conn[rows].reshape(-1), scale_c.reshape(-1, 2))
+    np.add.at(Rref, conn[rows].reshape(-1), out["R_cell"].reshape(-1, 2))
+    np.add.at(Aref, conn[rows].reshape(-1), np.abs(out["R_cell"]).reshape(-1, 2))
+    idx = torch.from_numpy(nodes).cuda()
+    Yg = Y[idx].cpu().numpy()
+    Rg = R[idx].cpu().numpy()
+    assert (np.abs(Yg - Yref[nodes]) <= TOL * Yscale[nodes]).all()
+    assert (np.abs(Rg - Rref[nodes]) <= TOL * Aref[nodes] + 1e-300).all()
