@@ -98,6 +98,12 @@ enum : int { ERR_DETJ = 1, ERR_CONN = 2, ERR_CSR = 4 };
 // ---------------------------------------------------------------------------
 // PTX helpers (sm_90+/sm_100a): mbarrier + 1-D bulk async copies (TMA engine)
 // ---------------------------------------------------------------------------
+// R[i] += v for a pointer into global memory (local or NVLink-mapped peer):
+// red.global.add.f64 straight away.  atomicAdd on a generic double* makes the
+// compiler test the address space first (two QSPC + branches per call).
+__device__ __forceinline__ void red_add(double *p, double v) {
+    asm volatile("red.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+}
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }

@@ -279,8 +279,8 @@ constexpr int REM_ROW = 1 + 2 * REM_MAX;
 // NVLink-mapped peer pointer): the halo sum happens inside the evaluation
 // kernel, no pack / exchange / unpack.
 __device__ __forceinline__ void scatter_node(const EvalArgs &a, int32_t node, double r0, double r1) {
-    atomicAdd(a.R + 2 * (int64_t)node + 0, r0);
-    atomicAdd(a.R + 2 * (int64_t)node + 1, r1);
+    red_add(a.R + 2 * (int64_t)node + 0, r0);
+    red_add(a.R + 2 * (int64_t)node + 1, r1);
     if (a.rem) {
         const int32_t row = __ldg(a.rem + node);
         if (row >= 0) {
@@ -288,8 +288,8 @@ __device__ __forceinline__ void scatter_node(const EvalArgs &a, int32_t node, do
             const int cnt = t[0];
             for (int k = 0; k < cnt; ++k) {
                 double *pr = a.peers[t[1 + 2 * k]] + 2 * (int64_t)t[2 + 2 * k];
-                atomicAdd(pr + 0, r0);
-                atomicAdd(pr + 1, r1);
+                red_add(pr + 0, r0);
+                red_add(pr + 1, r1);
             }
         }
     }
@@ -594,17 +594,17 @@ __device__ __forceinline__ void csr_scatter(double *vals, int c, int i, bool liv
         if (live) {
             const int sij = (int)((srow >> (8 * j)) & 0xff);
             double *p0 = vals + rp.x + 2 * sij, *p1 = vals + rp.y + 2 * sij;
-            atomicAdd(p0, Jb[k][0][0]);
-            atomicAdd(p0 + 1, Jb[k][0][1]);
-            atomicAdd(p1, Jb[k][1][0]);
-            atomicAdd(p1 + 1, Jb[k][1][1]);
+            red_add(p0, Jb[k][0][0]);
+            red_add(p0 + 1, Jb[k][0][1]);
+            red_add(p1, Jb[k][1][0]);
+            red_add(p1 + 1, Jb[k][1][1]);
             if (k > 0 && k < K) {  // J[(j,a),(i,b)] = J[(i,b),(j,a)]
                 const int sji = (int)((srow_j >> (8 * i)) & 0xff);
                 double *q0 = vals + rj0 + 2 * sji, *q1 = vals + rj1 + 2 * sji;
-                atomicAdd(q0, Jb[k][0][0]);
-                atomicAdd(q0 + 1, Jb[k][1][0]);
-                atomicAdd(q1, Jb[k][0][1]);
-                atomicAdd(q1 + 1, Jb[k][1][1]);
+                red_add(q0, Jb[k][0][0]);
+                red_add(q0 + 1, Jb[k][1][0]);
+                red_add(q1, Jb[k][0][1]);
+                red_add(q1 + 1, Jb[k][1][1]);
             }
         }
     }
@@ -926,8 +926,8 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
             if (a.R) scatter_node(a, gnode, R0, R1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
             if (JVP) {
-                atomicAdd(a.Y + 2 * (int64_t)gnode + 0, dR0);
-                atomicAdd(a.Y + 2 * (int64_t)gnode + 1, dR1);
+                red_add(a.Y + 2 * (int64_t)gnode + 0, dR0);
+                red_add(a.Y + 2 * (int64_t)gnode + 1, dR1);
             }
         }
         if (ntile < a.ntiles) gather_store<E, MODE>(smem + nst * S::STAGE, nxt);
@@ -1127,8 +1127,8 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
         if (act && c < nvalid) {
             if (a.R) scatter_node(a, gnode, R0, R1);
             if (JVP) {
-                atomicAdd(a.Y + 2 * (int64_t)gnode + 0, dR0);
-                atomicAdd(a.Y + 2 * (int64_t)gnode + 1, dR1);
+                red_add(a.Y + 2 * (int64_t)gnode + 0, dR0);
+                red_add(a.Y + 2 * (int64_t)gnode + 1, dR1);
             }
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }
@@ -1234,8 +1234,8 @@ __global__ void basal_friction_kernel(int64_t nfaces, const int32_t *__restrict_
     }
 #pragma unroll
     for (int i = 0; i < NB; ++i) {
-        atomicAdd(R + 2 * (int64_t)nid[i], Rf[i][0]);
-        atomicAdd(R + 2 * (int64_t)nid[i] + 1, Rf[i][1]);
+        red_add(R + 2 * (int64_t)nid[i], Rf[i][0]);
+        red_add(R + 2 * (int64_t)nid[i] + 1, Rf[i][1]);
     }
     if (Jf) {
         double *J = Jf + f * ND * ND;
@@ -1323,8 +1323,8 @@ __global__ void lateral_pressure_kernel(int64_t nfaces, int64_t ncells, const in
     }
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
-        atomicAdd(R + 2 * (int64_t)nid[i], Rf[i][0]);
-        atomicAdd(R + 2 * (int64_t)nid[i] + 1, Rf[i][1]);
+        red_add(R + 2 * (int64_t)nid[i], Rf[i][0]);
+        red_add(R + 2 * (int64_t)nid[i] + 1, Rf[i][1]);
     }
 }
 
@@ -1338,8 +1338,8 @@ __global__ void scatter_r_kernel(int64_t ncells, const int32_t *__restrict__ con
     if (gid >= ncells * N) return;
     const int64_t g = conn[gid];
     const double2 v = Rc[gid];
-    atomicAdd(R + 2 * g + 0, v.x);
-    atomicAdd(R + 2 * g + 1, v.y);
+    red_add(R + 2 * g + 0, v.x);
+    red_add(R + 2 * g + 1, v.y);
 }
 
 template <int N>
@@ -1361,7 +1361,7 @@ __global__ void scatter_csr_kernel(int64_t ncells, const int32_t *__restrict__ c
             if (colidx[mid] < col) lo = mid + 1; else hi = mid;
         }
         if (lo < hi0 && colidx[lo] == col)
-            atomicAdd(vals + lo, Jc[cell * ND * ND + r * ND + s]);
+            red_add(vals + lo, Jc[cell * ND * ND + r * ND + s]);
         else
             atomicOr(err, ERR_CSR);
     }
@@ -1412,8 +1412,8 @@ __global__ void scatter_csr_slots_kernel(int64_t ncells, const int32_t *__restri
     for (int j = 0; j < N; ++j) {
         const double2 v = __ldcs(Jr + j);  // streamed once
         double *p = base + 2 * (int)((w >> (8 * j)) & 0xff);
-        atomicAdd(p, v.x);
-        atomicAdd(p + 1, v.y);
+        red_add(p, v.x);
+        red_add(p + 1, v.y);
     }
 }
 
