@@ -215,6 +215,26 @@ def run_reference(args, rank, world):
 # GPU leg
 # ---------------------------------------------------------------------------
 
+def relaunch(n: int) -> int:
+    """`python bench.py --gpus N` without a torchrun environment: start N ranks
+    (one process per GPU) with torch.distributed.run on 127.0.0.1 and return
+    their exit status; rank 0 prints the JSON line."""
+    import socket
+    if os.environ.get("STOKESFO_BENCH_BACKEND", "nccl") == "nccl":
+        import torch
+        have = torch.cuda.device_count()
+        if have < n:
+            sys.stderr.write(f"bench.py: --gpus {n} needs {n} visible GPUs, found {have} "
+                             "(STOKESFO_BENCH_BACKEND=gloo shares one GPU for debugging)\n")
+            return 2
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -235,9 +255,14 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
+        return relaunch(args.gpus)
     rank, world, local = dist_env()
     if args.impl == "reference":
         return run_reference(args, rank, world)
+    if world != args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} but WORLD_SIZE = {world}\n")
+        return 2
 
     import numpy as np
     import torch
@@ -271,7 +296,9 @@ def main():
     stream = torch.cuda.current_stream(dev)
     ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream, geometry=args.geometry)
     J = torch.empty((C, 2 * N, 2 * N) if args.op == "jacobian" else (0,), dtype=torch.float64, device=dev)
-    Xd = torch.from_numpy(np.random.default_rng(5).normal(0, 10.0, (NN, 2))).to(dev) if args.op == "jvp" else None
+    # J.v direction: one global seeded field, restricted to this rank's nodes (consistent across ranks)
+    x_global = np.random.default_rng(5).normal(0, 10.0, (coords_g.shape[0], 2)) if args.op == "jvp" else None
+    Xd = torch.from_numpy(np.ascontiguousarray(x_global[gids])).to(dev) if args.op == "jvp" else None
     Yd = torch.zeros((NN, 2), dtype=torch.float64, device=dev) if args.op == "jvp" else None
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     nnz, vals = 0, None
@@ -285,7 +312,7 @@ def main():
     halo_mode = "none"
     if world > 1:
         if args.halo == "p2p":
-            p2p = P2PHalo(ctx, part, dev, gloo_debug=(backend != "nccl"))
+            p2p = P2PHalo(ctx, part, dev, gloo_debug=(backend != "nccl"), fields=2 if args.op == "jvp" else 1)
             if not p2p.ok:
                 p2p.close()
                 p2p = None
@@ -300,33 +327,47 @@ def main():
 
     k0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     k1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    R_last = [R]
+    R_last = [R, Yd]
 
-    def step(i=None):
+    def begin():
+        """This step's (R, Y) output buffers, zeroed (Y only for --op jvp)."""
         if p2p is not None:
-            Rc = p2p.begin()
-        else:
-            Rc = R
-            Rc.zero_()
-        if vals is not None:
-            vals.zero_()
-        if i is not None:
-            k0[i].record(stream)
-        if args.op == "jacobian":
-            ctx.jacobian(U, J, R=Rc)
-        elif args.op == "jac_csr":
-            ctx.jacobian_csr(U, vals, R=Rc)
-        elif args.op == "jvp":
-            ctx.jvp(U, Xd, Yd, R=Rc)
-        else:
-            ctx.viscosity_resid(U, R=Rc)
-        if i is not None:
-            k1[i].record(stream)
+            out = p2p.begin()
+            return out if args.op == "jvp" else (out, None)
+        R.zero_()
+        if Yd is not None:
+            Yd.zero_()
+        return R, Yd
+
+    def finish(Rc, Yc):
         if p2p is not None:
             p2p.end()
         elif halo is not None:
             halo.exchange(Rc)
-        R_last[0] = Rc
+            if Yc is not None:
+                halo.exchange(Yc)
+        R_last[0], R_last[1] = Rc, Yc
+
+    def evaluate(Uc, Rc, Yc):
+        if args.op == "jacobian":
+            ctx.jacobian(Uc, J, R=Rc)
+        elif args.op == "jac_csr":
+            ctx.jacobian_csr(Uc, vals, R=Rc)
+        elif args.op == "jvp":
+            ctx.jvp(Uc, Xd, Yc, R=Rc)
+        else:
+            ctx.viscosity_resid(Uc, R=Rc)
+
+    def step(i=None):
+        Rc, Yc = begin()
+        if vals is not None:
+            vals.zero_()
+        if i is not None:
+            k0[i].record(stream)
+        evaluate(U, Rc, Yc)
+        if i is not None:
+            k1[i].record(stream)
+        finish(Rc, Yc)
 
     for _ in range(args.warmup):
         step()
@@ -385,6 +426,7 @@ def main():
         s_d2h = torch.cuda.Stream(dev)
         Ub = [U, torch.empty_like(U)]
         Rb = [R, torch.zeros_like(R)]
+        Yb = [Yd, None if Yd is None else torch.zeros_like(Yd)]
         R_host = [torch.empty((NN, 2), dtype=torch.float64).pin_memory() for _ in range(2)]
         ev_h2d = [torch.cuda.Event() for _ in range(2)]
         ev_comp = [torch.cuda.Event() for _ in range(2)]
@@ -401,26 +443,19 @@ def main():
             if p2p is not None:
                 if t >= 1:
                     stream.wait_event(ev_d2h[(t - 1) % 2])  # begin() clears the other buffer
-                Rc = p2p.begin()
+                out = p2p.begin()
+                Rc, Yc = out if args.op == "jvp" else (out, None)
             else:
                 if t >= 2:
                     stream.wait_event(ev_d2h[b])        # R[b] of step t-2 has been downloaded
-                Rc = Rb[b]
+                Rc, Yc = Rb[b], Yb[b]
                 Rc.zero_()
+                if Yc is not None:
+                    Yc.zero_()
             if vals is not None:
                 vals.zero_()
-            if args.op == "jacobian":
-                ctx.jacobian(Ub[b], J, R=Rc)
-            elif args.op == "jac_csr":
-                ctx.jacobian_csr(Ub[b], vals, R=Rc)
-            elif args.op == "jvp":
-                ctx.jvp(Ub[b], Xd, Yd, R=Rc)
-            else:
-                ctx.viscosity_resid(Ub[b], R=Rc)
-            if p2p is not None:
-                p2p.end()
-            elif halo is not None:
-                halo.exchange(Rc)
+            evaluate(Ub[b], Rc, Yc)
+            finish(Rc, Yc)
             ev_comp[b].record(stream)
             with torch.cuda.stream(s_d2h):
                 s_d2h.wait_event(ev_comp[b])
@@ -451,28 +486,39 @@ def main():
     if args.check and world > 1:
         step()
         torch.cuda.synchronize(dev)
-        Rmine = R_last[0].cpu().numpy()
+        mine = [R_last[0].cpu().numpy()] + ([R_last[1].cpu().numpy()] if args.op == "jvp" else [])
         full = StokesFO(elem, torch.from_numpy(conn_g).to(dev), torch.from_numpy(coords_g).to(dev),
                         surface=torch.from_numpy(s_g).to(dev), flow_factor=torch.from_numpy(kc_g).to(dev),
                         geometry=args.geometry)
         Rf = torch.zeros((coords_g.shape[0], 2), dtype=torch.float64, device=dev)
-        Jf = torch.empty((conn_g.shape[0], 2 * N, 2 * N), dtype=torch.float64, device=dev)
-        full.jacobian(torch.from_numpy(U_g).to(dev), Jf, R=Rf)
+        if args.op == "jvp":
+            Yf = torch.zeros_like(Rf)
+            full.jvp(torch.from_numpy(U_g).to(dev), torch.from_numpy(x_global).to(dev), Yf, R=Rf)
+            refs = [Rf, Yf]
+        else:
+            Jf = torch.empty((conn_g.shape[0], 2 * N, 2 * N), dtype=torch.float64, device=dev)
+            full.jacobian(torch.from_numpy(U_g).to(dev), Jf, R=Rf)
+            refs = [Rf]
         full.sync()
-        Rref = Rf.cpu().numpy()[gids]
-        err = torch.tensor([float(np.abs(Rmine - Rref).max() / max(np.abs(Rref).max(), 1e-300))], dtype=torch.float64,
-                           device="cpu" if backend != "nccl" else dev)
+        e = 0.0
+        for m, r in zip(mine, refs):
+            rr = r.cpu().numpy()[gids]
+            e = max(e, float(np.abs(m - rr).max() / max(np.abs(rr).max(), 1e-300)))
+        err = torch.tensor([e], dtype=torch.float64, device="cpu" if backend != "nccl" else dev)
         dist.all_reduce(err, op=dist.ReduceOp.MAX)
         check = float(err.item())
 
     # ---- reduce over ranks (max time) ----
-    stats = torch.tensor([ms_total / args.steps, kern_ms, e2e[0] if e2e else 0.0], dtype=torch.float64, device=dev)
-    cells_all = torch.tensor([float(C)], dtype=torch.float64, device=dev)
+    mine_stats = [ms_total / args.steps, kern_ms, e2e[0] if e2e else 0.0, float(C)]
     if world > 1:
-        dist.all_reduce(stats, op=dist.ReduceOp.MAX)
-        dist.all_reduce(cells_all, op=dist.ReduceOp.SUM)
-    ms_step, kern_ms_max, e2e_ms = stats.tolist()
-    total_cells = int(cells_all.item())
+        allst = [None] * world
+        dist.all_gather_object(allst, mine_stats)
+    else:
+        allst = [mine_stats]
+    ms_step = max(a[0] for a in allst)
+    kern_ms_max = max(a[1] for a in allst)
+    e2e_ms = max(a[2] for a in allst)
+    total_cells = int(sum(a[3] for a in allst))
 
     if rank == 0:
         peak, peak_src = load_peaks()
@@ -522,10 +568,14 @@ def main():
                          "note": "live_copy_gbs: torch device-to-device copy of 2 GiB on this box before the timed "
                                  "region (context for box-to-box variance; not the denominator)"},
             "achieved_hbm_gbs": achieved,
-            "gpu_launches": args.steps * (1 + (halo.launches_per_exchange if halo else 0)),
+            "gpu_launches": args.steps * (1 + (halo.launches_per_exchange * (2 if args.op == "jvp" else 1)
+                                               if halo else 0)),
             "halo": halo_mode,
             "clocks": clk,
         }
+        if world > 1:
+            line["per_rank"] = [{"rank": r, "cells": int(a[3]), "ms_per_step": a[0], "kernel_ms": a[1]}
+                                for r, a in enumerate(allst)]
         if check is not None:
             line["halo_check_max_rel_err"] = check
         if nnz:

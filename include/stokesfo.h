@@ -109,8 +109,10 @@ int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes);
  * GradBF[c][n][q][:] = J_q^-T grad_xi phi_n(xi_q), wMeasure[c][q] = w_q det J_q
  * into the workspace (STORED mode; ON_THE_FLY mode stores node coordinates
  * instead and checks det J), plus a snapshot of conn and the flow factor.
- * Async on desc.stream; det J <= 0 or conn out of range is reported by
- * stokesfo_sync. */
+ * Synchronises desc.stream once: a conn entry outside [0, num_nodes) returns
+ * STOKESFO_EMESH here (no ctx is created), so no evaluation ever uses an
+ * out-of-range conn as an address (conn must not change while the ctx lives);
+ * det J <= 0 sets the sticky flag reported by stokesfo_sync. */
 int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out);
 
 /* Gather: U_cell[c][n][a] = U[2 conn[c][n] + a].
@@ -133,7 +135,9 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
  * Y += J(U) X with J = dR/dU assembled over all cells, computed as the forward
  * directional derivative of the fused chain along X (no element matrices are
  * formed); optionally R += R(U) in the same pass.  U, X: dev [num_nodes][2];
- * Y, R: dev [num_nodes][2] (+=). */
+ * Y, R: dev [num_nodes][2] (+=).  With a peer table attached
+ * (stokesfo_set_remote), Y is halo-summed like R and needs the peers' Y
+ * pointers (stokesfo_set_remote_jvp), else EINVAL. */
 int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, double *R);
 
 /* Basal friction side-set term (NEXT-4; P:L59 -> [24]; reading Z18):
@@ -179,7 +183,8 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R,
 /* CSR pattern over dofs (rows = 2*num_nodes; columns of a row = sorted dofs of
  * every node sharing a cell with the row's node).  Size query: pass rowptr =
  * colidx = NULL to get *nnz.  Fill: rowptr dev [2*num_nodes+1] int64, colidx
- * dev [nnz] int32.  Synchronises the stream (host-side construction). */
+ * dev [nnz] int32.  Synchronises the stream (host-side construction from a
+ * copy of conn; an entry outside [0, num_nodes) returns EMESH). */
 int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t *colidx);
 
 /* NEXT-2 per-cell CSR slots: slot[c][i][j] (uint8, j = 0..N-1, byte j of the
@@ -218,7 +223,7 @@ int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *
 
 /* Fused halo sum over peer memory: after
  * this call, the residual scatter of stokesfo_viscosity_resid / _jacobian /
- * _jvp also adds every contribution to a partition-boundary node into the R
+ * _jvp (and the R part of stokesfo_scatter_assemble) also adds every contribution to a partition-boundary node into the R
  * of each other GPU holding that node, with atomics through NVLink-mapped
  * peer pointers, so no pack / exchange / unpack is needed (one stream-ordered
  * barrier per evaluation; R passed to the calls must be the buffer the peers
@@ -227,6 +232,12 @@ int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *
  * device pointers (one per peer index; entries for this rank unused).  All
  * stay owned by the caller and must outlive their use; rem = NULL detaches. */
 int stokesfo_set_remote(stokesfo_ctx *c, const int32_t *rem, const int32_t *remtab, double *const *peers);
+/* The peers' J.v output buffers for stokesfo_jvp under the same node table:
+ * peers_y: dev array of device pointers (one per peer index), caller-owned;
+ * requires stokesfo_set_remote first (else EINVAL); NULL detaches (jvp then
+ * returns EINVAL while the table is attached).  stokesfo_set_remote(NULL)
+ * detaches both. */
+int stokesfo_set_remote_jvp(stokesfo_ctx *c, double *const *peers_y);
 /* CUDA IPC plumbing for the above (handle = 64 opaque bytes).  A handle maps
  * the whole allocation containing dev_ptr; *offset = dev_ptr - allocation
  * base, to add to the pointer the peer obtains from stokesfo_ipc_open_handle. */
@@ -257,7 +268,7 @@ int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid
  * friction removes the rigid null space; Jacobi diagonal from stokesfo_jacobian
  * and the basal face matrices), then Armijo backtracking on ||F||.  Stops when
  * ||F|| <= max(atol, rtol ||F_0||) or after max_newton steps.  Single-GPU ctx
- * (no stokesfo_set_remote).  U: dev [num_nodes][2], initial guess in, solution
+ * (a ctx with stokesfo_set_remote attached returns EINVAL).  U: dev [num_nodes][2], initial guess in, solution
  * out.  work: dev, stokesfo_newton_work_size bytes, 256-B aligned.  hist_F:
  * host [max_newton + 1] ||F|| per step; hist_cg: host [max_newton] CG
  * iterations (may be NULL); *iters = Newton steps taken. */

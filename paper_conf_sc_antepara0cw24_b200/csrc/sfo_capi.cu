@@ -31,6 +31,7 @@ struct stokesfo_ctx {
     const int32_t *rem = nullptr;     // fused halo over peer memory (stokesfo_set_remote)
     const int32_t *remtab = nullptr;
     double *const *peers = nullptr;
+    double *const *peers_y = nullptr;  // the peers' J.v outputs (stokesfo_set_remote_jvp)
     const int64_t *rowptr = nullptr;  // CSR pattern (set by stokesfo_csr_pattern)
     const int32_t *colidx = nullptr;
     int64_t csr_rows = 0;
@@ -245,6 +246,7 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.rem = c->rem;
     a.remtab = c->remtab;
     a.peers = c->peers;
+    a.peers_y = c->peers_y;
     a.rowptr = c->rowptr;
     a.slots = c->slots;
     a.csr_vals = csr_vals;
@@ -326,6 +328,16 @@ int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
         c->recs = ws + WS_HEADER;
     }
     int st = (d->elem == STOKESFO_HEX8) ? create_impl<Hex8>(c) : create_impl<Wedge6>(c);
+    // conn out of range is checked before any evaluation can use conn as an address (the on-the-fly
+    // kernels and the side-set kernels read the caller's conn): one stream synchronisation at create
+    if (st == STOKESFO_OK) {
+        int h = 0;
+        if (cudaMemcpyAsync(&h, c->err, sizeof(int), cudaMemcpyDeviceToHost, c->stream) != cudaSuccess ||
+            cudaStreamSynchronize(c->stream) != cudaSuccess)
+            st = cuda_status();
+        else if (h & ERR_CONN)
+            st = STOKESFO_EMESH;
+    }
     if (st) {
         delete c;
         return st;
@@ -436,6 +448,7 @@ int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, d
     if (c->d.num_cells == 0) return STOKESFO_OK;
     if (!U || !X || !Y || !aligned(U, 16) || !aligned(X, 16) || !aligned(Y, 16) || (R && !aligned(R, 16)))
         return STOKESFO_EINVAL;
+    if (c->rem && !c->peers_y) return STOKESFO_EINVAL;  // Y would miss the peers' boundary contributions
 #define CALL(E) eval_impl<E, M_JVP>(c, U, nullptr, nullptr, R, nullptr, X, Y)
     return DISPATCH(c, CALL);
 #undef CALL
@@ -502,8 +515,8 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
         const int64_t work = C * c->N;
         const unsigned g = (unsigned)((work + bs - 1) / bs);
         auto Rc = reinterpret_cast<const double2 *>(R_cell);
-        if (c->N == 8) scatter_r_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, Rc, R);
-        else scatter_r_kernel<6><<<g, bs, 0, c->stream>>>(C, c->d.conn, Rc, R);
+        if (c->N == 8) scatter_r_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, Rc, R, c->rem, c->remtab, c->peers);
+        else scatter_r_kernel<6><<<g, bs, 0, c->stream>>>(C, c->d.conn, Rc, R, c->rem, c->remtab, c->peers);
     }
     if (J_cell && csr_vals && C > 0) {
         if (!c->rowptr || !c->colidx) return STOKESFO_EINVAL;
@@ -582,12 +595,20 @@ int stokesfo_set_remote(stokesfo_ctx *c, const int32_t *rem, const int32_t *remt
         c->rem = nullptr;
         c->remtab = nullptr;
         c->peers = nullptr;
+        c->peers_y = nullptr;
         return STOKESFO_OK;
     }
     if (!remtab || !peers) return STOKESFO_EINVAL;
     c->rem = rem;
     c->remtab = remtab;
     c->peers = peers;
+    return STOKESFO_OK;
+}
+
+int stokesfo_set_remote_jvp(stokesfo_ctx *c, double *const *peers_y) {
+    if (!c) return STOKESFO_EINVAL;
+    if (peers_y && !c->rem) return STOKESFO_EINVAL;  // needs the node table of stokesfo_set_remote
+    c->peers_y = peers_y;
     return STOKESFO_OK;
 }
 
@@ -762,6 +783,7 @@ int stokesfo_newton_solve(stokesfo_ctx *c, const int32_t *basal_cells, int64_t n
     if (!c || !U || !work || !o || !hist_F || !iters || nbasal < 0 || (nbasal > 0 && (!basal_cells || !beta)))
         return STOKESFO_EINVAL;
     if (!aligned(U, 16) || !aligned(work, 256)) return STOKESFO_EINVAL;
+    if (c->rem) return STOKESFO_EINVAL;  // single-GPU driver: a peer table would add into other ranks' buffers
     NewtonWork w = newton_layout(c, nbasal, reinterpret_cast<char *>(work));
     const int64_t n = 2 * c->d.num_nodes;
     const size_t vb = (size_t)n * 8;
@@ -879,6 +901,9 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
         cudaMemcpyAsync(conn.data(), c->d.conn, conn.size() * 4, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess)
         return cuda_status();
     if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_status();
+    // conn is used as a host index below: range-check it first (EMESH, as the header states)
+    for (int64_t i = 0; i < C * N; ++i)
+        if (conn[i] < 0 || conn[i] >= NN) return STOKESFO_EMESH;
     // node -> cells (CSR)
     std::vector<int64_t> nc(NN + 1, 0);
     for (int64_t i = 0; i < C * N; ++i) nc[conn[i] + 1]++;

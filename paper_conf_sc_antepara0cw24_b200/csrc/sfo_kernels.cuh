@@ -263,6 +263,7 @@ struct EvalArgs {
     const int32_t *rem;
     const int32_t *remtab;
     double *const *peers;
+    double *const *peers_y;   // M_JVP: the peers' Y (required when rem is set)
     // NEXT-2 fused CSR assembly (M_CSR): J contributions go straight into
     // csr_vals[rowptr[2 g_i + a] + 2 slot[c][i][j] + b] (no element matrices)
     const int64_t *rowptr;    // [2 nodes + 1]
@@ -274,20 +275,22 @@ struct EvalArgs {
 constexpr int REM_MAX = 7;                 // remote copies of one node (<= 8 parts meet at a vertex)
 constexpr int REM_ROW = 1 + 2 * REM_MAX;
 
-// R[node] += (r0, r1) locally and, for nodes on a partition boundary, into the
-// R of every other GPU that holds the node (red.global.add.f64 through the
-// NVLink-mapped peer pointer): the halo sum happens inside the evaluation
-// kernel, no pack / exchange / unpack.
-__device__ __forceinline__ void scatter_node(const EvalArgs &a, int32_t node, double r0, double r1) {
-    red_add(a.R + 2 * (int64_t)node + 0, r0);
-    red_add(a.R + 2 * (int64_t)node + 1, r1);
-    if (a.rem) {
-        const int32_t row = __ldg(a.rem + node);
+// V[node] += (r0, r1) locally and, for nodes on a partition boundary, into the
+// V of every other GPU that holds the node (red.global.add.f64 through the
+// NVLink-mapped peer pointers `peers`): the halo sum happens inside the
+// evaluation kernel, no pack / exchange / unpack (DESIGN.md
+// "Multi-GPU").  V = R (peers) or the J.v output Y (peers_y).
+__device__ __forceinline__ void scatter_node(const int32_t *rem, const int32_t *remtab, double *V,
+                                             double *const *peers, int32_t node, double r0, double r1) {
+    red_add(V + 2 * (int64_t)node + 0, r0);
+    red_add(V + 2 * (int64_t)node + 1, r1);
+    if (rem) {
+        const int32_t row = __ldg(rem + node);
         if (row >= 0) {
-            const int32_t *t = a.remtab + (int64_t)row * REM_ROW;
+            const int32_t *t = remtab + (int64_t)row * REM_ROW;
             const int cnt = t[0];
             for (int k = 0; k < cnt; ++k) {
-                double *pr = a.peers[t[1 + 2 * k]] + 2 * (int64_t)t[2 + 2 * k];
+                double *pr = peers[t[1 + 2 * k]] + 2 * (int64_t)t[2 + 2 * k];
                 red_add(pr + 0, r0);
                 red_add(pr + 1, r1);
             }
@@ -923,12 +926,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
             }
         }
         if (act && c < nvalid) {
-            if (a.R) scatter_node(a, gnode, R0, R1);
+            if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, R0, R1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
-            if (JVP) {
-                red_add(a.Y + 2 * (int64_t)gnode + 0, dR0);
-                red_add(a.Y + 2 * (int64_t)gnode + 1, dR1);
-            }
+            if (JVP) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
         }
         if (ntile < a.ntiles) gather_store<E, MODE>(smem + nst * S::STAGE, nxt);
     }
@@ -1125,11 +1125,8 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
             if (l == 0) store_J<E>(a.J_cell, cell0, nvalid, reinterpret_cast<const char *>(rg), pol_stream);
         }
         if (act && c < nvalid) {
-            if (a.R) scatter_node(a, gnode, R0, R1);
-            if (JVP) {
-                red_add(a.Y + 2 * (int64_t)gnode + 0, dR0);
-                red_add(a.Y + 2 * (int64_t)gnode + 1, dR1);
-            }
+            if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, R0, R1);
+            if (JVP) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }
         g_cur = g_nxt; kc_cur = kc_nxt; live_cur = live_nxt;
@@ -1331,15 +1328,16 @@ __global__ void lateral_pressure_kernel(int64_t nfaces, int64_t ncells, const in
 // ---------------------------------------------------------------------------
 // G5: assembly.  R part: thread <-> (cell, node).  CSR part: thread <-> (cell, row).
 // ---------------------------------------------------------------------------
+// With a peer table attached (stokesfo_set_remote) the same fused halo sum as
+// the evaluation kernels' epilogue (scatter_node).
 template <int N>
 __global__ void scatter_r_kernel(int64_t ncells, const int32_t *__restrict__ conn, const double2 *__restrict__ Rc,
-                                 double *__restrict__ R) {
+                                 double *__restrict__ R, const int32_t *rem, const int32_t *remtab,
+                                 double *const *peers) {
     const int64_t gid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (gid >= ncells * N) return;
-    const int64_t g = conn[gid];
     const double2 v = Rc[gid];
-    red_add(R + 2 * g + 0, v.x);
-    red_add(R + 2 * g + 1, v.y);
+    scatter_node(rem, remtab, R, peers, conn[gid], v.x, v.y);
 }
 
 template <int N>

@@ -70,52 +70,64 @@ class P2PHalo:
     step is  zero(R_next) -> evaluate(R_cur) -> one stream-ordered barrier.
     R is double-buffered (step t writes R[t % 2]; R[(t+1) % 2] is zeroed before
     the barrier of step t, so no peer can write it before it is clear).
+    fields = 2 adds the J.v output Y under the same protocol (stokesfo_jvp).
 
-    Use: h = P2PHalo(ctx, part, nodes, device); for each step: R = h.begin();
-    ctx.jacobian(U, J, R=R); h.end()  (R now holds the full sum)."""
+    Use: h = P2PHalo(ctx, part, device); for each step: R = h.begin();
+    ctx.jacobian(U, J, R=R); h.end()  (R now holds the full sum).  With
+    fields = 2, begin() returns (R, Y)."""
 
-    def __init__(self, ctx, part: LocalPart, device, gloo_debug: bool = False):
+    def __init__(self, ctx, part: LocalPart, device, gloo_debug: bool = False, fields: int = 1):
         import torch
         import torch.distributed as dist
         self.ctx, self.device, self.gloo = ctx, device, gloo_debug
         self.rank, self.world = part.rank, part.world
+        self.fields = fields
         nn = part.gids.size
-        self.R = [torch.zeros((nn, 2), dtype=torch.float64, device=device) for _ in range(2)]
+        # one allocation per buffer parity holding every field: [fields][nn][2]
+        self.buf = [torch.zeros((fields, nn, 2), dtype=torch.float64, device=device) for _ in range(2)]
         rem, remtab = part.remote_table()
         self.rem = torch.from_numpy(rem).to(device)
         self.remtab = torch.from_numpy(remtab).to(device)
-        handles = [S.ipc_get_handle(R) for R in self.R]
+        handles = [S.ipc_get_handle(b) for b in self.buf]
         allh = [None] * self.world
         dist.all_gather_object(allh, handles)
+        nns = [None] * self.world      # node counts: the field stride of each peer's buffer
+        dist.all_gather_object(nns, int(nn))
         self.opened = []
         ok = 1
-        ptrs = [[0] * self.world for _ in range(2)]
+        ptrs = [[[0] * self.world for _ in range(fields)] for _ in range(2)]
         bases = {}   # one mapping per distinct peer allocation (handles may repeat)
         try:
             for b in range(2):
-                ptrs[b][self.rank] = self.R[b].data_ptr()
+                for f in range(fields):
+                    ptrs[b][f][self.rank] = self.buf[b].data_ptr() + f * nn * 16
                 for r in part.neighbors:
                     raw, off = allh[r][b]
                     if raw not in bases:
                         bases[raw] = S.ipc_open_handle((raw, 0))
                         self.opened.append(bases[raw])
-                    ptrs[b][r] = bases[raw] + off
+                    for f in range(fields):
+                        ptrs[b][f][r] = bases[raw] + off + f * nns[r] * 16
         except Exception:
             ok = 0
         flag = torch.tensor([ok], dtype=torch.int32, device="cpu" if gloo_debug else device)
         dist.all_reduce(flag, op=dist.ReduceOp.MIN)
         self.ok = bool(flag.item())
-        self.peers = [torch.tensor(ptrs[b], dtype=torch.int64, device=device) for b in range(2)]
+        self.peers = [[torch.tensor(ptrs[b][f], dtype=torch.int64, device=device) for f in range(fields)]
+                      for b in range(2)]
         self.token = torch.zeros(1, dtype=torch.float32, device=device)
         self.t = 0
-        self.launches_per_step = 0  # no pack/unpack kernels: the halo rides the evaluation kernel
+        self.launches_per_step = 1  # the buffer clear; the halo itself rides the evaluation kernel
 
     def begin(self):
-        """Returns this step's R (already zero); zeroes the next step's buffer."""
-        cur = self.R[self.t % 2]
-        self.R[(self.t + 1) % 2].zero_()
-        self.ctx.set_remote(self.rem, self.remtab, self.peers[self.t % 2])
-        return cur
+        """Returns this step's R (or (R, Y)), already zero; zeroes the next step's buffers."""
+        b = self.t % 2
+        self.buf[(self.t + 1) % 2].zero_()
+        self.ctx.set_remote(self.rem, self.remtab, self.peers[b][0])
+        if self.fields > 1:
+            self.ctx.set_remote_jvp(self.peers[b][1])
+        cur = self.buf[b]
+        return cur[0] if self.fields == 1 else tuple(cur[f] for f in range(self.fields))
 
     def end(self):
         """Stream-ordered barrier: after it, every rank's kernel of this step is complete."""
@@ -127,7 +139,8 @@ class P2PHalo:
         else:
             dist.all_reduce(self.token)
         self.t += 1
-        return self.R[(self.t - 1) % 2]
+        cur = self.buf[(self.t - 1) % 2]
+        return cur[0] if self.fields == 1 else tuple(cur[f] for f in range(self.fields))
 
     def close(self):
         self.ctx.set_remote(None, None, None)

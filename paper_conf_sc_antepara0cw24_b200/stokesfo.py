@@ -54,7 +54,7 @@ EXPORTS = [
     "stokesfo_mesh_partition_columns", "stokesfo_mesh_localize", "stokesfo_mesh_halo_list",
     "stokesfo_albany_scratch_size", "stokesfo_albany_setup", "stokesfo_albany_evaluators",
     "stokesfo_albany_resid", "stokesfo_albany_extract", "stokesfo_jvp", "stokesfo_basal_friction",
-    "stokesfo_set_remote", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
+    "stokesfo_set_remote", "stokesfo_set_remote_jvp", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
     "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
     "stokesfo_mesh_lateral_faces", "stokesfo_set_lateral", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
 ]
@@ -104,6 +104,8 @@ def _lib():
                                                 ctypes.POINTER(I32)]
         if hasattr(L, "stokesfo_set_remote"):
             L.stokesfo_set_remote.argtypes = [P, P, P, P]
+            if hasattr(L, "stokesfo_set_remote_jvp"):
+                L.stokesfo_set_remote_jvp.argtypes = [P, P]
             L.stokesfo_ipc_get_handle.argtypes = [P, P, ctypes.POINTER(I64)]
             L.stokesfo_ipc_open_handle.argtypes = [P, ctypes.POINTER(ctypes.c_void_p)]
             L.stokesfo_ipc_close.argtypes = [P]
@@ -305,6 +307,13 @@ class StokesFO:
         """Fused halo over peer memory (stokesfo_set_remote); rem=None detaches."""
         self._remote_keep = (rem, remtab, peers)
         _check(_lib().stokesfo_set_remote(self._h, _ptr(rem), _ptr(remtab), _ptr(peers)), "set_remote")
+        if rem is None:
+            self._remote_y_keep = None
+
+    def set_remote_jvp(self, peers_y):
+        """The peers' J.v outputs for jvp under the attached node table (stokesfo_set_remote_jvp)."""
+        self._remote_y_keep = peers_y
+        _check(_lib().stokesfo_set_remote_jvp(self._h, _ptr(peers_y)), "set_remote_jvp")
 
     def csr_pattern(self):
         import torch

@@ -61,3 +61,25 @@ def interior_nodes(fp, L, conn_nodes_count):
         for k in range(1, L):
             ids.append(v * (L + 1) + k)
     return np.array(ids, dtype=np.int64)
+
+
+def rounding_scale_R(e, conn, G, wm, mu, U, s, rho_g):
+    """A-priori rounding scale of R_cell[c][i][a] = sum_q wM_q (sigma_a(q) . G_i(q)
+    + f_a(q) phi_i(q)): the sum of the absolute values of the terms that are added,
+    with every Ugrad entry bounded by gbar_q = sum_n sum_a sum_d |U_n,a| |G_n[q][d]|
+    (its value before cancellation) and |beta| <= 3 gbar:
+        scale = sum_q wM_q (2 mu_q 3 gbar_q sum_d |G_i[q][d]|
+                            + rho_g (sum_n |s_n| (|G_n0| + |G_n1|)) phi_i(q)).
+    Two correct fp64 evaluations differ by O(eps) of it: on thin, wide cells (C4p:
+    1 m x 16 km) the Ugrad sums cancel by up to 1e6 and the oracle itself moves by
+    1e-11 of sum |R_cell| under a translation of the coordinates."""
+    bf, _, _ = O.ref_element(e)               # [N][Q]
+    Uc = np.abs(U[conn])                      # [C][N][2]
+    aG = np.abs(G)                            # [C][N][Q][3]
+    gbar = np.einsum("cna,cnqd->cq", Uc, aG)  # [C][Q]
+    Gi = aG.sum(-1)                           # [C][N][Q]
+    sc = np.einsum("cq,cnq->cn", wm * 2.0 * mu * 3.0 * gbar, Gi)
+    if s is not None:
+        fs = rho_g * np.einsum("cn,cnq->cq", np.abs(s[conn]), aG[..., 0] + aG[..., 1])
+        sc = sc + np.einsum("cq,nq->cn", wm * fs, bf)
+    return np.repeat(sc[:, :, None], 2, axis=2)

@@ -268,12 +268,37 @@ def test_edge_cases_and_errors(torch, geometry):
     ctxb = StokesFO("hex8", _t(torch, bad), _t(torch, coords), geometry=geometry)
     with pytest.raises(StokesFOError, match="EMESH"):
         ctxb.sync()
-    # conn out of range -> EMESH
-    bad2 = conn.copy()
-    bad2[1, 3] = coords.shape[0] + 5
-    ctxc = StokesFO("hex8", _t(torch, bad2), _t(torch, coords), geometry=geometry)
+    # conn out of range (past the end, or negative) -> EMESH from create itself: no ctx
+    # exists that could use it as an address (on-the-fly and side-set kernels)
+    for v in (coords.shape[0] + 5, -1):
+        bad2 = conn.copy()
+        bad2[1, 3] = v
+        with pytest.raises(StokesFOError, match="EMESH"):
+            StokesFO("hex8", _t(torch, bad2), _t(torch, coords), geometry=geometry)
+    # csr_pattern range-checks conn on the host before indexing with it (a caller
+    # that corrupts conn after create gets EMESH, not a heap overwrite)
+    connd = _t(torch, conn)
+    ctxd = StokesFO("hex8", connd, _t(torch, coords), geometry=geometry)
+    ctxd.sync()
+    connd[0, 0] = coords.shape[0] + 1
     with pytest.raises(StokesFOError, match="EMESH"):
-        ctxc.sync()
+        ctxd.csr_pattern()
+    # a peer table without the peers' Y -> jvp refuses (Y would miss boundary
+    # contributions); the single-GPU Newton driver refuses any peer table
+    nn = coords.shape[0]
+    rem = torch.full((nn,), -1, dtype=torch.int32, device="cuda")
+    remtab = torch.zeros((1, 15), dtype=torch.int32, device="cuda")
+    peers = torch.zeros(2, dtype=torch.int64, device="cuda")
+    ctx1.set_remote(rem, remtab, peers)
+    Z = torch.zeros((nn, 2), dtype=torch.float64, device="cuda")
+    with pytest.raises(StokesFOError, match="EINVAL"):
+        ctx1.jvp(Z, Z, Z.clone())
+    with pytest.raises(StokesFOError, match="EINVAL"):
+        ctx1.newton_solve(None, None, Z.clone(), max_newton=1)
+    ctx1.set_remote_jvp(peers)
+    ctx1.jvp(Z, Z, Z.clone())
+    ctx1.set_remote(None, None, None)
+    ctx1.sync()
     # misaligned output pointer -> EINVAL
     big = torch.empty(2 * 16 * 16 + 1, dtype=torch.float64, device="cuda")
     lib = __import__("paper_conf_sc_antepara0cw24_b200.stokesfo", fromlist=["_lib"])._lib()

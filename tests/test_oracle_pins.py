@@ -398,6 +398,30 @@ def test_extrusion_counts_and_numbering():
     assert coords[v * (L + 1) + L, 2] == fp.b[v] + fp.H[v]  # surface node: z = b + H exactly
 
 
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_gather_node_id_probe(elem):
+    """O-gather (eq. (3): the element sees U at its own nodes, interleaved dof
+    2 node + comp, reading Z9): with the probe field U[v] = (v, -v - 1/2) the
+    gathered block must be exactly (conn, -conn - 1/2) -- integers and halves are
+    exact in fp64, so any wrong index, swapped component or node-order slip in
+    the oracle's gather shows up as a bit difference.  A ragged subset of cells
+    (every 7th, reversed) pins that gather is per cell, not a prefix copy."""
+    e = O.ELEM[elem]
+    fp, conn, coords = M.tiny(elem)
+    nn = coords.shape[0]
+    v = np.arange(nn, dtype=np.float64)
+    U = np.stack([v, -v - 0.5], 1)
+    got = O.gather(e, conn, U)
+    assert got.shape == (conn.shape[0], O.NODES[e], 2)
+    assert np.array_equal(got[..., 0], conn.astype(np.float64))
+    assert np.array_equal(got[..., 1], -conn.astype(np.float64) - 0.5)
+    sub = np.ascontiguousarray(conn[::-7])
+    got2 = O.gather(e, sub, U)
+    assert np.array_equal(got2[..., 0], sub.astype(np.float64))
+    # empty mesh: nothing gathered
+    assert O.gather(e, conn[:0], U).shape == (0, O.NODES[e], 2)
+
+
 def test_scatter_valence_probe():
     fp, conn, coords = M.tiny("hex8")
     R = O.scatter(HEX, conn, np.ones((conn.shape[0], 8, 2)), coords.shape[0])
