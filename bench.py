@@ -60,6 +60,35 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
     return cells * per_cell + nodes * (16 + 8 + 32 + xy) + vals
 
 
+MESH_SIZES = {"C4": (8431650, 9313304), "C5": (16863300, 9313304), "C3": (2033100, 2274459),
+              "C4p": (1053660, 1124697), "C1": (1280, 1734)}
+
+
+def units_per_launch(key: str) -> int:
+    """Tiles of one evaluation launch for a traffic key 'CFG:elem:op:geometry'
+    (hex8 4 cells per tile, wedge6 5): the unit of the per-tile ncu breakdowns."""
+    cfg, elem = key.split(":")[:2]
+    tc = 4 if elem == "hex8" else 5
+    return (MESH_SIZES[cfg][0] + tc - 1) // tc
+
+
+def lookup_traffic(config: str, elem: str, op: str, geometry: str, world: int):
+    """(dram bytes per launch, source) from profiles/traffic.json when an ncu
+    capture of THIS build's kernel exists (entries are keyed by workload and
+    carry the source revision they were measured with), else (None, why)."""
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    key = f"{config}:{elem}:{op}:{geometry}"
+    if world != 1 or os.environ.get("STOKESFO_LIB") or not os.path.exists(tpath):
+        return None, "no ncu capture for this launch configuration"
+    from paper_conf_sc_antepara0cw24_b200 import build as B
+    with open(tpath) as f:
+        tr = json.load(f)
+    e = tr.get(key)
+    if e is None or e.get("rev") != B.source_rev():
+        return None, "no ncu capture of this build (profiles/traffic.json is keyed by source revision)"
+    return e["dram_bytes_per_launch"], f"profiles/{e['tag']}_ncu_summary.md (ncu --set full, rev {e['rev']})"
+
+
 def load_peaks():
     path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(path):
@@ -524,14 +553,7 @@ def main():
         peak, peak_src = load_peaks()
         bpl = bytes_per_launch(elem, C, NN, args.geometry, args.op, nnz)
         achieved = bpl / (kern_ms_max * 1e-3) / 1e9
-        traffic = None
-        tpath = os.path.join(ROOT, "profiles", "traffic.json")
-        if os.path.exists(tpath):
-            with open(tpath) as f:
-                tr = json.load(f)
-            key = f"{args.config}:{elem}:{args.op}:{args.geometry}"
-            if key in tr and world == 1:
-                traffic = tr[key]["dram_bytes_per_launch"]
+        traffic, traffic_src = lookup_traffic(args.config, elem, args.op, args.geometry, world)
         l2_bytes = 126 * 2 ** 20
         line = {
             "metric": {"jacobian": METRIC,
@@ -557,7 +579,7 @@ def main():
                        else "inputs fit in L2 (not flushed; small-config line)",
                        "launch": ctx.launch_info()},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic,
+                         "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
                          "kernel": ("eval_otf_kernel" if args.geometry == "on_the_fly" else "eval_kernel")
                          + ("<Hex8," if elem == "hex8" else "<Wedge6,")
                          + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>"}[args.op]

@@ -43,6 +43,23 @@ def raw_metrics(rep):
     return res
 
 
+UNIT = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
+        "KB": 1e3, "MB": 1e6, "GB": 1e9, "KiB": 1024.0, "MiB": 1024.0 ** 2, "GiB": 1024.0 ** 3}
+
+
+def to_bytes(value: str, unit: str) -> float:
+    """One ncu raw-page value in bytes, with ITS OWN unit (ncu scales every
+    metric independently: reads may print in Gbyte while writes print in Mbyte)."""
+    if unit not in UNIT:
+        raise ValueError(f"unknown byte unit {unit!r}")
+    return float(value.replace(",", "")) * UNIT[unit]
+
+
+def dram_bytes(d) -> float:
+    """dram__bytes_read.sum + dram__bytes_write.sum of one kernel row, in bytes."""
+    return to_bytes(*d["dram__bytes_read.sum"]) + to_bytes(*d["dram__bytes_write.sum"])
+
+
 def stall_summary(rep):
     rows = ncu_csv(["-i", rep, "--page", "source", "--csv", "--print-source", "sass"])
     if len(rows) < 3:
@@ -84,7 +101,15 @@ def main():
     ap.add_argument("--launches")
     ap.add_argument("--key", default="C4:hex8:jacobian:stored")
     ap.add_argument("--note", default="")
+    ap.add_argument("--rev", default=None,
+                    help="source revision the capture was made with (build.source_rev() of that build); "
+                         "default: the current tree's")
     a = ap.parse_args()
+    if a.rev is None:
+        import sys
+        sys.path.insert(0, ROOT)
+        from paper_conf_sc_antepara0cw24_b200 import build as B
+        a.rev = B.source_rev()
     prof = os.path.join(ROOT, "profiles")
     os.makedirs(prof, exist_ok=True)
     md = [f"# ncu summary {a.tag} ({a.key})", "", a.note, ""]
@@ -106,15 +131,11 @@ def main():
             for m in METRICS:
                 if m in d:
                     md.append(f"| {m} | {d[m][0]} | {d[m][1]} |")
-            rd = float(d["dram__bytes_read.sum"][0].replace(",", ""))
-            wr = float(d["dram__bytes_write.sum"][0].replace(",", ""))
-            unit = d["dram__bytes_read.sum"][1]
-            mult = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
-            traffic = (rd + wr) * mult
+            traffic = dram_bytes(d)
             md += ["", f"DRAM traffic per launch: {traffic:.4e} B", ""]
             tp = os.path.join(prof, "traffic.json")
             tr = json.load(open(tp)) if os.path.exists(tp) else {}
-            tr[a.key] = {"dram_bytes_per_launch": traffic, "tag": a.tag,
+            tr[a.key] = {"dram_bytes_per_launch": traffic, "tag": a.tag, "rev": a.rev,
                          "kernel": d.get("Kernel Name", ("?", ""))[0][:100]}
             json.dump(tr, open(tp, "w"), indent=1)
         st = stall_summary(a.rep)

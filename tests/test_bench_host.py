@@ -48,3 +48,48 @@ def test_clock_window_shorter_than_period_takes_next_sample():
     rows = [(now + 0.1 * k, 1965 - 100 * k, 300 + k, False) for k in range(5)]
     out = _sampler(rows, now + 0.15, now + 0.16).stop()
     assert out["samples"] == 1 and out["sm_mhz"] == 1765
+
+
+def test_ncu_byte_units_are_per_metric():
+    """ncu prints every metric in its own unit: a Gbyte read plus a Mbyte write
+    (profiles/r49_jvp: 14.76 Gbyte + 338.40 Mbyte) is 15.10e9 B, not 353e9 B
+    (the r1 bug: the read's unit applied to both)."""
+    import importlib.util
+    import os
+    spec = importlib.util.spec_from_file_location(
+        "ncu_summary", os.path.join(os.path.dirname(bench.__file__), "scripts", "ncu_summary.py"))
+    ns = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(ns)
+    d = {"dram__bytes_read.sum": ("14.76", "Gbyte"), "dram__bytes_write.sum": ("338.40", "Mbyte")}
+    assert abs(ns.dram_bytes(d) - 15.0984e9) < 1e3
+    d = {"dram__bytes_read.sum": ("1,234.5", "Kbyte"), "dram__bytes_write.sum": ("7", "byte")}
+    assert ns.dram_bytes(d) == 1234500.0 + 7.0
+    import pytest
+    with pytest.raises(ValueError):
+        ns.to_bytes("1", "furlong")
+
+
+def test_traffic_entries_are_keyed_to_this_build_and_plausible():
+    """profiles/traffic.json: bench.py reports an entry only when its source
+    revision is this build's; every entry of this build is within [0.95, 1.10] of
+    the algorithmic bytes of its launch (DESIGN §6 byte model), so a unit slip or a
+    stale capture cannot reach a bench line."""
+    import json
+    import os
+    from paper_conf_sc_antepara0cw24_b200 import build as B
+    sizes = bench.MESH_SIZES
+    tp = os.path.join(os.path.dirname(bench.__file__), "profiles", "traffic.json")
+    tr = json.load(open(tp))
+    rev = B.source_rev()
+    for key, e in tr.items():
+        assert "rev" in e and "tag" in e, key
+        cfg, elem, op, geo = key.split(":")
+        if e["rev"] != rev or op not in ("jacobian", "resid", "jvp") or cfg not in sizes:
+            continue
+        cells, nodes = sizes[cfg]
+        algo = bench.bytes_per_launch(elem, cells, nodes, geo, op)
+        assert 0.95 <= e["dram_bytes_per_launch"] / algo <= 1.10, (key, e["dram_bytes_per_launch"] / algo)
+        got, src = bench.lookup_traffic(cfg, elem, op, geo, 1)
+        assert got == e["dram_bytes_per_launch"] and e["tag"] in src
+    # a stale or foreign entry is never reported
+    assert bench.lookup_traffic("C4", "hex8", "jacobian", "stored", 2)[0] is None
