@@ -939,45 +939,81 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
 // Same evaluation; GradBF and wM are recomputed per tile from the gathered
 // node coordinates (cell-local, reading Z17) instead of being streamed: 40
 // streamed B/cell instead of 1,640 (hex8).  conn and k_c are read straight
-// from the caller's arrays one tile ahead; U, s and coordinates are gathered
-// with cp.async one tile ahead.
+// from the caller's arrays two tiles ahead; U, s and the node coordinates are
+// gathered into registers one tile ahead (at the middle of the previous tile's
+// node phase) and stored to shared memory after it, already cell-local
+// (x_n - x_0 with x_0 from the cell's node-0 lane by shuffle): one conflict-free
+// shared store per value instead of a cp.async gather, which costs one
+// shared-memory wavefront per lane (ncu r2 p1: 32 per LDGSTS.128 vs 4 ideal).
+// The reference gradients at the lane's QP are evaluated in registers from
+// its QP coordinates (no shared table).
 
 template <class E, int MODE>
 struct OtfSmem {
     static constexpr int N = E::N, Q = E::Q, TC = E::TC, SLAB = E::SLAB;
-    static constexpr int UP = E::UPITCH;
-    static constexpr int IN_U = 0, IN_XY = TC * UP * 16, IN_ZW = 2 * TC * UP * 16, IN_X = 3 * TC * UP * 16;
-    static constexpr int IN_S = IN_X + (MODE == M_JVP ? TC * UP * 16 : 0);
-    static constexpr int IN_BYTES = (int)round_up(IN_S + TC * UP * 8, 128);  // one gathered-input buffer
-    static constexpr int DPITCH = 3 * N + 1;                                 // odd pitch: conflict-free
-    static constexpr int OFF_DPHI = 2 * IN_BYTES;                            // double [Q][DPITCH]
-    static constexpr int OFF_G = (int)round_up(OFF_DPHI + Q * DPITCH * 8, 128);  // GradBF [Q][3][SLAB]
+    // gathered-input cell pitch: hex8 9 (the 4 cells' broadcast 16-B reads fall in distinct banks)
+    static constexpr int UP = E::N == 8 ? 9 : E::UPITCH;
+    static constexpr int IN_U = 0;                        // double2 [TC][UP]  U
+    static constexpr int IN_XY = TC * UP * 16;            // double2 [TC][UP]  cell-local (x, y)
+    static constexpr int IN_Z = 2 * TC * UP * 16;         // double  [TC][UP]  cell-local z
+    static constexpr int IN_S = IN_Z + TC * UP * 8;       // double  [TC][UP]  s
+    static constexpr int IN_X = (int)round_up(IN_S + TC * UP * 8, 16);  // double2 [TC][UP] X (M_JVP)
+    static constexpr int IN_BYTES = (int)round_up(IN_X + (MODE == M_JVP ? TC * UP * 16 : 0), 128);
+    static constexpr int OFF_G = 2 * IN_BYTES;                               // GradBF [Q][3][SLAB]
     static constexpr int OFF_QS = OFF_G + Q * 3 * SLAB * 8;                  // double [NQS][TC][Q]
     static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;   // J staging overlays G + qs
     static_assert(J_BYTES <= OFF_QS + nqs<MODE>() * TC * Q * 8 - OFF_G, "J staging must fit over G + qs");
     static constexpr int BYTES = OFF_QS + nqs<MODE>() * TC * Q * 8;
-    static_assert(IN_X % 16 == 0 && IN_BYTES % 128 == 0 && OFF_G % 128 == 0 && OFF_QS % 16 == 0, "alignment");
+    static_assert(IN_XY % 16 == 0 && IN_X % 16 == 0 && IN_BYTES % 128 == 0 && OFF_G % 128 == 0 && OFF_QS % 16 == 0,
+                  "alignment");
 };
 
-template <class E, int MODE>
-__device__ __forceinline__ void issue_gather_otf(char *in, int32_t g, bool live, const double *U,
-                                                 const double4 *xyz4, const double *surface, bool have_s,
-                                                 const double *X) {
-    using S = OtfSmem<E, MODE>;
-    const int l = threadIdx.x;
+struct OtfGathered {
+    double2 u, xy, x;
+    double z, s;
+};
+
+// lane (cell, node) loads its node's inputs into registers (zeros for dead lanes)
+template <int MODE>
+__device__ __forceinline__ OtfGathered otf_load(int32_t g, bool live, const double *U, const double4 *xyz4,
+                                                const double *surface, bool have_s, const double *X) {
+    OtfGathered v{make_double2(0.0, 0.0), make_double2(0.0, 0.0), make_double2(0.0, 0.0), 0.0, 0.0};
     if (live) {
-        const int e = E::lane_cell(l) * E::UPITCH + E::lane_sub(l);  // [cell][node]
-        cp_async16(in + S::IN_U + e * 16, U + 2 * (int64_t)g);
-        cp_async16(in + S::IN_XY + e * 16, reinterpret_cast<const double *>(xyz4 + g));
-        cp_async16(in + S::IN_ZW + e * 16, reinterpret_cast<const double *>(xyz4 + g) + 2);
-        if (have_s) cp_async8(in + S::IN_S + e * 8, surface + g);
-        if (MODE == M_JVP) cp_async16(in + S::IN_X + e * 16, X + 2 * (int64_t)g);
+        v.u = __ldg(reinterpret_cast<const double2 *>(U) + g);
+        const double *p = reinterpret_cast<const double *>(xyz4 + g);
+        v.xy = __ldg(reinterpret_cast<const double2 *>(p));
+        v.z = __ldg(p + 2);
+        if (have_s) v.s = __ldg(surface + g);
+        if (MODE == M_JVP) v.x = __ldg(reinterpret_cast<const double2 *>(X) + g);
     }
-    cp_async_commit();
+    return v;
 }
 
+// store one tile's gathered inputs, coordinates made cell-local (reading Z17);
+// every lane of the warp must call this (shuffles)
 template <class E, int MODE>
-__global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_kernel(EvalArgs a) {
+__device__ __forceinline__ void otf_store(char *in, const OtfGathered &v, int c, int n, bool act) {
+    using S = OtfSmem<E, MODE>;
+    const int src = act ? E::lane_of(c, 0) : (int)(threadIdx.x & 31);
+    const double x0 = __shfl_sync(0xffffffffu, v.xy.x, src);
+    const double y0 = __shfl_sync(0xffffffffu, v.xy.y, src);
+    const double z0 = __shfl_sync(0xffffffffu, v.z, src);
+    if (act) {
+        const int e = c * S::UP + n;
+        reinterpret_cast<double2 *>(in + S::IN_U)[e] = v.u;
+        reinterpret_cast<double2 *>(in + S::IN_XY)[e] = make_double2(v.xy.x - x0, v.xy.y - y0);
+        reinterpret_cast<double *>(in + S::IN_Z)[e] = v.z - z0;
+        reinterpret_cast<double *>(in + S::IN_S)[e] = v.s;
+        if (MODE == M_JVP) reinterpret_cast<double2 *>(in + S::IN_X)[e] = v.x;
+    }
+}
+
+// resident one-warp CTAs per SM the on-the-fly kernels' register budget is sized for
+#ifndef SFO_OTF_JAC_WARPS
+#define SFO_OTF_JAC_WARPS 12
+#endif
+template <class E, int MODE>
+__global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_OTF_JAC_WARPS : 16)) eval_otf_kernel(EvalArgs a) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N == Q, "lane mappings assume N == Q");
     constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
@@ -985,7 +1021,6 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
     extern __shared__ __align__(128) char smem[];
     double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
     const QsView<E, nqs<MODE>()> qs{reinterpret_cast<double *>(smem + S::OFF_QS), nullptr};
-    double *dphi = reinterpret_cast<double *>(smem + S::OFF_DPHI);
     const int l = threadIdx.x;
     const bool act = l < TC * N;
     const int c = act ? E::lane_cell(l) : TC, s = act ? E::lane_sub(l) : 0;
@@ -993,19 +1028,9 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
     uint64_t pol_stream = 0;
     if (l == 0) pol_stream = policy_evict_first();
 
-    // reference gradients d phi_n / d xi at every QP (shared table)
-    for (int e = l; e < Q * N; e += 32) {
-        const int q = e / N, n = e % N;
-        double x, y, z, w, phi;
-        qp_coords<E>(q, x, y, z, w);
-        basis<E>(n, x, y, z, phi, dphi[q * S::DPITCH + n * 3 + 0], dphi[q * S::DPITCH + n * 3 + 1],
-                 dphi[q * S::DPITCH + n * 3 + 2]);
-    }
-    double wq;
-    {
-        double x, y, z;
-        qp_coords<E>(act ? s : 0, x, y, z, wq);
-    }
+    // this lane's QP (per-QP phase) and phi_i at every QP (node phase)
+    double xq, yq, zq, wq;
+    qp_coords<E>(act ? s : 0, xq, yq, zq, wq);
     double bfi[Q];
     basis_row<E>(act ? s : 0, bfi);
 
@@ -1021,42 +1046,43 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
     bool live_cur, live_nxt;
     load_tile(blockIdx.x, g_cur, kc_cur, live_cur);
     load_tile(blockIdx.x + (int64_t)gridDim.x, g_nxt, kc_nxt, live_nxt);
-    __syncwarp();
     if ((int64_t)blockIdx.x < a.ntiles)
-        issue_gather_otf<E, MODE>(smem, g_cur, live_cur, a.U, a.xyz4, a.surface, have_s, a.X);
+        otf_store<E, MODE>(smem, otf_load<MODE>(g_cur, live_cur, a.U, a.xyz4, a.surface, have_s, a.X), c, s, act);
 
     int it = 0;
     for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
         const char *in = smem + (it & 1) * S::IN_BYTES;
         const double2 *Us = reinterpret_cast<const double2 *>(in + S::IN_U);
         const double2 *XY = reinterpret_cast<const double2 *>(in + S::IN_XY);
-        const double2 *ZW = reinterpret_cast<const double2 *>(in + S::IN_ZW);
+        const double *Zs = reinterpret_cast<const double *>(in + S::IN_Z);
         const double *ss = reinterpret_cast<const double *>(in + S::IN_S);
         const double2 *Xs = reinterpret_cast<const double2 *>(in + S::IN_X);
         const int64_t cell0 = tile * TC;
         const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
 
-        cp_async_wait_all();
         if (JAC && l == 0) bulk_wait_read0();  // previous tile's J staging (over G + qs) has been read
-        __syncwarp();
+        __syncwarp();                          // + this tile's gathered inputs are visible
 
         // ---- per-QP phase: geometry, GradBF -> smem, then Ugrad etc. ----
         // every lane of cell c loaded its k_c; take it from the cell's node-0 lane
         const double kc = __shfl_sync(0xffffffffu, kc_cur, act ? E::lane_of(c, 0) : 0);
         if (act) {
             const int q = s;
-            const double *dq = dphi + q * S::DPITCH;
-            double J00 = 0, J01 = 0, J02 = 0, J10 = 0, J11 = 0, J12 = 0, J20 = 0, J21 = 0, J22 = 0;
-            const double2 xy0 = XY[c * E::UPITCH];
-            const double z0 = ZW[c * E::UPITCH].x;
+            // reference gradients d phi_n / d xi at this lane's QP, in registers
+            double dq[N][3];
 #pragma unroll
             for (int n = 0; n < N; ++n) {
-                const double2 xy = XY[c * E::UPITCH + n];
-                const double x = xy.x - xy0.x, y = xy.y - xy0.y;  // cell-local (reading Z17)
-                const double z = ZW[c * E::UPITCH + n].x - z0;
-                const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
-                J00 = fma(x, d0, J00); J01 = fma(x, d1, J01); J02 = fma(x, d2, J02);
-                J10 = fma(y, d0, J10); J11 = fma(y, d1, J11); J12 = fma(y, d2, J12);
+                double phi;
+                basis<E>(n, xq, yq, zq, phi, dq[n][0], dq[n][1], dq[n][2]);
+            }
+            double J00 = 0, J01 = 0, J02 = 0, J10 = 0, J11 = 0, J12 = 0, J20 = 0, J21 = 0, J22 = 0;
+#pragma unroll
+            for (int n = 1; n < N; ++n) {  // cell-local: node 0 sits at the origin
+                const double2 xy = XY[c * S::UP + n];
+                const double z = Zs[c * S::UP + n];
+                const double d0 = dq[n][0], d1 = dq[n][1], d2 = dq[n][2];
+                J00 = fma(xy.x, d0, J00); J01 = fma(xy.x, d1, J01); J02 = fma(xy.x, d2, J02);
+                J10 = fma(xy.y, d0, J10); J11 = fma(xy.y, d1, J11); J12 = fma(xy.y, d2, J12);
                 J20 = fma(z, d0, J20); J21 = fma(z, d1, J21); J22 = fma(z, d2, J22);
             }
             // cofactors: (J^-T)[r][s] = cof[r][s] / det
@@ -1070,22 +1096,22 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
             double dg[6] = {0, 0, 0, 0, 0, 0};
 #pragma unroll
             for (int n = 0; n < N; ++n) {
-                const double d0 = dq[n * 3 + 0], d1 = dq[n * 3 + 1], d2 = dq[n * 3 + 2];
+                const double d0 = dq[n][0], d1 = dq[n][1], d2 = dq[n][2];
                 const double g0 = fma(c00, d0, fma(c01, d1, c02 * d2)) * id;
                 const double g1 = fma(c10, d0, fma(c11, d1, c12 * d2)) * id;
                 const double g2 = fma(c20, d0, fma(c21, d1, c22 * d2)) * id;
                 rg[gidx<E>(n, q, 0, c)] = g0;
                 rg[gidx<E>(n, q, 1, c)] = g1;
                 rg[gidx<E>(n, q, 2, c)] = g2;
-                const double2 uv = Us[c * E::UPITCH + n];
+                const double2 uv = Us[c * S::UP + n];
                 ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
                 vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
                 if (have_s) {
-                    const double sn = ss[c * E::UPITCH + n];
+                    const double sn = ss[c * S::UP + n];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
                 if (JVP) {
-                    const double2 xv = Xs[c * E::UPITCH + n];
+                    const double2 xv = Xs[c * S::UP + n];
                     dg[0] = fma(xv.x, g0, dg[0]); dg[1] = fma(xv.x, g1, dg[1]); dg[2] = fma(xv.x, g2, dg[2]);
                     dg[3] = fma(xv.y, g0, dg[3]); dg[4] = fma(xv.y, g1, dg[4]); dg[5] = fma(xv.y, g2, dg[5]);
                 }
@@ -1095,16 +1121,15 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
         }
         __syncwarp();
 
-        // ---- per-node phase (+ gather of the next tile, load of the one after) ----
+        // ---- per-node phase (+ register gather of the next tile, conn of the one after) ----
         const int32_t gnode = g_cur;
         int32_t g_nn = 0;
         double kc_nn = 0.0;
         bool live_nn = false;
+        OtfGathered nxt{make_double2(0.0, 0.0), make_double2(0.0, 0.0), make_double2(0.0, 0.0), 0.0, 0.0};
         auto prefetch = [&]() {
-            const int64_t nt = tile + gridDim.x;
-            if (nt < a.ntiles)
-                issue_gather_otf<E, MODE>(smem + ((it + 1) & 1) * S::IN_BYTES, g_nxt, live_nxt, a.U, a.xyz4,
-                                          a.surface, have_s, a.X);
+            if (tile + gridDim.x < a.ntiles)
+                nxt = otf_load<MODE>(g_nxt, live_nxt, a.U, a.xyz4, a.surface, have_s, a.X);
             load_tile(tile + 2 * (int64_t)gridDim.x, g_nn, kc_nn, live_nn);
         };
         double R0 = 0.0, R1 = 0.0, dR0 = 0.0, dR1 = 0.0;
@@ -1129,6 +1154,8 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? 12 : 16)) eval_otf_ke
             if (JVP) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }
+        // the other input buffer was last read in the previous tile's per-QP phase
+        if (tile + gridDim.x < a.ntiles) otf_store<E, MODE>(smem + ((it + 1) & 1) * S::IN_BYTES, nxt, c, s, act);
         g_cur = g_nxt; kc_cur = kc_nxt; live_cur = live_nxt;
         g_nxt = g_nn; kc_nxt = kc_nn; live_nxt = live_nn;
     }
