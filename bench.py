@@ -53,7 +53,12 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
         # rowptr pair 16, and every CSR value read + written once (16 nnz)
         J = 8 * N
         xy = 16
-    vals = 16 * nnz if op == "jac_csr" else 0
+    if op == "jac_global":
+        # jacobian (J_cell written) + pull assembly (DESIGN §6 NEXT-2): J_cell read again, per cell the
+        # slot row 8N and incidence 4N, per node rowptr pair 16 + incidence pointer 8, CSR values read + written
+        J = 2 * 8 * (2 * N) ** 2 + 8 * N + 4 * N
+        xy = 24
+    vals = 16 * nnz if op in ("jac_csr", "jac_global") else 0
     if geometry == "on_the_fly":
         return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32 + xy) + vals
     per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + J
@@ -169,10 +174,19 @@ def dist_env():
     return rank, world, local
 
 
-def build_mesh(cfg: str):
-    from paper_conf_sc_antepara0cw24_b200 import mesh_extrude, synth
+def build_mesh(cfg: str, oracle_side: bool = False):
+    """Seeded synthetic mesh + fields of a config.  The GPU arm extrudes with the
+    product's C ABI (stokesfo_mesh_extrude); the oracle arm (--impl reference)
+    with the oracle's own extrusion (bit-exact equal, tests/test_abi_mesh.py), so
+    that arm loads nothing from the product."""
+    from paper_conf_sc_antepara0cw24_b200 import synth
     fp, L, elem = synth.make_config(cfg)
-    conn, coords = mesh_extrude(fp.xy, fp.polys, fp.b, fp.H, L)
+    if oracle_side:
+        import oracle as O
+        conn, coords = O.extrude(fp.xy, fp.polys, fp.b, fp.H, L)
+    else:
+        from paper_conf_sc_antepara0cw24_b200 import mesh_extrude
+        conn, coords = mesh_extrude(fp.xy, fp.polys, fp.b, fp.H, L)
     U = synth.velocity_balance(fp, L, seed=11 if cfg == "C3" else 12)
     s = synth.surface_nodal(fp, L)
     kc = synth.flow_factor(fp, L)
@@ -182,6 +196,18 @@ def build_mesh(cfg: str):
 # ---------------------------------------------------------------------------
 # CPU oracle leg (cpu_baseline and --impl reference)
 # ---------------------------------------------------------------------------
+
+def host_cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
 
 def oracle_sample_rate(elem, conn, coords, U, s, kc, target_s=12.0, start_cell=0, mode="jac"):
     """Time the oracle (as it stands) on a bounded contiguous sample of cells;
@@ -210,7 +236,7 @@ def run_reference(args, rank, world):
         return 0
     import oracle as O
     cfg = args.config
-    fp, L, elem, conn, coords, U, s, kc = build_mesh(cfg)
+    fp, L, elem, conn, coords, U, s, kc = build_mesh(cfg, oracle_side=True)
     import numpy as np
     e = O.ELEM[elem]
     # calibrate a per-step sample so that warmup + steps end within a few minutes
@@ -232,7 +258,7 @@ def run_reference(args, rank, world):
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": WORKLOADS[cfg], "cells": int(conn.shape[0]), "sampled_cells_per_step": n},
         "cpu_baseline": {"value": value, "unit": "cells/s", "cores": O.num_threads(), "kind": "oracle",
-                         "sample": sample},
+                         "sample": sample, "host_cpu": host_cpu_model()},
         "e2e": {"value": value, "unit": "cells/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
         "gpu_launches": 0,
     }
@@ -272,7 +298,7 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly"])
-    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jac_csr"],
+    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jac_csr", "jac_global"],
                     help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
                          "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
     ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
@@ -282,6 +308,9 @@ def main():
                     help="N>1: compare every rank's halo-summed R with a one-GPU evaluation of the whole mesh")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--sustain", type=float, default=2.0,
+                    help="seconds of back-to-back steps after the timed region (0 = off): the 'sustained' "
+                         "sub-object, i.e. the throughput once the board's power controller has settled")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
@@ -324,14 +353,18 @@ def main():
     N = conn.shape[1]
     stream = torch.cuda.current_stream(dev)
     ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream, geometry=args.geometry)
-    J = torch.empty((C, 2 * N, 2 * N) if args.op == "jacobian" else (0,), dtype=torch.float64, device=dev)
+    if world > 1 and args.op in ("jac_csr", "jac_global"):
+        sys.stderr.write("bench.py: the global-matrix ops are single-GPU (no CSR row exchange)\n")
+        return 2
+    J = torch.empty((C, 2 * N, 2 * N) if args.op in ("jacobian", "jac_global") else (0,), dtype=torch.float64,
+                    device=dev)
     # J.v direction: one global seeded field, restricted to this rank's nodes (consistent across ranks)
     x_global = np.random.default_rng(5).normal(0, 10.0, (coords_g.shape[0], 2)) if args.op == "jvp" else None
     Xd = torch.from_numpy(np.ascontiguousarray(x_global[gids])).to(dev) if args.op == "jvp" else None
     Yd = torch.zeros((NN, 2), dtype=torch.float64, device=dev) if args.op == "jvp" else None
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     nnz, vals = 0, None
-    if args.op == "jac_csr":   # NEXT-2: pattern + slot table once per mesh (untimed)
+    if args.op in ("jac_csr", "jac_global"):   # NEXT-2: pattern + slot table once per mesh (untimed)
         _, colidx = ctx.csr_pattern()
         ctx.csr_slots()
         nnz = int(colidx.numel())
@@ -382,6 +415,9 @@ def main():
             ctx.jacobian(Uc, J, R=Rc)
         elif args.op == "jac_csr":
             ctx.jacobian_csr(Uc, vals, R=Rc)
+        elif args.op == "jac_global":   # element matrices, then the atomic-free pull assembly into CSR
+            ctx.jacobian(Uc, J, R=Rc)
+            ctx.scatter_assemble(J_cell=J, csr_vals=vals)
         elif args.op == "jvp":
             ctx.jvp(Uc, Xd, Yc, R=Rc)
         else:
@@ -444,6 +480,46 @@ def main():
     ms_total = t0.elapsed_time(t1)
     kern_ms = sum(a.elapsed_time(b) for a, b in zip(k0, k1)) / args.steps
     ctx.sync()
+
+    # ---- sustained: back-to-back steps for --sustain seconds (power controller settled) ----
+    sustained = None
+    if args.sustain > 0:
+        n_sus = max(1, int(args.sustain * 1e3 / max(ms_total / args.steps, 1e-3)) + 1)
+        if world > 1:
+            nt = torch.tensor([n_sus], dtype=torch.int64, device="cpu" if backend != "nccl" else dev)
+            dist.all_reduce(nt, op=dist.ReduceOp.MAX)
+            n_sus = int(nt.item())
+        ks0 = [torch.cuda.Event(enable_timing=True) for _ in range(n_sus)]
+        ks1 = [torch.cuda.Event(enable_timing=True) for _ in range(n_sus)]
+        clk_s = ClockSampler(local)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        clk_s.start()
+        time.sleep(0.3)
+        s0 = torch.cuda.Event(enable_timing=True)
+        s1 = torch.cuda.Event(enable_timing=True)
+        clk_s.mark_start()
+        s0.record(stream)
+        for i in range(n_sus):
+            Rc, Yc = begin()
+            if vals is not None:
+                vals.zero_()
+            ks0[i].record(stream)
+            evaluate(U, Rc, Yc)
+            ks1[i].record(stream)
+            finish(Rc, Yc)
+        s1.record(stream)
+        torch.cuda.synchronize(dev)
+        clk_s.mark_stop()
+        if world > 1:
+            dist.barrier()
+        ck = clk_s.stop()
+        kms = [a.elapsed_time(b) for a, b in zip(ks0, ks1)]
+        q = max(1, n_sus // 4)
+        sustained = {"seconds": s0.elapsed_time(s1) * 1e-3, "steps": n_sus,
+                     "ms_per_step": s0.elapsed_time(s1) / n_sus, "kernel_ms": sum(kms) / n_sus,
+                     "kernel_ms_last_quarter": sum(kms[-q:]) / q, "clocks": ck}
 
     # ---- end-to-end through the public API with host buffers ----
     # Every step uploads that step's U from pinned host memory and downloads its R;
@@ -538,7 +614,9 @@ def main():
         check = float(err.item())
 
     # ---- reduce over ranks (max time) ----
-    mine_stats = [ms_total / args.steps, kern_ms, e2e[0] if e2e else 0.0, float(C)]
+    mine_stats = [ms_total / args.steps, kern_ms, e2e[0] if e2e else 0.0, float(C),
+                  sustained["ms_per_step"] if sustained else 0.0, sustained["kernel_ms"] if sustained else 0.0,
+                  sustained["kernel_ms_last_quarter"] if sustained else 0.0]
     if world > 1:
         allst = [None] * world
         dist.all_gather_object(allst, mine_stats)
@@ -560,7 +638,9 @@ def main():
                        "resid": "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s",
                        "jvp": "Stokes-FO matrix-free J(U)X + residual (stokesfo_jvp) cells/s and achieved HBM GB/s",
                        "jac_csr": "Stokes-FO residual + Jacobian assembled into global CSR (stokesfo_jacobian_csr) "
-                                  "cells/s and achieved HBM GB/s"}[args.op],
+                                  "cells/s and achieved HBM GB/s",
+                       "jac_global": "Stokes-FO residual + Jacobian assembled into global CSR (stokesfo_jacobian + "
+                                     "stokesfo_scatter_assemble) cells/s and achieved HBM GB/s"}[args.op],
             "value": total_cells / (ms_step * 1e-3),
             "unit": "cells/s",
             "n_gpus": world,
@@ -582,22 +662,37 @@ def main():
                          "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
                          "kernel": ("eval_otf_kernel" if args.geometry == "on_the_fly" else "eval_kernel")
                          + ("<Hex8," if elem == "hex8" else "<Wedge6,")
-                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>"}[args.op]
+                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>",
+                            "jac_global": "M_JAC> + csr_gather_kernel"}[args.op]
                          + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
-                            "jvp": " (stokesfo_jvp)", "jac_csr": " (stokesfo_jacobian_csr)"}[args.op],
+                            "jvp": " (stokesfo_jvp)", "jac_csr": " (stokesfo_jacobian_csr)",
+                            "jac_global": " (stokesfo_jacobian + stokesfo_scatter_assemble, both timed)"}[args.op],
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src,
                          "live_copy_gbs": live_copy,
                          "note": "live_copy_gbs: torch device-to-device copy of 2 GiB on this box before the timed "
                                  "region (context for box-to-box variance; not the denominator)"},
             "achieved_hbm_gbs": achieved,
-            "gpu_launches": args.steps * (1 + (halo.launches_per_exchange * (2 if args.op == "jvp" else 1)
-                                               if halo else 0)),
+            "gpu_launches": args.steps * ((2 if args.op == "jac_global" else 1)
+                                          + (halo.launches_per_exchange * (2 if args.op == "jvp" else 1)
+                                             if halo else 0)),
             "halo": halo_mode,
             "clocks": clk,
         }
         if world > 1:
             line["per_rank"] = [{"rank": r, "cells": int(a[3]), "ms_per_step": a[0], "kernel_ms": a[1]}
                                 for r, a in enumerate(allst)]
+        if sustained:
+            sms = max(a[4] for a in allst)
+            skm = max(a[5] for a in allst)
+            skq = max(a[6] for a in allst)
+            sach = bpl / (skq * 1e-3) / 1e9
+            line["sustained"] = {
+                "value": total_cells / (sms * 1e-3), "unit": "cells/s", "seconds": sustained["seconds"],
+                "steps": sustained["steps"], "ms_per_step": sms, "kernel_ms": skm, "kernel_ms_last_quarter": skq,
+                "roofline_frac_last_quarter": sach / peak, "clocks": sustained["clocks"],
+                "note": "back-to-back steps for --sustain seconds right after the timed region (the burst value "
+                        "above is the first ~0.1 s, before the 1000 W power controller reacts); "
+                        "roofline_frac_last_quarter = algorithmic bytes / mean kernel time of the last quarter / peak"}
         if check is not None:
             line["halo_check_max_rel_err"] = check
         if nnz:
@@ -612,9 +707,17 @@ def main():
             rate, n, dt = oracle_sample_rate(elem, conn_g, coords_g, U_g, s_g, kc_g, target_s=12.0,
                                              mode="resid" if args.op == "resid" else "jac")
             what = "residual" if args.op == "resid" else "residual+AD Jacobian"
-            line["cpu_baseline"] = {"value": rate, "unit": "cells/s", "cores": O.num_threads(), "kind": "oracle",
+            cores = O.num_threads()
+            O.set_num_threads(1)
+            rate1, n1, dt1 = oracle_sample_rate(elem, conn_g, coords_g, U_g, s_g, kc_g, target_s=3.0,
+                                                mode="resid" if args.op == "resid" else "jac")
+            O.set_num_threads(cores)
+            line["cpu_baseline"] = {"value": rate, "unit": "cells/s", "cores": cores, "kind": "oracle",
                                     "sample": f"first {n} cells of {args.config} ({what}, "
-                                              f"geometry precomputed untimed), {dt:.1f} s"}
+                                              f"geometry precomputed untimed), {dt:.1f} s",
+                                    "value_1_thread": rate1,
+                                    "sample_1_thread": f"first {n1} cells, {dt1:.1f} s, OpenMP 1 thread",
+                                    "host_cpu": host_cpu_model()}
         print(json.dumps(line), flush=True)
     if world > 1:
         if p2p is not None:

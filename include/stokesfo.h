@@ -140,6 +140,15 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
  * pointers (stokesfo_set_remote_jvp), else EINVAL. */
 int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, double *R);
 
+/* Diagonal of the assembled Jacobian (NEXT-3, the Jacobi preconditioner of the
+ * Newton-Krylov driver): diag[2 node + a] += sum over the cells holding the node
+ * of J_cell[(i,a),(i,a)] (the same forward derivative as stokesfo_jacobian,
+ * P:L215-221; no element matrices are formed), optionally R += R(U) in the same
+ * pass.  U: dev [num_nodes][2]; diag, R: dev [num_nodes][2] (+=).  With a peer
+ * table attached it is halo-summed like stokesfo_jvp's Y (needs
+ * stokesfo_set_remote_jvp, else EINVAL). */
+int stokesfo_jacobian_diag(stokesfo_ctx *c, const double *U, double *diag, double *R);
+
 /* Basal friction side-set term (NEXT-4; P:L59 -> [24]; reading Z18):
  * on the bottom face of each listed basal cell (local nodes 0..3 hex8 /
  * 0..2 wedge6), R[2 node_i + a] += int beta_h u_h,a phi_i dGamma and

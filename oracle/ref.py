@@ -57,6 +57,8 @@ def lib():
         _lib.oracle_basis_at.argtypes = [ctypes.c_int, P, P, P]
         _lib.oracle_quadrature.argtypes = [ctypes.c_int, P, P]
         _lib.oracle_num_threads.restype = ctypes.c_int
+        _lib.oracle_set_num_threads.argtypes = [ctypes.c_int]
+        _lib.oracle_set_num_threads.restype = None
     return _lib
 
 
@@ -70,6 +72,11 @@ def _c(a, dtype):
 
 def num_threads() -> int:
     return int(lib().oracle_num_threads())
+
+
+def set_num_threads(n: int) -> None:
+    """OpenMP threads of the oracle's cell loops (timing only; results do not depend on it)."""
+    lib().oracle_set_num_threads(int(n))
 
 
 # ---------------------------------------------------------------------------

@@ -9,6 +9,8 @@
 #include <new>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX3 (no link dependency; inert without a tool attached)
+
 #include "../../include/stokesfo.h"
 #include "sfo_kernels.cuh"
 #include "sfo_albany.cuh"
@@ -25,7 +27,7 @@ struct stokesfo_ctx {
     char *recs;            // device records (full or light)
     double4 *xyz4;         // node coordinates (on-the-fly geometry mode)
     int mode;              // stokesfo_geometry_mode_t
-    int grid_resid, grid_jac, grid_jvp, grid_csr;
+    int grid_resid, grid_jac, grid_jvp, grid_csr, grid_diag;
     int rec_bytes;
     int nstage_resid, nstage_jac;  // TMA record ring depth of the eval kernels
     const int32_t *rem = nullptr;     // fused halo over peer memory (stokesfo_set_remote)
@@ -53,6 +55,26 @@ struct stokesfo_ctx {
 };
 
 namespace {
+
+// NVTX range around every C-ABI entry point when STOKESFO_PROFILE=1 (nsys / ncu --nvtx
+// timelines of a multi-rank step); a no-op otherwise.
+bool profile_on() {
+    static const bool on = [] {
+        const char *e = getenv("STOKESFO_PROFILE");
+        return e && atoi(e) == 1;
+    }();
+    return on;
+}
+struct NvtxRange {
+    bool on;
+    explicit NvtxRange(const char *name) : on(profile_on()) {
+        if (on) nvtxRangePushA(name);
+    }
+    ~NvtxRange() {
+        if (on) nvtxRangePop();
+    }
+};
+#define SFO_RANGE(name) NvtxRange sfo_nvtx_range_(name)
 
 bool aligned(const void *p, size_t a) { return (reinterpret_cast<uintptr_t>(p) % a) == 0; }
 
@@ -140,6 +162,8 @@ int create_impl(stokesfo_ctx *c) {
         if (st) return st;
         st = configure_otf<E, M_CSR>(&c->grid_csr);
         if (st) return st;
+        st = configure_otf<E, M_DIAG>(&c->grid_diag);
+        if (st) return st;
     } else {
         // ring depth: default per element, STOKESFO_STAGES_{RESID,JAC} override (2 or 3)
         c->nstage_resid = default_stages<E, false>();
@@ -155,6 +179,8 @@ int create_impl(stokesfo_ctx *c) {
         st = configure_eval<E, M_JVP, 2>(&c->grid_jvp);
         if (st) return st;
         st = configure_eval<E, M_CSR, 2>(&c->grid_csr);
+        if (st) return st;
+        st = configure_eval<E, M_DIAG, 2>(&c->grid_diag);
         if (st) return st;
     }
     if (cudaMemsetAsync(c->err, 0, sizeof(int), c->stream) != cudaSuccess) return cuda_status();
@@ -252,7 +278,8 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.csr_vals = csr_vals;
     const int g = MODE == M_JAC ? c->grid_jac
                 : MODE == M_JVP ? c->grid_jvp
-                : MODE == M_CSR ? c->grid_csr : c->grid_resid;
+                : MODE == M_CSR ? c->grid_csr
+                : MODE == M_DIAG ? c->grid_diag : c->grid_resid;
     const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
     a.use_jmap = (!otf && MODE == M_JAC && wedge_jmap<E>(c, J_cell)) ? 1 : 0;
     const CUtensorMap jm = a.use_jmap ? c->jmap : CUtensorMap{};
@@ -288,6 +315,7 @@ const char *stokesfo_strerror(int s) {
 }
 
 int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes) {
+    SFO_RANGE("stokesfo_workspace_size");
     if (!d || !bytes || d->num_cells < 0) return STOKESFO_EINVAL;
     if (d->geometry_mode != STOKESFO_GEOMETRY_STORED && d->geometry_mode != STOKESFO_GEOMETRY_ON_THE_FLY)
         return STOKESFO_EINVAL;
@@ -298,6 +326,7 @@ int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes) {
 }
 
 int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
+    SFO_RANGE("stokesfo_create");
     if (!d || !out) return STOKESFO_EINVAL;
     *out = nullptr;
     if (d->abi_version != STOKESFO_ABI_VERSION) return STOKESFO_EINVAL;
@@ -346,9 +375,11 @@ int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
     return STOKESFO_OK;
 }
 
-void stokesfo_destroy(stokesfo_ctx *c) { delete c; }
+void stokesfo_destroy(stokesfo_ctx *c) {
+    SFO_RANGE("stokesfo_destroy"); delete c; }
 
 int stokesfo_gather(stokesfo_ctx *c, const double *U, double *U_cell) {
+    SFO_RANGE("stokesfo_gather");
     if (!c) return STOKESFO_EINVAL;
     if (c->d.num_cells == 0) return STOKESFO_OK;
     if (!U || !U_cell || !aligned(U, 16) || !aligned(U_cell, 16)) return STOKESFO_EINVAL;
@@ -364,6 +395,7 @@ int stokesfo_gather(stokesfo_ctx *c, const double *U, double *U_cell) {
 }
 
 int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R) {
+    SFO_RANGE("stokesfo_viscosity_resid");
     if (!c) return STOKESFO_EINVAL;
     if (c->d.num_cells == 0) return STOKESFO_OK;
     if (!U || !aligned(U, 16)) return STOKESFO_EINVAL;
@@ -376,6 +408,7 @@ int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, do
 }
 
 int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *R_cell, double *R) {
+    SFO_RANGE("stokesfo_jacobian");
     if (!c) return STOKESFO_EINVAL;
     if (c->d.num_cells == 0) return STOKESFO_OK;  // nothing to evaluate (outputs may be NULL)
     if (!U || !J_cell || !aligned(U, 16) || !aligned(J_cell, 16)) return STOKESFO_EINVAL;
@@ -388,6 +421,7 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
 }
 
 int stokesfo_jacobian_csr(stokesfo_ctx *c, const double *U, double *csr_vals, double *R) {
+    SFO_RANGE("stokesfo_jacobian_csr");
     if (!c) return STOKESFO_EINVAL;
     if (c->d.num_cells == 0) return STOKESFO_OK;
     if (!c->slots || !c->rowptr) return STOKESFO_EINVAL;  // needs stokesfo_csr_slots
@@ -405,12 +439,14 @@ static int64_t slots_off_inc(const stokesfo_ctx *c) {
 }
 
 int stokesfo_csr_slots_size(stokesfo_ctx *c, size_t *bytes) {
+    SFO_RANGE("stokesfo_csr_slots_size");
     if (!c || !bytes) return STOKESFO_EINVAL;
     *bytes = (size_t)(slots_off_inc(c) + round_up(c->d.num_cells * c->N * 4, 16));
     return STOKESFO_OK;
 }
 
 int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots) {
+    SFO_RANGE("stokesfo_csr_slots");
     if (!c || !slots || !aligned(slots, 16)) return STOKESFO_EINVAL;
     if (!c->rowptr || !c->colidx) return STOKESFO_EINVAL;  // needs the stokesfo_csr_pattern fill
     if (c->csr_maxdeg > 256) return STOKESFO_EUNSUPPORTED;
@@ -444,6 +480,7 @@ int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots) {
 }
 
 int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, double *R) {
+    SFO_RANGE("stokesfo_jvp");
     if (!c) return STOKESFO_EINVAL;
     if (c->d.num_cells == 0) return STOKESFO_OK;
     if (!U || !X || !Y || !aligned(U, 16) || !aligned(X, 16) || !aligned(Y, 16) || (R && !aligned(R, 16)))
@@ -454,8 +491,20 @@ int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, d
 #undef CALL
 }
 
+int stokesfo_jacobian_diag(stokesfo_ctx *c, const double *U, double *diag, double *R) {
+    SFO_RANGE("stokesfo_jacobian_diag");
+    if (!c) return STOKESFO_EINVAL;
+    if (c->d.num_cells == 0) return STOKESFO_OK;
+    if (!U || !diag || !aligned(U, 16) || !aligned(diag, 16) || (R && !aligned(R, 16))) return STOKESFO_EINVAL;
+    if (c->rem && !c->peers_y) return STOKESFO_EINVAL;  // diag would miss the peers' boundary contributions
+#define CALL(E) eval_impl<E, M_DIAG>(c, U, nullptr, nullptr, R, nullptr, nullptr, diag)
+    return DISPATCH(c, CALL);
+#undef CALL
+}
+
 int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nfaces, const double *beta,
                             const double *U, double *R, double *J_face) {
+    SFO_RANGE("stokesfo_basal_friction");
     if (!c || nfaces < 0) return STOKESFO_EINVAL;
     if (nfaces == 0) return STOKESFO_OK;
     if (!basal_cells || !beta || !U || !R || !aligned(U, 16) || !aligned(R, 16) || (J_face && !aligned(J_face, 16)))
@@ -473,6 +522,7 @@ int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t
 
 int stokesfo_lateral_pressure(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
                               double rho_i_g, double rho_w_g, double sea_level, double *R) {
+    SFO_RANGE("stokesfo_lateral_pressure");
     if (!c || nfaces < 0) return STOKESFO_EINVAL;
     if (nfaces == 0) return STOKESFO_OK;
     if (!faces || !surface || !R || !aligned(faces, 8) || !aligned(R, 16)) return STOKESFO_EINVAL;
@@ -490,6 +540,7 @@ int stokesfo_lateral_pressure(stokesfo_ctx *c, const int32_t *faces, int64_t nfa
 
 int stokesfo_set_lateral(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
                          double rho_i_g, double rho_w_g, double sea_level) {
+    SFO_RANGE("stokesfo_set_lateral");
     if (!c || nfaces < 0) return STOKESFO_EINVAL;
     if (nfaces > 0 && (!faces || !surface || !aligned(faces, 8))) return STOKESFO_EINVAL;
     c->lat_faces = nfaces > 0 ? faces : nullptr;
@@ -503,6 +554,7 @@ int stokesfo_set_lateral(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, 
 
 int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, const double *J_cell,
                               double *csr_vals) {
+    SFO_RANGE("stokesfo_scatter_assemble");
     if (!c) return STOKESFO_EINVAL;
     const void *ps[] = {R_cell, R, J_cell, csr_vals};
     for (const void *p : ps)
@@ -546,6 +598,7 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
 }
 
 int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure) {
+    SFO_RANGE("stokesfo_geometry");
     if (!c) return STOKESFO_EINVAL;
     if ((grad_bf && !aligned(grad_bf, 16)) || (w_measure && !aligned(w_measure, 16))) return STOKESFO_EINVAL;
     const int64_t work = c->d.num_cells * c->Q;
@@ -570,6 +623,7 @@ int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure) {
 }
 
 int stokesfo_halo_pack(stokesfo_ctx *c, const double *R, const int32_t *send_nodes, int64_t n, double *buf) {
+    SFO_RANGE("stokesfo_halo_pack");
     if (!c || n < 0) return STOKESFO_EINVAL;
     if (n == 0) return STOKESFO_OK;
     if (!R || !send_nodes || !buf || !aligned(R, 16) || !aligned(buf, 16)) return STOKESFO_EINVAL;
@@ -580,6 +634,7 @@ int stokesfo_halo_pack(stokesfo_ctx *c, const double *R, const int32_t *send_nod
 }
 
 int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *recv_nodes, int64_t n, double *R) {
+    SFO_RANGE("stokesfo_halo_unpack_add");
     if (!c || n < 0) return STOKESFO_EINVAL;
     if (n == 0) return STOKESFO_OK;
     if (!R || !recv_nodes || !buf || !aligned(R, 16) || !aligned(buf, 16)) return STOKESFO_EINVAL;
@@ -590,6 +645,7 @@ int stokesfo_halo_unpack_add(stokesfo_ctx *c, const double *buf, const int32_t *
 }
 
 int stokesfo_set_remote(stokesfo_ctx *c, const int32_t *rem, const int32_t *remtab, double *const *peers) {
+    SFO_RANGE("stokesfo_set_remote");
     if (!c) return STOKESFO_EINVAL;
     if (!rem) {  // detach
         c->rem = nullptr;
@@ -606,6 +662,7 @@ int stokesfo_set_remote(stokesfo_ctx *c, const int32_t *rem, const int32_t *remt
 }
 
 int stokesfo_set_remote_jvp(stokesfo_ctx *c, double *const *peers_y) {
+    SFO_RANGE("stokesfo_set_remote_jvp");
     if (!c) return STOKESFO_EINVAL;
     if (peers_y && !c->rem) return STOKESFO_EINVAL;  // needs the node table of stokesfo_set_remote
     c->peers_y = peers_y;
@@ -613,6 +670,7 @@ int stokesfo_set_remote_jvp(stokesfo_ctx *c, double *const *peers_y) {
 }
 
 int stokesfo_ipc_get_handle(const void *dev_ptr, void *handle, int64_t *offset) {
+    SFO_RANGE("stokesfo_ipc_get_handle");
     if (!dev_ptr || !handle || !offset) return STOKESFO_EINVAL;
     cudaIpcMemHandle_t h;
     if (cudaIpcGetMemHandle(&h, const_cast<void *>(dev_ptr)) != cudaSuccess) return cuda_status();
@@ -633,6 +691,7 @@ int stokesfo_ipc_get_handle(const void *dev_ptr, void *handle, int64_t *offset) 
 }
 
 int stokesfo_ipc_open_handle(const void *handle, void **dev_ptr) {
+    SFO_RANGE("stokesfo_ipc_open_handle");
     if (!dev_ptr || !handle) return STOKESFO_EINVAL;
     cudaIpcMemHandle_t h;
     memcpy(&h, handle, sizeof(h));
@@ -641,12 +700,14 @@ int stokesfo_ipc_open_handle(const void *handle, void **dev_ptr) {
 }
 
 int stokesfo_ipc_close(void *dev_ptr) {
+    SFO_RANGE("stokesfo_ipc_close");
     if (!dev_ptr) return STOKESFO_EINVAL;
     if (cudaIpcCloseMemHandle(dev_ptr) != cudaSuccess) return cuda_status();
     return STOKESFO_OK;
 }
 
 int stokesfo_sync(stokesfo_ctx *c) {
+    SFO_RANGE("stokesfo_sync");
     if (!c) return STOKESFO_EINVAL;
     if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_status();
     int h = 0;
@@ -656,6 +717,7 @@ int stokesfo_sync(stokesfo_ctx *c) {
 
 int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid_resid, int32_t *grid_jac,
                          int64_t *record_bytes_per_tile) {
+    SFO_RANGE("stokesfo_launch_info");
     if (!c) return STOKESFO_EINVAL;
     if (cells_per_tile) *cells_per_tile = c->TC;
     if (grid_resid) *grid_resid = (int32_t)std::min<int64_t>(c->grid_resid, std::max<int64_t>(c->ntiles, 1));
@@ -689,12 +751,15 @@ int albany_run(stokesfo_ctx *c, int stage, int variant, const double *U, double 
             viscosity_kernel<E, ND><<<gq, bs, 0, c->stream>>>(C, c->d.flow_factor, c->d.k, c->d.delta, S);
             bodyforce_kernel<E, ND><<<gq, bs, 0, c->stream>>>(C, c->d.conn, c->d.surface, c->d.rho_g, S);
             break;
-        case 2:  // StokesFOResid (Fig. 2)
+        case 2: {  // StokesFOResid (Fig. 2), SFO_ALBANY_MAXT threads per block (its launch bound)
+            const int bt = SFO_ALBANY_MAXT;
+            const unsigned gt = (unsigned)((C + bt - 1) / bt);
             if (variant == STOKESFO_FIG2_BASELINE)
-                stokesfo_resid_baseline_kernel<E, ND><<<gc, bs, 0, c->stream>>>(C, S);
+                stokesfo_resid_baseline_kernel<E, ND><<<gt, bt, 0, c->stream>>>(C, S);
             else
-                stokesfo_resid_optimized_kernel<E, ND><<<gc, bs, 0, c->stream>>>(C, S);
+                stokesfo_resid_optimized_kernel<E, ND><<<gt, bt, 0, c->stream>>>(C, S);
             break;
+        }
         case 3: {  // extract
             const unsigned gr = (unsigned)((C * 2 * E::N + bs - 1) / bs);
             extract_kernel<E, ND><<<gr, bs, 0, c->stream>>>(C, S, R_cell, J_cell);
@@ -721,6 +786,7 @@ int albany_dispatch(stokesfo_ctx *c, int derivs, int stage, int variant, const d
 extern "C" {
 
 int stokesfo_albany_scratch_size(stokesfo_ctx *c, int derivs, size_t *bytes) {
+    SFO_RANGE("stokesfo_albany_scratch_size");
     if (!c || !bytes || (derivs != 0 && derivs != 1)) return STOKESFO_EINVAL;
     int64_t per;
     if (c->N == 8) per = derivs ? sfo::albany::Scratch<Hex8, 16>::TOTAL : sfo::albany::Scratch<Hex8, 0>::TOTAL;
@@ -729,16 +795,20 @@ int stokesfo_albany_scratch_size(stokesfo_ctx *c, int derivs, size_t *bytes) {
     return STOKESFO_OK;
 }
 int stokesfo_albany_setup(stokesfo_ctx *c, int derivs, double *scratch) {
+    SFO_RANGE("stokesfo_albany_setup");
     return albany_dispatch(c, derivs, 0, 0, nullptr, scratch, nullptr, nullptr);
 }
 int stokesfo_albany_evaluators(stokesfo_ctx *c, int derivs, const double *U, double *scratch) {
+    SFO_RANGE("stokesfo_albany_evaluators");
     if (!U) return STOKESFO_EINVAL;
     return albany_dispatch(c, derivs, 1, 0, U, scratch, nullptr, nullptr);
 }
 int stokesfo_albany_resid(stokesfo_ctx *c, int derivs, int variant, double *scratch) {
+    SFO_RANGE("stokesfo_albany_resid");
     return albany_dispatch(c, derivs, 2, variant, nullptr, scratch, nullptr, nullptr);
 }
 int stokesfo_albany_extract(stokesfo_ctx *c, int derivs, const double *scratch, double *R_cell, double *J_cell) {
+    SFO_RANGE("stokesfo_albany_extract");
     return albany_dispatch(c, derivs, 3, 0, nullptr, const_cast<double *>(scratch), R_cell, J_cell);
 }
 
@@ -748,13 +818,14 @@ int stokesfo_albany_extract(stokesfo_ctx *c, int derivs, const double *scratch, 
 }  // extern "C"
 
 namespace {
+constexpr int CG_BLOCK = 8;  // CG iterations per graph replay (one host convergence check per block)
 struct NewtonWork {
-    double *F, *D, *Rr, *P, *AP, *Z, *Ut, *diag, *Jc, *Jf, *scal;
+    double *F, *D, *Rr, *P, *AP, *Z, *Ut, *diag, *Jf, *scal, *hist;
     int64_t bytes;
 };
 NewtonWork newton_layout(const stokesfo_ctx *c, int64_t nbasal, char *base) {
     NewtonWork w{};
-    const int64_t n = 2 * c->d.num_nodes, C = c->d.num_cells, ND = 2 * c->N, NFD = c->N;  // face: 2*NB = N
+    const int64_t n = 2 * c->d.num_nodes, NFD = c->N;  // face matrix: 2*NB = N
     int64_t off = 0;
     auto take = [&](int64_t count) {
         double *p = reinterpret_cast<double *>(base + off);
@@ -762,7 +833,7 @@ NewtonWork newton_layout(const stokesfo_ctx *c, int64_t nbasal, char *base) {
         return p;
     };
     w.F = take(n); w.D = take(n); w.Rr = take(n); w.P = take(n); w.AP = take(n); w.Z = take(n); w.Ut = take(n);
-    w.diag = take(n); w.Jc = take(C * ND * ND); w.Jf = take(nbasal * NFD * NFD); w.scal = take(32);
+    w.diag = take(n); w.Jf = take(nbasal * NFD * NFD); w.scal = take(32); w.hist = take(CG_BLOCK);
     w.bytes = off;
     return w;
 }
@@ -771,6 +842,7 @@ NewtonWork newton_layout(const stokesfo_ctx *c, int64_t nbasal, char *base) {
 extern "C" {
 
 int stokesfo_newton_work_size(stokesfo_ctx *c, int64_t nbasal, size_t *bytes) {
+    SFO_RANGE("stokesfo_newton_work_size");
     if (!c || !bytes || nbasal < 0) return STOKESFO_EINVAL;
     *bytes = (size_t)newton_layout(c, nbasal, nullptr).bytes;
     return STOKESFO_OK;
@@ -779,6 +851,7 @@ int stokesfo_newton_work_size(stokesfo_ctx *c, int64_t nbasal, size_t *bytes) {
 int stokesfo_newton_solve(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nbasal, const double *beta,
                           double *U, void *work, const stokesfo_newton_opts_t *o, double *hist_F, int32_t *hist_cg,
                           int32_t *iters) {
+    SFO_RANGE("stokesfo_newton_solve");
     using namespace sfo::newton;
     if (!c || !U || !work || !o || !hist_F || !iters || nbasal < 0 || (nbasal > 0 && (!basal_cells || !beta)))
         return STOKESFO_EINVAL;
@@ -787,112 +860,163 @@ int stokesfo_newton_solve(stokesfo_ctx *c, const int32_t *basal_cells, int64_t n
     NewtonWork w = newton_layout(c, nbasal, reinterpret_cast<char *>(work));
     const int64_t n = 2 * c->d.num_nodes;
     const size_t vb = (size_t)n * 8;
-    cudaStream_t st = c->stream;
     const int bs = 256;
     const unsigned gv = (unsigned)std::min<int64_t>((n + bs - 1) / bs, 148 * 8);
-    int rc = STOKESFO_OK;
-#define CK(x)                     \
-    do {                          \
-        rc = (x);                 \
-        if (rc != STOKESFO_OK) return rc; \
-    } while (0)
-    auto dot = [&](const double *x, const double *y, double &out) -> int {
-        if (cudaMemsetAsync(w.scal, 0, 8, st) != cudaSuccess) return cuda_status();
-        dot_kernel<<<gv, bs, 0, st>>>(n, x, y, w.scal);
-        if (cudaMemcpyAsync(&out, w.scal, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess) return cuda_status();
-        if (cudaStreamSynchronize(st) != cudaSuccess) return cuda_status();
-        return STOKESFO_OK;
-    };
-    auto eval_F = [&](const double *u, double *F) -> int {  // F = R_visc(u) + R_basal(u) + R_lateral
-        if (cudaMemsetAsync(F, 0, vb, st) != cudaSuccess) return cuda_status();
-        int r = stokesfo_viscosity_resid(c, u, nullptr, nullptr, F);
-        if (r == STOKESFO_OK && nbasal > 0) r = stokesfo_basal_friction(c, basal_cells, nbasal, beta, u, F, nullptr);
-        if (r == STOKESFO_OK && c->lat_n > 0)
-            r = stokesfo_lateral_pressure(c, c->lat_faces, c->lat_n, c->lat_surface, c->lat_rho_i_g, c->lat_rho_w_g,
-                                          c->lat_sea, F);
-        return r;
-    };
-    auto apply_A = [&](const double *v, double *Av) -> int {  // Av = J(U) v + J_basal v
-        if (cudaMemsetAsync(Av, 0, vb, st) != cudaSuccess) return cuda_status();
-        int r = stokesfo_jvp(c, U, v, Av, nullptr);
-        if (r == STOKESFO_OK && nbasal > 0) r = stokesfo_basal_friction(c, basal_cells, nbasal, beta, v, Av, nullptr);
-        return r;
-    };
-    double nF0 = 0.0;
-    int k = 0;
-    for (;; ++k) {
-        CK(eval_F(U, w.F));
-        double ff;
-        CK(dot(w.F, w.F, ff));
-        const double nF = sqrt(ff);
-        hist_F[k] = nF;
-        if (k == 0) nF0 = nF;
-        if (nF <= std::max(o->atol_newton, o->rtol_newton * nF0) || k >= o->max_newton) break;
-        // Jacobi diagonal of J(U) + J_basal
-        CK(stokesfo_jacobian(c, U, w.Jc, nullptr, nullptr));
-        if (cudaMemsetAsync(w.diag, 0, vb, st) != cudaSuccess) return cuda_status();
-        {
-            const int64_t work_c = c->d.num_cells * 2 * c->N;
-            const unsigned g = (unsigned)((work_c + bs - 1) / bs);
-            if (c->N == 8) diag_cells_kernel<8><<<g, bs, 0, st>>>(c->d.num_cells, c->d.conn, w.Jc, w.diag);
-            else diag_cells_kernel<6><<<g, bs, 0, st>>>(c->d.num_cells, c->d.conn, w.Jc, w.diag);
-        }
-        if (nbasal > 0) {
-            if (cudaMemsetAsync(w.Z, 0, vb, st) != cudaSuccess) return cuda_status();
-            CK(stokesfo_basal_friction(c, basal_cells, nbasal, beta, U, w.Z, w.Jf));
-            const unsigned g = (unsigned)((nbasal * c->N + bs - 1) / bs);
-            if (c->N == 8) diag_faces_kernel<8><<<g, bs, 0, st>>>(nbasal, basal_cells, c->d.conn, w.Jf, w.diag);
-            else diag_faces_kernel<6><<<g, bs, 0, st>>>(nbasal, basal_cells, c->d.conn, w.Jf, w.diag);
-        }
-        // CG on J D = -F
-        if (cudaMemsetAsync(w.D, 0, vb, st) != cudaSuccess) return cuda_status();
-        if (cudaMemsetAsync(w.Rr, 0, vb, st) != cudaSuccess) return cuda_status();
-        axpby_kernel<<<gv, bs, 0, st>>>(n, -1.0, w.F, 0.0, w.Rr);            // r = -F
-        jacobi_kernel<<<gv, bs, 0, st>>>(n, w.Rr, w.diag, w.Z);             // z = r / diag
-        if (cudaMemcpyAsync(w.P, w.Z, vb, cudaMemcpyDeviceToDevice, st) != cudaSuccess) return cuda_status();
-        double rz;
-        CK(dot(w.Rr, w.Z, rz));
-        int j = 0;
-        for (; j < o->max_cg; ++j) {
-            CK(apply_A(w.P, w.AP));
-            double pAp;
-            CK(dot(w.P, w.AP, pAp));
-            const double alpha = rz / pAp;
-            axpby_kernel<<<gv, bs, 0, st>>>(n, alpha, w.P, 1.0, w.D);       // D += alpha p
-            axpby_kernel<<<gv, bs, 0, st>>>(n, -alpha, w.AP, 1.0, w.Rr);    // r -= alpha A p
-            double rr;
-            CK(dot(w.Rr, w.Rr, rr));
-            if (sqrt(rr) <= o->rtol_cg * nF) {
-                ++j;
-                break;
-            }
-            jacobi_kernel<<<gv, bs, 0, st>>>(n, w.Rr, w.diag, w.Z);
-            double rz_new;
-            CK(dot(w.Rr, w.Z, rz_new));
-            axpby_kernel<<<gv, bs, 0, st>>>(n, 1.0, w.Z, rz_new / rz, w.P);  // p = z + (rz_new / rz) p
-            rz = rz_new;
-        }
-        if (hist_cg) hist_cg[k] = j;
-        // Armijo backtracking on ||F||
-        double a = 1.0;
-        for (int ls = 0;; ++ls) {
-            if (cudaMemcpyAsync(w.Ut, U, vb, cudaMemcpyDeviceToDevice, st) != cudaSuccess) return cuda_status();
-            axpby_kernel<<<gv, bs, 0, st>>>(n, a, w.D, 1.0, w.Ut);
-            CK(eval_F(w.Ut, w.Rr));
-            double ft;
-            CK(dot(w.Rr, w.Rr, ft));
-            if (sqrt(ft) <= (1.0 - o->ls_c * a) * nF || ls >= o->max_ls) break;
-            a *= 0.5;
-        }
-        if (cudaMemcpyAsync(U, w.Ut, vb, cudaMemcpyDeviceToDevice, st) != cudaSuccess) return cuda_status();
+    // the solve runs on a stream of its own (graph capture needs a non-legacy stream), ordered
+    // after the caller's work on the ctx stream and before anything the caller enqueues next
+    cudaStream_t user = c->stream, st = nullptr;
+    cudaEvent_t ev = nullptr;
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t gexec = nullptr;
+    if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess || cudaEventRecord(ev, user) != cudaSuccess ||
+        cudaStreamWaitEvent(st, ev, 0) != cudaSuccess) {
+        if (st) cudaStreamDestroy(st);
+        if (ev) cudaEventDestroy(ev);
+        return cuda_status();
     }
+    c->stream = st;
+    int rc = STOKESFO_OK;
+    double host_hist[CG_BLOCK];
+#define CK(x)                            \
+    do {                                 \
+        rc = (x);                        \
+        if (rc != STOKESFO_OK) goto done; \
+    } while (0)
+#define CU(x)                                   \
+    do {                                        \
+        if ((x) != cudaSuccess) {               \
+            rc = cuda_status();                 \
+            if (rc == STOKESFO_OK) rc = STOKESFO_ECUDA; \
+            goto done;                          \
+        }                                       \
+    } while (0)
+    {
+        auto dot_dev = [&](const double *x, const double *y, double *slot) -> int {  // *slot = x . y (async)
+            if (cudaMemsetAsync(slot, 0, 8, st) != cudaSuccess) return cuda_status();
+            dot_kernel<<<gv, bs, 0, st>>>(n, x, y, slot);
+            return cuda_status();
+        };
+        auto dot_host = [&](const double *x, const double *y, double &out) -> int {
+            int r = dot_dev(x, y, w.scal + 16);
+            if (r != STOKESFO_OK) return r;
+            if (cudaMemcpyAsync(&out, w.scal + 16, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+                cudaStreamSynchronize(st) != cudaSuccess)
+                return cuda_status();
+            return STOKESFO_OK;
+        };
+        auto eval_F = [&](const double *u, double *F) -> int {  // F = R_visc(u) + R_basal(u) + R_lateral
+            if (cudaMemsetAsync(F, 0, vb, st) != cudaSuccess) return cuda_status();
+            int r = stokesfo_viscosity_resid(c, u, nullptr, nullptr, F);
+            if (r == STOKESFO_OK && nbasal > 0) r = stokesfo_basal_friction(c, basal_cells, nbasal, beta, u, F, nullptr);
+            if (r == STOKESFO_OK && c->lat_n > 0)
+                r = stokesfo_lateral_pressure(c, c->lat_faces, c->lat_n, c->lat_surface, c->lat_rho_i_g,
+                                              c->lat_rho_w_g, c->lat_sea, F);
+            return r;
+        };
+        // one CG iteration with device-side scalars (captured CG_BLOCK times into the graph)
+        auto cg_iter = [&]() -> int {
+            if (cudaMemsetAsync(w.AP, 0, vb, st) != cudaSuccess) return cuda_status();
+            int r = stokesfo_jvp(c, U, w.P, w.AP, nullptr);                   // Ap = J(U) p
+            if (r == STOKESFO_OK && nbasal > 0) r = stokesfo_basal_friction(c, basal_cells, nbasal, beta, w.P, w.AP, nullptr);
+            if (r == STOKESFO_OK) r = dot_dev(w.P, w.AP, w.scal + S_PAP);
+            if (r != STOKESFO_OK) return r;
+            cg_alpha_kernel<<<1, 1, 0, st>>>(w.scal);
+            axpy_dev_kernel<<<gv, bs, 0, st>>>(n, w.scal + S_ALPHA, 1.0, w.P, w.D);     // D += alpha p
+            axpy_dev_kernel<<<gv, bs, 0, st>>>(n, w.scal + S_ALPHA, -1.0, w.AP, w.Rr);  // r -= alpha Ap
+            r = dot_dev(w.Rr, w.Rr, w.scal + S_RR);
+            if (r != STOKESFO_OK) return r;
+            jacobi_kernel<<<gv, bs, 0, st>>>(n, w.Rr, w.diag, w.Z);                      // z = r / diag
+            r = dot_dev(w.Rr, w.Z, w.scal + S_RZN);
+            if (r != STOKESFO_OK) return r;
+            cg_beta_kernel<<<1, 1, 0, st>>>(w.scal, w.hist);
+            xpby_dev_kernel<<<gv, bs, 0, st>>>(n, w.Z, w.scal + S_BETA, w.P);           // p = z + beta p
+            return cuda_status();
+        };
+        // the CG block graph: every pointer it touches is fixed for the whole solve (U is updated in place)
+        CU(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed));
+        {
+            int r = STOKESFO_OK;
+            for (int k = 0; k < CG_BLOCK && r == STOKESFO_OK; ++k) r = cg_iter();
+            cudaGraph_t g = nullptr;
+            const cudaError_t e = cudaStreamEndCapture(st, &g);
+            graph = g;
+            if (r != STOKESFO_OK) { rc = r; goto done; }
+            CU(e);
+        }
+        CU(cudaGraphInstantiate(&gexec, graph, 0));
+
+        double nF0 = 0.0;
+        int k = 0;
+        for (;; ++k) {
+            CK(eval_F(U, w.F));
+            double ff;
+            CK(dot_host(w.F, w.F, ff));
+            const double nF = sqrt(ff);
+            hist_F[k] = nF;
+            if (k == 0) nF0 = nF;
+            if (nF <= std::max(o->atol_newton, o->rtol_newton * nF0) || k >= o->max_newton) break;
+            // Jacobi diagonal of J(U) + J_basal: the diagonal-only evaluation (no element matrices)
+            CU(cudaMemsetAsync(w.diag, 0, vb, st));
+            CK(stokesfo_jacobian_diag(c, U, w.diag, nullptr));
+            if (nbasal > 0) {
+                CU(cudaMemsetAsync(w.Z, 0, vb, st));
+                CK(stokesfo_basal_friction(c, basal_cells, nbasal, beta, U, w.Z, w.Jf));
+                const unsigned g = (unsigned)((nbasal * c->N + bs - 1) / bs);
+                if (c->N == 8) diag_faces_kernel<8><<<g, bs, 0, st>>>(nbasal, basal_cells, c->d.conn, w.Jf, w.diag);
+                else diag_faces_kernel<6><<<g, bs, 0, st>>>(nbasal, basal_cells, c->d.conn, w.Jf, w.diag);
+            }
+            // CG on J D = -F: D = 0, r = -F, z = r / diag, p = z, r.z -> s[RZ]
+            CU(cudaMemsetAsync(w.D, 0, vb, st));
+            CU(cudaMemsetAsync(w.Rr, 0, vb, st));
+            axpby_kernel<<<gv, bs, 0, st>>>(n, -1.0, w.F, 0.0, w.Rr);
+            jacobi_kernel<<<gv, bs, 0, st>>>(n, w.Rr, w.diag, w.Z);
+            CU(cudaMemcpyAsync(w.P, w.Z, vb, cudaMemcpyDeviceToDevice, st));
+            CK(dot_dev(w.Rr, w.Z, w.scal + S_RZ));
+            const double tol2 = (o->rtol_cg * nF) * (o->rtol_cg * nF);
+            int j = 0, done_at = -1;
+            while (j < o->max_cg && done_at < 0) {
+                CU(cudaMemsetAsync(w.scal + S_IT, 0, 8, st));
+                CU(cudaGraphLaunch(gexec, st));
+                CU(cudaMemcpyAsync(host_hist, w.hist, sizeof(host_hist), cudaMemcpyDeviceToHost, st));
+                CU(cudaStreamSynchronize(st));
+                for (int t = 0; t < CG_BLOCK; ++t)
+                    if (done_at < 0 && host_hist[t] <= tol2) done_at = j + t + 1;
+                j += CG_BLOCK;
+            }
+            if (hist_cg) hist_cg[k] = done_at > 0 ? done_at : j;  // iterations to convergence (the block may run a few more)
+            // Armijo backtracking on ||F||
+            double a = 1.0;
+            for (int ls = 0;; ++ls) {
+                CU(cudaMemcpyAsync(w.Ut, U, vb, cudaMemcpyDeviceToDevice, st));
+                axpby_kernel<<<gv, bs, 0, st>>>(n, a, w.D, 1.0, w.Ut);
+                CK(eval_F(w.Ut, w.Rr));
+                double ft;
+                CK(dot_host(w.Rr, w.Rr, ft));
+                if (sqrt(ft) <= (1.0 - o->ls_c * a) * nF || ls >= o->max_ls) break;
+                a *= 0.5;
+            }
+            CU(cudaMemcpyAsync(U, w.Ut, vb, cudaMemcpyDeviceToDevice, st));
+        }
+        *iters = k;
+    }
+done:
 #undef CK
-    *iters = k;
-    return cuda_status();
+#undef CU
+    cudaStreamSynchronize(st);
+    if (gexec) cudaGraphExecDestroy(gexec);
+    if (graph) cudaGraphDestroy(graph);
+    c->stream = user;
+    cudaEventRecord(ev, st);
+    cudaStreamWaitEvent(user, ev, 0);
+    cudaEventDestroy(ev);
+    cudaStreamDestroy(st);
+    return rc != STOKESFO_OK ? rc : cuda_status();
 }
 
 // CSR pattern: host-side construction from a device->host copy of conn.
 int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t *colidx) {
+    SFO_RANGE("stokesfo_csr_pattern");
     if (!c || !nnz) return STOKESFO_EINVAL;
     const int64_t C = c->d.num_cells, NN = c->d.num_nodes;
     const int N = c->N;

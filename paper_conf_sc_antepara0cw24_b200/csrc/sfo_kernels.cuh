@@ -256,14 +256,14 @@ struct EvalArgs {
     double *R;                // [nodes][2] or null (+=)
     double *J_cell;           // [C][2N][2N] (M_JAC)
     const double *X;          // [nodes][2] direction (M_JVP)
-    double *Y;                // [nodes][2] += J(U) X (M_JVP)
+    double *Y;                // [nodes][2] += J(U) X (M_JVP), or += diag J(U) (M_DIAG)
     // fused halo over peer memory (null = none): rem[node] = row of remtab or -1;
     // remtab[row] = {count, peer_0, idx_0, peer_1, idx_1, ...} (REM_ROW ints);
     // peers[p] = device pointer of peer p's R, mapped into this process
     const int32_t *rem;
     const int32_t *remtab;
     double *const *peers;
-    double *const *peers_y;   // M_JVP: the peers' Y (required when rem is set)
+    double *const *peers_y;   // M_JVP / M_DIAG: the peers' Y (required when rem is set)
     // NEXT-2 fused CSR assembly (M_CSR): J contributions go straight into
     // csr_vals[rowptr[2 g_i + a] + 2 slot[c][i][j] + b] (no element matrices)
     const int64_t *rowptr;    // [2 nodes + 1]
@@ -310,7 +310,10 @@ __device__ __forceinline__ void scatter_node(const int32_t *rem, const int32_t *
 #endif
 
 // Evaluation modes of the fused kernels
-enum { M_RESID = 0, M_JAC = 1, M_JVP = 2, M_CSR = 3 };
+// M_DIAG: residual + the diagonal of the assembled Jacobian only (Jacobi
+// preconditioner of the Newton-Krylov driver): J[(i,a),(i,a)] of every cell
+// scatter-added into Y, no element matrices.
+enum { M_RESID = 0, M_JAC = 1, M_JVP = 2, M_CSR = 3, M_DIAG = 4 };
 // modes that form the tangent blocks (element matrices or CSR contributions)
 template <int MODE>
 __host__ __device__ constexpr bool forms_jac() {
@@ -465,6 +468,14 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const QS &qs, 
             const double e1 = fma(gi2, d12, fma(gi1, d11, gi0 * d01));
             dR0 = fma(gt, h0, fma(wmu2, e0, dR0));
             dR1 = fma(gt, h1, fma(wmu2, e1, dR1));
+        }
+        if (MODE == M_DIAG) {
+            // J[(i,a),(i,a)] = wM 2 mu G_i^T B_aa G_i + gamma h_(i,a)^2,
+            // B_00 = diag(2, 1/2, 1/2), B_11 = diag(1/2, 2, 1/2) (the k = 0 block's diagonal)
+            const double gam = qs(6, c2, q);
+            const double t = 0.5 * fma(gi2, gi2, fma(gi1, gi1, gi0 * gi0));
+            dR0 = fma(gam * h0, h0, fma(wmu2, fma(1.5 * gi0, gi0, t), dR0));
+            dR1 = fma(gam * h1, h1, fma(wmu2, fma(1.5 * gi1, gi1, t), dR1));
         }
         if (JAC) {
             const double gam = qs(6, c2, q);
@@ -928,7 +939,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
         if (act && c < nvalid) {
             if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, R0, R1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
-            if (JVP) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
+            if (JVP || MODE == M_DIAG) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
         }
         if (ntile < a.ntiles) gather_store<E, MODE>(smem + nst * S::STAGE, nxt);
     }
@@ -1151,7 +1162,7 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_OTF_JAC_WARPS : 1
         }
         if (act && c < nvalid) {
             if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, R0, R1);
-            if (JVP) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
+            if (JVP || MODE == M_DIAG) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
             if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
         }
         // the other input buffer was last read in the previous tile's per-QP phase

@@ -6,10 +6,12 @@
 // stokesfo_basal_friction); each Newton step solves J dU = -F with Jacobi-
 // preconditioned CG on the matrix-free operator J v = stokesfo_jvp(U; v) +
 // R_basal(v) (the basal term is linear in U), the Jacobi diagonal coming from
-// the element Jacobians (stokesfo_jacobian) and the basal face matrices; then
-// Armijo backtracking on ||F||.  J is symmetric positive definite once basal
-// friction removes the rigid null space.  Host loop in C++, vector algebra in
-// the small kernels below; the evaluator kernels are the product's own.
+// the diagonal-only evaluation (stokesfo_jacobian_diag) and the basal face
+// matrices; then Armijo backtracking on ||F||.  J is symmetric positive
+// definite once basal friction removes the rigid null space.  Host loop in
+// C++; the CG scalars stay on the device and blocks of CG iterations replay
+// as one CUDA graph; vector algebra in the small kernels below, the evaluator
+// kernels are the product's own.
 #pragma once
 #include "sfo_common.cuh"
 
@@ -35,6 +37,40 @@ __global__ void dot_kernel(int64_t n, const double *__restrict__ x, const double
     }
 }
 
+// CG scalars live on the device (slots of `s`), so a block of CG iterations runs
+// without host round trips and is captured once into a CUDA graph:
+//   s[RZ] = r.z, s[PAP] = p.Ap, s[RR] = r.r, s[RZN] = new r.z, s[ALPHA], s[BETA]
+enum { S_RZ = 0, S_PAP = 1, S_RR = 2, S_RZN = 3, S_ALPHA = 4, S_BETA = 5, S_IT = 6, S_SLOTS = 8 };
+
+// alpha = r.z / p.Ap (0 once the iteration has converged to p.Ap = 0: a no-op step)
+__global__ void cg_alpha_kernel(double *s) {
+    const double pap = s[S_PAP];
+    s[S_ALPHA] = (pap != 0.0 && isfinite(pap)) ? s[S_RZ] / pap : 0.0;
+}
+// beta = r.z_new / r.z; r.z <- r.z_new; hist[it] = r.r (the block's residual history)
+__global__ void cg_beta_kernel(double *s, double *hist) {
+    const double rz = s[S_RZ];
+    s[S_BETA] = (rz != 0.0 && isfinite(rz)) ? s[S_RZN] / rz : 0.0;
+    s[S_RZ] = s[S_RZN];
+    const int it = (int)s[S_IT];
+    hist[it] = s[S_RR];
+    s[S_IT] = it + 1;
+}
+// y += sign * (*a) * x
+__global__ void axpy_dev_kernel(int64_t n, const double *__restrict__ a, double sign, const double *__restrict__ x,
+                                double *__restrict__ y) {
+    const double al = sign * *a;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        y[i] = fma(al, x[i], y[i]);
+}
+// y = x + (*b) y
+__global__ void xpby_dev_kernel(int64_t n, const double *__restrict__ x, const double *__restrict__ b,
+                                double *__restrict__ y) {
+    const double be = *b;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        y[i] = fma(be, y[i], x[i]);
+}
+
 // y = a x + b y
 __global__ void axpby_kernel(int64_t n, double a, const double *__restrict__ x, double b, double *__restrict__ y) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -46,18 +82,6 @@ __global__ void jacobi_kernel(int64_t n, const double *__restrict__ r, const dou
                              double *__restrict__ z) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         z[i] = r[i] / d[i];
-}
-
-// diag[dof(c, r)] += J_cell[c][r][r]
-template <int N>
-__global__ void diag_cells_kernel(int64_t C, const int32_t *__restrict__ conn, const double *__restrict__ J,
-                                  double *__restrict__ diag) {
-    constexpr int ND = 2 * N;
-    const int64_t gid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (gid >= C * ND) return;
-    const int64_t c = gid / ND;
-    const int r = (int)(gid % ND);
-    atomicAdd(diag + 2 * (int64_t)conn[c * N + r / 2] + (r & 1), J[(c * ND + r) * ND + r]);
 }
 
 // diag[dof] += J_face[f][r][r] (bottom face nodes 0..NB-1 of the basal cell)

@@ -14,9 +14,28 @@ schedule runs with index_select / index_add_.
 """
 from __future__ import annotations
 
+import contextlib
+import os
+
 import numpy as np
 
 from . import stokesfo as S
+
+_PROFILE = os.environ.get("STOKESFO_PROFILE") == "1"
+
+
+@contextlib.contextmanager
+def nvtx(name: str):
+    """NVTX range (torch.cuda.nvtx) when STOKESFO_PROFILE=1, as the C ABI's entry points."""
+    if not _PROFILE:
+        yield
+        return
+    import torch
+    torch.cuda.nvtx.range_push(name)
+    try:
+        yield
+    finally:
+        torch.cuda.nvtx.range_pop()
 
 
 class LocalPart:
@@ -121,6 +140,10 @@ class P2PHalo:
 
     def begin(self):
         """Returns this step's R (or (R, Y)), already zero; zeroes the next step's buffers."""
+        with nvtx("halo.p2p.begin"):
+            return self._begin()
+
+    def _begin(self):
         b = self.t % 2
         self.buf[(self.t + 1) % 2].zero_()
         self.ctx.set_remote(self.rem, self.remtab, self.peers[b][0])
@@ -133,11 +156,12 @@ class P2PHalo:
         """Stream-ordered barrier: after it, every rank's kernel of this step is complete."""
         import torch
         import torch.distributed as dist
-        if self.gloo:
-            torch.cuda.synchronize(self.device)
-            dist.barrier()
-        else:
-            dist.all_reduce(self.token)
+        with nvtx("halo.p2p.barrier"):
+            if self.gloo:
+                torch.cuda.synchronize(self.device)
+                dist.barrier()
+            else:
+                dist.all_reduce(self.token)
         self.t += 1
         cur = self.buf[(self.t - 1) % 2]
         return cur[0] if self.fields == 1 else tuple(cur[f] for f in range(self.fields))
@@ -168,6 +192,10 @@ class Halo:
         return 2 * len(self.idx)
 
     def exchange(self, R):
+        with nvtx("halo.nccl.exchange"):
+            self._exchange(R)
+
+    def _exchange(self, R):
         import torch.distributed as dist
         if not self.idx:
             return

@@ -57,6 +57,7 @@ EXPORTS = [
     "stokesfo_set_remote", "stokesfo_set_remote_jvp", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
     "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
     "stokesfo_mesh_lateral_faces", "stokesfo_set_lateral", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
+    "stokesfo_jacobian_diag",
 ]
 
 
@@ -88,6 +89,8 @@ def _lib():
         L.stokesfo_jacobian.argtypes = [P, P, P, P, P]
         if hasattr(L, "stokesfo_jvp"):  # absent only in older builds loaded via STOKESFO_LIB
             L.stokesfo_jvp.argtypes = [P, P, P, P, P]
+        if hasattr(L, "stokesfo_jacobian_diag"):
+            L.stokesfo_jacobian_diag.argtypes = [P, P, P, P]
         if hasattr(L, "stokesfo_basal_friction"):
             L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
         if hasattr(L, "stokesfo_lateral_pressure"):
@@ -247,6 +250,14 @@ class StokesFO:
             _dev(t, torch.float64, (self.num_nodes, 2), n)
         _dev(R, torch.float64, (self.num_nodes, 2), "R")
         _check(_lib().stokesfo_jvp(self._h, _ptr(U), _ptr(X), _ptr(Y), _ptr(R)), "jvp")
+
+    def jacobian_diag(self, U, diag, R=None):
+        """diag += diagonal of the assembled Jacobian J(U) (no element matrices); optionally R += R(U)."""
+        import torch
+        for t, n in ((U, "U"), (diag, "diag")):
+            _dev(t, torch.float64, (self.num_nodes, 2), n)
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_jacobian_diag(self._h, _ptr(U), _ptr(diag), _ptr(R)), "jacobian_diag")
 
     def basal_friction(self, basal_cells, beta, U, R, J_face=None):
         """R += basal friction term on the bottom faces of basal_cells (int32 cuda);
