@@ -61,6 +61,8 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
     vals = 16 * nnz if op in ("jac_csr", "jac_global") else 0
     if geometry == "on_the_fly":
         return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32 + xy) + vals
+    if geometry == "compact":   # A_q = J_q^-T (9 doubles) + wM per QP instead of GradBF
+        return cells * (4 * N + 72 * Q + 8 * Q + 8 + J) + nodes * (16 + 8 + 32 + xy) + vals
     per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + J
     return cells * per_cell + nodes * (16 + 8 + 32 + xy) + vals
 
@@ -297,7 +299,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly"])
+    ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly", "compact"])
     ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jac_csr", "jac_global"],
                     help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
                          "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
@@ -660,7 +662,8 @@ def main():
                        "launch": ctx.launch_info()},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
-                         "kernel": ("eval_otf_kernel" if args.geometry == "on_the_fly" else "eval_kernel")
+                         "kernel": {"on_the_fly": "eval_otf_kernel", "compact": "eval_compact_kernel",
+                                    "stored": "eval_kernel"}[args.geometry]
                          + ("<Hex8," if elem == "hex8" else "<Wedge6,")
                          + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>",
                             "jac_global": "M_JAC> + csr_gather_kernel"}[args.op]

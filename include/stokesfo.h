@@ -68,8 +68,15 @@ typedef enum { STOKESFO_HEX8 = 0, STOKESFO_WEDGE6 = 1 } stokesfo_elem_t;
  *   ON_THE_FLY: recomputed per tile from the gathered node coordinates inside
  *               the evaluation kernels (40 streamed B/cell hex8; det J <= 0 is
  *               re-checked at every evaluation).
- * Both give the same results up to rounding (parity-tested at 1e-12). */
-typedef enum { STOKESFO_GEOMETRY_STORED = 0, STOKESFO_GEOMETRY_ON_THE_FLY = 1 } stokesfo_geometry_mode_t;
+ *   COMPACT:    precomputed once by stokesfo_create as A_q = J_q^-T and wMeasure
+ *               (680 B/cell hex8, 515 B/cell wedge6) and streamed at every
+ *               evaluation, which forms GradBF = A_q grad_xi phi_n in registers.
+ * All give the same results up to rounding (parity-tested at 1e-12). */
+typedef enum {
+    STOKESFO_GEOMETRY_STORED = 0,
+    STOKESFO_GEOMETRY_ON_THE_FLY = 1,
+    STOKESFO_GEOMETRY_COMPACT = 2
+} stokesfo_geometry_mode_t;
 
 typedef enum {
     STOKESFO_OK = 0,

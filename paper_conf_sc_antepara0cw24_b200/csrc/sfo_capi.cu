@@ -101,7 +101,22 @@ template <class E>
 int64_t ws_bytes(int64_t ncells, int64_t nnodes, int mode) {
     const int64_t ntiles = (ncells + E::TC - 1) / E::TC;
     if (mode == STOKESFO_GEOMETRY_ON_THE_FLY) return WS_HEADER + xyz4_bytes<E>(nnodes);
+    if (mode == STOKESFO_GEOMETRY_COMPACT) return WS_HEADER + ntiles * (int64_t)RecC<E>::BYTES;
     return WS_HEADER + ntiles * (int64_t)Rec<E>::BYTES;
+}
+
+template <class E, int MODE>
+int configure_compact(int *grid) {
+    auto fn = eval_compact_kernel<E, MODE>;
+    constexpr int bytes = CompactSmem<E, MODE>::BYTES;
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
+        return cuda_status();
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, bytes) != cudaSuccess) return cuda_status();
+    *grid = std::max(1, sms * std::max(1, per_sm));
+    return STOKESFO_OK;
 }
 
 template <class E, int MODE>
@@ -150,9 +165,17 @@ int create_impl(stokesfo_ctx *c) {
     c->TC = E::TC;
     c->ntiles = (c->d.num_cells + E::TC - 1) / E::TC;
     const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
-    c->rec_bytes = otf ? 0 : Rec<E>::BYTES;
+    const bool compact = c->mode == STOKESFO_GEOMETRY_COMPACT;
+    c->rec_bytes = otf ? 0 : (compact ? RecC<E>::BYTES : Rec<E>::BYTES);
     int st;
-    if (otf) {
+    if (compact) {
+        c->nstage_resid = c->nstage_jac = 2;
+        if ((st = configure_compact<E, M_RESID>(&c->grid_resid))) return st;
+        if ((st = configure_compact<E, M_JAC>(&c->grid_jac))) return st;
+        if ((st = configure_compact<E, M_JVP>(&c->grid_jvp))) return st;
+        if ((st = configure_compact<E, M_CSR>(&c->grid_csr))) return st;
+        if ((st = configure_compact<E, M_DIAG>(&c->grid_diag))) return st;
+    } else if (otf) {
         c->nstage_resid = c->nstage_jac = 0;
         st = configure_otf<E, M_RESID>(&c->grid_resid);
         if (st) return st;
@@ -193,6 +216,11 @@ int create_impl(stokesfo_ctx *c) {
             geometry_kernel<E, GEO_CHECK><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
                 c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.coords, nullptr, 0.0, nullptr, nullptr, nullptr,
                 c->err);
+        } else if (compact) {
+            const int64_t work = c->ntiles * E::TC * E::Q;
+            geometry_kernel<E, GEO_COMPACT><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
+                c->d.num_cells, c->d.num_nodes, c->d.conn, c->d.coords, c->d.flow_factor, c->d.k, c->recs, nullptr,
+                nullptr, c->err);
         } else {
             const int64_t work = c->ntiles * E::TC * E::Q;
             geometry_kernel<E, GEO_RECORDS><<<(unsigned)((work + bs - 1) / bs), bs, 0, c->stream>>>(
@@ -286,7 +314,10 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     constexpr int WPC = warps_per_cta<E, MODE>();  // eval_kernel only (the on-the-fly kernel: 1)
     const int grid = (int)std::min<int64_t>(g, otf ? c->ntiles : (c->ntiles + WPC - 1) / WPC);
     const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_RESID ? c->nstage_resid : 2);
-    if (otf)
+    if (c->mode == STOKESFO_GEOMETRY_COMPACT)
+        eval_compact_kernel<E, MODE><<<(int)std::min<int64_t>(g, c->ntiles), 32, CompactSmem<E, MODE>::BYTES,
+                                        c->stream>>>(a, jm);
+    else if (otf)
         eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
     else if (MODE != M_CSR && ns == 3)
         eval_kernel<E, MODE, 3><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 3>(), c->stream>>>(a, jm);
@@ -317,7 +348,8 @@ const char *stokesfo_strerror(int s) {
 int stokesfo_workspace_size(const stokesfo_desc_t *d, size_t *bytes) {
     SFO_RANGE("stokesfo_workspace_size");
     if (!d || !bytes || d->num_cells < 0) return STOKESFO_EINVAL;
-    if (d->geometry_mode != STOKESFO_GEOMETRY_STORED && d->geometry_mode != STOKESFO_GEOMETRY_ON_THE_FLY)
+    if (d->geometry_mode != STOKESFO_GEOMETRY_STORED && d->geometry_mode != STOKESFO_GEOMETRY_ON_THE_FLY &&
+        d->geometry_mode != STOKESFO_GEOMETRY_COMPACT)
         return STOKESFO_EINVAL;
     if (d->elem == STOKESFO_HEX8) *bytes = (size_t)ws_bytes<Hex8>(d->num_cells, d->num_nodes, d->geometry_mode);
     else if (d->elem == STOKESFO_WEDGE6) *bytes = (size_t)ws_bytes<Wedge6>(d->num_cells, d->num_nodes, d->geometry_mode);
@@ -614,6 +646,12 @@ int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure) {
             geometry_kernel<Wedge6, GEO_CANON><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->d.num_nodes, c->d.conn,
                                                                         c->d.coords, nullptr, 0.0, nullptr, grad_bf,
                                                                         w_measure, c->err);
+    } else if (c->mode == STOKESFO_GEOMETRY_COMPACT) {
+        if (c->N == 8)
+            geometry_export_compact_kernel<Hex8><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
+        else
+            geometry_export_compact_kernel<Wedge6><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf,
+                                                                            w_measure);
     } else if (c->N == 8) {
         geometry_export_kernel<Hex8><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->recs, grad_bf, w_measure);
     } else {

@@ -29,9 +29,18 @@ struct Hex8 {
     // lanes over (c,q)) and the per-node loads (fixed q, lanes over (c,j)) hit 16
     // distinct bank pairs per half-warp
     __host__ __device__ static constexpr int slot(int c, int n, int q) { return c * N + (n + q) % N; }
-    // gathered U/s per (cell, node) and per-QP scalars (f, cell, qp) in shared memory
+    // gathered U/s per (cell, node) in shared memory: node slot rotated by the cell, (n + c) mod 8, so
+    // that the per-QP phase's broadcast reads of one node (one address per cell) hit 4 distinct bank
+    // groups: 1 wavefront per LDS.128 / LDS.64 instead of 4 / 2 (cell pitch 128 B put every cell's
+    // node n in the same banks; ncu r2p1: the U reads were LDS.128 at 4 wavefronts)
     static constexpr int UPITCH = N;
-    __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * TC + c) * Q + q; }
+    __host__ __device__ static constexpr int uidx(int c, int n) { return c * UPITCH + ((n + c) & 7); }
+    // per-QP scalars (f, cell, qp): qp slot rotated by 2 c, so the node phase's broadcast (q, q+1)
+    // pair reads (one LDS.128 per field and QP pair, one address per cell) are conflict-free (1
+    // wavefront instead of 2) while the per-QP phase's stores stay conflict-free (each cell's 8
+    // lanes still fill its own 16 banks); q even => the pair (q, q+1) is adjacent and 16-B aligned
+    static constexpr bool QS_PAIRS = true;
+    __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * TC + c) * Q + ((q + 2 * c) & 7); }
 };
 #ifndef SFO_WEDGE_SLAB32
 #define SFO_WEDGE_SLAB32 1
@@ -61,6 +70,8 @@ struct Wedge6 {
     // odd 16-B cell pitch for the gathered U rows; per-QP scalars qp-major
     // (lanes (c, q) of the per-QP phase then write consecutive addresses)
     static constexpr int UPITCH = 7;
+    __host__ __device__ static constexpr int uidx(int c, int n) { return c * UPITCH + n; }
+    static constexpr bool QS_PAIRS = false;
     __host__ __device__ static constexpr int qsi(int f, int c, int q) { return (f * Q + q) * TC + c; }
 };
 
@@ -89,6 +100,28 @@ struct Rec {
     __host__ __device__ static constexpr int conn(int n, int c) { return c * N + n; }
     __host__ __device__ static constexpr int wm(int q, int c) { return q * TC + c; }
     __host__ __device__ static constexpr int g(int n, int q, int d, int c) { return (q * 3 + d) * SLAB + E::slot(c, n, q); }
+};
+
+// Compact per-tile record (STOKESFO_GEOMETRY_COMPACT): the geometry as
+// A_q = J_q^-T (9 doubles per (cell, qp), row-major, r = physical component, s =
+// reference direction) instead of GradBF; the evaluation forms GradBF_n(q) =
+// A_q grad_xi phi_n(xi_q) in registers (9 FMA per node).  Layout:
+//   conn  int32 [TC][N]
+//   kc    fp64  [TC]
+//   wm    fp64  [Q][TC]
+//   A     fp64  [9][Q][TC]      (k = 3 r + s; lanes (c, q) of one k read 32 consecutive doubles)
+// 2,720 B per hex8 tile (680 B/cell instead of 1,640), 2,576 B per wedge6 tile.
+template <class E>
+struct RecC {
+    static constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    static constexpr int CONN_OFF = 0;
+    static constexpr int KC_OFF = (int)round_up(N * TC * 4, 16);
+    static constexpr int WM_OFF = KC_OFF + (int)round_up(TC * 8, 16);
+    static constexpr int A_OFF = WM_OFF + (int)round_up(Q * TC * 8, 16);
+    static constexpr int BYTES = A_OFF + 9 * Q * TC * 8;
+    __host__ __device__ static constexpr int conn(int n, int c) { return c * N + n; }
+    __host__ __device__ static constexpr int wm(int q, int c) { return q * TC + c; }
+    __host__ __device__ static constexpr int a(int k, int q, int c) { return (k * Q + q) * TC + c; }
 };
 
 // Workspace: [0, 256) header (error flag), then ntiles records.

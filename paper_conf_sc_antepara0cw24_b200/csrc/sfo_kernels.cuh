@@ -91,7 +91,8 @@ __host__ __device__ __forceinline__ int gidx(int n, int q, int d, int c) {
 //   OUT = GEO_ALBANY:  GradBF, wGradBF, wBF component-major [entry][cell] at
 //                      grad_bf (NEXT-1 scratch, see sfo_albany.cuh)
 // ---------------------------------------------------------------------------
-enum { GEO_RECORDS = 0, GEO_CANON = 1, GEO_CHECK = 2, GEO_ALBANY = 3 };
+//   OUT = GEO_COMPACT: compact per-tile records (A_q = J_q^-T, wM; RecC)
+enum { GEO_RECORDS = 0, GEO_CANON = 1, GEO_CHECK = 2, GEO_ALBANY = 3, GEO_COMPACT = 4 };
 
 template <class E, int OUT>
 __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *__restrict__ conn,
@@ -99,29 +100,36 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
                                 char *__restrict__ recs, double *__restrict__ grad_bf, double *__restrict__ w_measure,
                                 int *__restrict__ err) {
     using R = Rec<E>;
+    using RC = RecC<E>;
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    constexpr bool REC = OUT == GEO_RECORDS || OUT == GEO_COMPACT;
     const int64_t ntiles = (ncells + TC - 1) / TC;
     const int64_t gid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    const int64_t nwork = (OUT == GEO_RECORDS ? ntiles * TC : ncells) * Q;
+    const int64_t nwork = (REC ? ntiles * TC : ncells) * Q;
     if (gid >= nwork) return;
     const int q = (int)(gid % Q);
     const int64_t cell = gid / Q;
     const int64_t tile = cell / TC;
     const int c = (int)(cell % TC);
-    char *rec = OUT == GEO_RECORDS ? recs + tile * (int64_t)R::BYTES : nullptr;
-    int32_t *rconn = reinterpret_cast<int32_t *>(rec + R::CONN_OFF);
-    double *rkc = reinterpret_cast<double *>(rec + R::KC_OFF);
-    double *rwm = reinterpret_cast<double *>(rec + R::WM_OFF);
+    char *rec = REC ? recs + tile * (int64_t)(OUT == GEO_COMPACT ? RC::BYTES : R::BYTES) : nullptr;
+    int32_t *rconn = reinterpret_cast<int32_t *>(rec + (OUT == GEO_COMPACT ? RC::CONN_OFF : R::CONN_OFF));
+    double *rkc = reinterpret_cast<double *>(rec + (OUT == GEO_COMPACT ? RC::KC_OFF : R::KC_OFF));
+    double *rwm = reinterpret_cast<double *>(rec + (OUT == GEO_COMPACT ? RC::WM_OFF : R::WM_OFF));
     double *rg = reinterpret_cast<double *>(rec + R::G_OFF);
+    double *ra = reinterpret_cast<double *>(rec + RC::A_OFF);
     if (cell >= ncells) {  // padding cells of the ragged last tile: zero record
-        if (OUT == GEO_RECORDS) {
+        if (REC) {
             if (q == 0) {
                 for (int n = 0; n < N; ++n) rconn[R::conn(n, c)] = 0;
                 rkc[c] = 0.0;
             }
             rwm[R::wm(q, c)] = 0.0;
-            for (int n = 0; n < N; ++n)
-                for (int d = 0; d < 3; ++d) rg[gidx<E>(n, q, d, c)] = 0.0;
+            if (OUT == GEO_COMPACT) {
+                for (int k = 0; k < 9; ++k) ra[RC::a(k, q, c)] = 0.0;
+            } else {
+                for (int n = 0; n < N; ++n)
+                    for (int d = 0; d < 3; ++d) rg[gidx<E>(n, q, d, c)] = 0.0;
+            }
         }
         return;
     }
@@ -135,7 +143,7 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
         }
     }
     if (bad_conn) atomicOr(err, ERR_CONN);
-    if (OUT == GEO_RECORDS && q == 0) {
+    if (REC && q == 0) {
         for (int n = 0; n < N; ++n) rconn[R::conn(n, c)] = nid[n];
         rkc[c] = kc_in ? kc_in[cell] : kscal;
     }
@@ -177,6 +185,14 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
     if (!(det > 0.0)) atomicOr(err, ERR_DETJ);
     if (OUT == GEO_CHECK) return;
     const double idet = 1.0 / det;
+    if (OUT == GEO_COMPACT) {  // A = J^-T = cof / det
+#pragma unroll
+        for (int r = 0; r < 3; ++r)
+#pragma unroll
+            for (int s2 = 0; s2 < 3; ++s2) ra[RC::a(3 * r + s2, q, c)] = cof[r][s2] * idet;
+        rwm[RC::wm(q, c)] = wq * det;
+        return;
+    }
 #pragma unroll
     for (int n = 0; n < N; ++n)
 #pragma unroll
@@ -222,6 +238,34 @@ __global__ void geometry_export_kernel(int64_t ncells, const char *__restrict__ 
     if (grad_bf)
         for (int n = 0; n < N; ++n)
             for (int d = 0; d < 3; ++d) grad_bf[((cell * N + n) * Q + q) * 3 + d] = rg[gidx<E>(n, q, d, c)];
+}
+
+// Export compact records -> canonical grad_bf = A_q grad_xi phi_n, w_measure (what the
+// compact evaluation forms in registers).
+template <class E>
+__global__ void geometry_export_compact_kernel(int64_t ncells, const char *__restrict__ recs,
+                                               double *__restrict__ grad_bf, double *__restrict__ w_measure) {
+    using RC = RecC<E>;
+    constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    const int64_t gid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (gid >= ncells * Q) return;
+    const int q = (int)(gid % Q);
+    const int64_t cell = gid / Q;
+    const char *rec = recs + (cell / TC) * (int64_t)RC::BYTES;
+    const int c = (int)(cell % TC);
+    const double *ra = reinterpret_cast<const double *>(rec + RC::A_OFF);
+    if (w_measure) w_measure[cell * Q + q] = reinterpret_cast<const double *>(rec + RC::WM_OFF)[RC::wm(q, c)];
+    if (!grad_bf) return;
+    double A[9];
+    for (int k = 0; k < 9; ++k) A[k] = ra[RC::a(k, q, c)];
+    double xq, yq, zq, wq;
+    qp_coords<E>(q, xq, yq, zq, wq);
+    for (int n = 0; n < N; ++n) {
+        double phi, d0, d1, d2;
+        basis<E>(n, xq, yq, zq, phi, d0, d1, d2);
+        for (int r = 0; r < 3; ++r)
+            grad_bf[((cell * N + n) * Q + q) * 3 + r] = fma(A[3 * r + 0], d0, fma(A[3 * r + 1], d1, A[3 * r + 2] * d2));
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -344,7 +388,17 @@ struct QsView {
     __device__ __forceinline__ double &operator()(int f, int c, int q) const {
         return f < SPLIT ? lo[E::qsi(f, c, q)] : hi[E::qsi(f - SPLIT, c, q)];
     }
+    // fields of QPs (q, q+1), q even, as one 16-B load (E::QS_PAIRS layouts keep the pair adjacent)
+    __device__ __forceinline__ double2 pair(int f, int c, int q) const {
+        return *reinterpret_cast<const double2 *>(&(*this)(f, c, q));
+    }
 };
+
+// per-QP scalar fields the per-node phase of a mode reads (JVP: 0-5, 7-14; residual: 0-5, 7, 8; else 0-8)
+template <int MODE>
+__host__ __device__ constexpr bool qs_used(int f) {
+    return MODE == M_JVP ? f != 6 : (MODE == M_RESID ? (f != 6 && f < 9) : f < 9);
+}
 
 // Per-QP scalars kept in registers (the residual-only and J.v modes of the
 // stored-geometry kernel, which exchange per-node partial sums instead).
@@ -443,14 +497,30 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const QS &qs, 
 #pragma unroll
         for (int k = 0; k <= K; ++k) Jb[k][0][0] = Jb[k][0][1] = Jb[k][1][0] = Jb[k][1][1] = 0.0;
     }
+    constexpr int NF = nqs<MODE>();
+    double sq[NF], sq1[NF];  // this QP's scalars; the next QP's when they arrive as a (q, q+1) pair
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
         if (q == Q / 2) pf();
-        const double b00 = qs(0, c2, q), b01 = qs(1, c2, q), b02 = qs(2, c2, q);
-        const double b11 = qs(3, c2, q), b12 = qs(4, c2, q);
+#pragma unroll
+        for (int f = 0; f < NF; ++f) {
+            if (!qs_used<MODE>(f)) {
+                sq[f] = 0.0;
+            } else if (E::QS_PAIRS && (q & 1) == 0) {
+                const double2 v = qs.pair(f, c2, q);
+                sq[f] = v.x;
+                sq1[f] = v.y;
+            } else if (E::QS_PAIRS) {
+                sq[f] = sq1[f];
+            } else {
+                sq[f] = qs(f, c2, q);
+            }
+        }
+        const double b00 = sq[0], b01 = sq[1], b02 = sq[2];
+        const double b11 = sq[3], b12 = sq[4];
         const double b10 = b01;
-        const double wmu2 = qs(5, c2, q);
-        const double wf0 = qs(7, c2, q), wf1 = qs(8, c2, q);
+        const double wmu2 = sq[5];
+        const double wf0 = sq[7], wf1 = sq[8];
         const double gi0 = rg[gidx<E>(i, q, 0, c2)];
         const double gi1 = rg[gidx<E>(i, q, 1, c2)];
         const double gi2 = rg[gidx<E>(i, q, 2, c2)];
@@ -461,9 +531,9 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const QS &qs, 
         R1 = fma(wf1, bfi[q], fma(wmu2, h1, R1));
         if (MODE == M_JVP) {
             // dR_(i,a) += wmu2 G_i . dbeta_a + gamma tau h_(i,a)
-            const double d00 = qs(9, c2, q), d01 = qs(10, c2, q), d02 = qs(11, c2, q);
-            const double d11 = qs(12, c2, q), d12 = qs(13, c2, q);
-            const double gt = qs(14, c2, q);
+            const double d00 = sq[9 % NF], d01 = sq[10 % NF], d02 = sq[11 % NF];
+            const double d11 = sq[12 % NF], d12 = sq[13 % NF];
+            const double gt = sq[14 % NF];
             const double e0 = fma(gi2, d02, fma(gi1, d01, gi0 * d00));
             const double e1 = fma(gi2, d12, fma(gi1, d11, gi0 * d01));
             dR0 = fma(gt, h0, fma(wmu2, e0, dR0));
@@ -472,13 +542,13 @@ __device__ __forceinline__ void node_accumulate(const double *rg, const QS &qs, 
         if (MODE == M_DIAG) {
             // J[(i,a),(i,a)] = wM 2 mu G_i^T B_aa G_i + gamma h_(i,a)^2,
             // B_00 = diag(2, 1/2, 1/2), B_11 = diag(1/2, 2, 1/2) (the k = 0 block's diagonal)
-            const double gam = qs(6, c2, q);
+            const double gam = sq[6];
             const double t = 0.5 * fma(gi2, gi2, fma(gi1, gi1, gi0 * gi0));
             dR0 = fma(gam * h0, h0, fma(wmu2, fma(1.5 * gi0, gi0, t), dR0));
             dR1 = fma(gam * h1, h1, fma(wmu2, fma(1.5 * gi1, gi1, t), dR1));
         }
         if (JAC) {
-            const double gam = qs(6, c2, q);
+            const double gam = sq[6];
             const double gh0 = gam * h0, gh1 = gam * h1;
             const double w0 = wmu2 * gi0, w1 = wmu2 * gi1, w2 = wmu2 * gi2;
             const double m00x = fma(2.0, w0, gh0 * b00), m00y = fma(0.5, w1, gh0 * b01),
@@ -725,7 +795,7 @@ __device__ __forceinline__ void gather_store(char *stage, const Gathered &v) {
     using S = EvalSmem<E, MODE>;
     const int l = threadIdx.x & 31;
     if (l < E::TC * E::N) {
-        const int e = E::lane_cell(l) * E::UPITCH + E::lane_sub(l);  // [cell][node]
+        const int e = E::uidx(E::lane_cell(l), E::lane_sub(l));  // [cell][node]
         reinterpret_cast<double2 *>(stage + S::U_OFF)[e] = v.u;
         reinterpret_cast<double *>(stage + S::S_OFF)[e] = v.s;
         if (MODE == M_JVP) reinterpret_cast<double2 *>(stage + S::X_OFF)[e] = v.x;
@@ -815,15 +885,16 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
                     gq[n][1] = g1;
                     gq[n][2] = g2;
                 }
-                const double2 uv = Us[c * E::UPITCH + n];
+                const int e = E::uidx(c, n);
+                const double2 uv = Us[e];
                 ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
                 vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
                 if (have_s) {
-                    const double sn = ss[c * E::UPITCH + n];
+                    const double sn = ss[e];
                     gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
                 }
                 if (JVP) {
-                    const double2 xv = Xs[c * E::UPITCH + n];
+                    const double2 xv = Xs[e];
                     dg[0] = fma(xv.x, g0, dg[0]); dg[1] = fma(xv.x, g1, dg[1]); dg[2] = fma(xv.x, g2, dg[2]);
                     dg[3] = fma(xv.y, g0, dg[3]); dg[4] = fma(xv.y, g1, dg[4]); dg[5] = fma(xv.y, g2, dg[5]);
                 }
@@ -942,6 +1013,278 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
             if (JVP || MODE == M_DIAG) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
         }
         if (ntile < a.ntiles) gather_store<E, MODE>(smem + nst * S::STAGE, nxt);
+    }
+    if (JAC && l == 0) bulk_wait0();
+}
+
+// ---- G3/G4 with compact stored geometry (A_q = J_q^-T streamed per tile) ----
+// The stored kernel's TMA record ring and register gather, with the compact
+// record (RecC): the per-QP phase forms GradBF_n(q) = A_q grad_xi phi_n(xi_q)
+// in registers (reference gradients at the lane's QP from its QP coordinates)
+// and, for the tangent modes, stores it to a per-warp GradBF region in the
+// stored kernel's slot layout, so the per-node phase is unchanged.  680 B/cell
+// of geometry instead of 1,640 (hex8): the evaluation moves 26% fewer HBM bytes
+// for 9 FMA per (node, QP) more.  Shared memory per warp: 2 record stages +
+// GradBF region + per-QP scalars; the element-Jacobian staging overlays the
+// GradBF + scalar regions (as in the on-the-fly kernel), so the next record can
+// land while the TMA store drains.
+template <class E, int MODE>
+struct CompactSmem {
+    static constexpr int N = E::N, Q = E::Q, TC = E::TC, SLAB = E::SLAB;
+    static constexpr int REC = RecC<E>::BYTES;
+    static constexpr int U_OFF = (int)round_up(REC, 16);                         // double2 [TC][UPITCH]
+    static constexpr int S_OFF = U_OFF + TC * E::UPITCH * 16;                      // double  [TC][UPITCH]
+    static constexpr int X_OFF = (int)round_up(S_OFF + TC * E::UPITCH * 8, 16);   // double2 [TC][UPITCH] (M_JVP)
+    static constexpr int IN_BYTES = X_OFF + (MODE == M_JVP ? TC * E::UPITCH * 16 : 0);
+    static constexpr int STAGE = (int)round_up(IN_BYTES, 128);
+    static constexpr bool PSUM = MODE == M_RESID || MODE == M_JVP;
+    static constexpr int G_BYTES = Q * 3 * SLAB * 8;                               // GradBF (or partial sums)
+    static constexpr int OFF_G = 2 * STAGE;
+    static constexpr int OFF_QS = OFF_G + G_BYTES;                                 // double [NQS][TC][Q]
+    static constexpr int QS_BYTES = PSUM ? 0 : nqs<MODE>() * TC * Q * 8;
+    static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;         // J staging over G + qs
+    static constexpr int TAIL = (G_BYTES + QS_BYTES > J_BYTES ? G_BYTES + QS_BYTES : J_BYTES);
+    static constexpr int OFF_BAR = (int)round_up(OFF_G + TAIL, 8);
+    static constexpr int BYTES = OFF_BAR + 2 * 8;
+    static_assert(!PSUM || psum_bytes<E>() <= G_BYTES, "partial sums overlay the GradBF region");
+    static_assert(U_OFF % 16 == 0 && X_OFF % 16 == 0 && STAGE % 128 == 0 && OFF_G % 128 == 0 && OFF_QS % 16 == 0,
+                  "alignment");
+};
+
+template <class E, int MODE>
+__device__ __forceinline__ Gathered gather_load_c(const char *stage, const double *U, const double *surface,
+                                                  bool have_s, const double *X) {
+    using R = RecC<E>;
+    Gathered v{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
+    const int l = threadIdx.x & 31;
+    if (l < E::TC * E::N) {
+        const int c = E::lane_cell(l), n = E::lane_sub(l);
+        const int32_t g = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF)[R::conn(n, c)];
+        v.u = __ldg(reinterpret_cast<const double2 *>(U) + g);
+        if (have_s) v.s = __ldg(surface + g);
+        if (MODE == M_JVP) v.x = __ldg(reinterpret_cast<const double2 *>(X) + g);
+    }
+    return v;
+}
+template <class E, int MODE>
+__device__ __forceinline__ void gather_store_c(char *stage, const Gathered &v) {
+    using S = CompactSmem<E, MODE>;
+    const int l = threadIdx.x & 31;
+    if (l < E::TC * E::N) {
+        const int e = E::uidx(E::lane_cell(l), E::lane_sub(l));
+        reinterpret_cast<double2 *>(stage + S::U_OFF)[e] = v.u;
+        reinterpret_cast<double *>(stage + S::S_OFF)[e] = v.s;
+        if (MODE == M_JVP) reinterpret_cast<double2 *>(stage + S::X_OFF)[e] = v.x;
+    }
+}
+
+#ifndef SFO_COMPACT_JAC_WARPS
+#define SFO_COMPACT_JAC_WARPS 12
+#endif
+template <class E, int MODE>
+__global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS : 16))
+    eval_compact_kernel(EvalArgs a, const __grid_constant__ CUtensorMap jmap) {
+    constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
+    static_assert(N == Q, "lane mappings assume N == Q");
+    using R = RecC<E>;
+    using S = CompactSmem<E, MODE>;
+    extern __shared__ __align__(128) char smem[];
+    double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
+    const QsView<E, nqs<MODE>()> qs{reinterpret_cast<double *>(smem + S::OFF_QS), nullptr};
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
+    const int l = threadIdx.x & 31;
+    const bool act = l < TC * N;
+    const int c = act ? E::lane_cell(l) : TC, s = act ? E::lane_sub(l) : 0;  // (cell, node-or-qp)
+    const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
+    const int64_t vb = blockIdx.x, vg = gridDim.x;
+
+    uint64_t pol_stream = 0;
+    if (l == 0) {
+        pol_stream = policy_evict_first();
+        for (int k = 0; k < 2; ++k) mbar_init(&bar[k], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (int k = 0; k < 2; ++k) {
+            const int64_t tile = vb + (int64_t)k * vg;
+            if (tile < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[k], R::BYTES);
+                bulk_g2s(smem + k * S::STAGE, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[k], pol_stream);
+            }
+        }
+    }
+    __syncwarp();
+    if (vb < a.ntiles) {
+        mbar_wait(&bar[0], 0);
+        gather_store_c<E, MODE>(smem, gather_load_c<E, MODE>(smem, a.U, a.surface, have_s, a.X));
+    }
+    double xq, yq, zq, wq;  // this lane's QP (per-QP phase)
+    qp_coords<E>(act ? s : 0, xq, yq, zq, wq);
+    double bfi[Q];
+    basis_row<E>(act ? s : 0, bfi);
+    double bq[N];  // phi_n at this lane's QP, every n (partial-sum modes)
+    {
+        double dx, dy, dz;
+#pragma unroll
+        for (int n = 0; n < N; ++n) basis<E>(n, xq, yq, zq, bq[n], dx, dy, dz);
+    }
+
+    int it = 0;
+    for (int64_t tile = vb; tile < a.ntiles; tile += vg, ++it) {
+        const int st = it & 1;
+        char *stage = smem + st * S::STAGE;
+        const int32_t *rconn = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF);
+        const double *rkc = reinterpret_cast<const double *>(stage + R::KC_OFF);
+        const double *rwm = reinterpret_cast<const double *>(stage + R::WM_OFF);
+        const double *ra = reinterpret_cast<const double *>(stage + R::A_OFF);
+        const double2 *Us = reinterpret_cast<const double2 *>(stage + S::U_OFF);
+        const double *ss = reinterpret_cast<const double *>(stage + S::S_OFF);
+        const double2 *Xs = reinterpret_cast<const double2 *>(stage + S::X_OFF);
+        const int64_t cell0 = tile * TC;
+        const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
+
+        if (JAC && l == 0) bulk_wait_read0();  // the previous tile's J staging (over G + qs) has been read
+        __syncwarp();                          // + this tile's gathered U, s are visible
+        const int32_t gnode = act ? rconn[R::conn(s, c)] : 0;
+
+        // ---- per-QP phase: lane <-> (cell c, qp s); GradBF = A grad_xi phi in registers ----
+        double gq[S::PSUM ? N : 1][3];
+        double qv[S::PSUM ? 15 : 1];
+        if (act) {
+            const int q = s;
+            double A[9];
+#pragma unroll
+            for (int k = 0; k < 9; ++k) A[k] = ra[R::a(k, q, c)];
+            double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+            double dg[6] = {0, 0, 0, 0, 0, 0};
+#pragma unroll
+            for (int n = 0; n < N; ++n) {
+                double phi, d0, d1, d2;
+                basis<E>(n, xq, yq, zq, phi, d0, d1, d2);
+                const double g0 = fma(A[0], d0, fma(A[1], d1, A[2] * d2));
+                const double g1 = fma(A[3], d0, fma(A[4], d1, A[5] * d2));
+                const double g2 = fma(A[6], d0, fma(A[7], d1, A[8] * d2));
+                if constexpr (S::PSUM) {
+                    gq[n][0] = g0;
+                    gq[n][1] = g1;
+                    gq[n][2] = g2;
+                } else {
+                    rg[gidx<E>(n, q, 0, c)] = g0;
+                    rg[gidx<E>(n, q, 1, c)] = g1;
+                    rg[gidx<E>(n, q, 2, c)] = g2;
+                }
+                const int e = E::uidx(c, n);
+                const double2 uv = Us[e];
+                ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
+                vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
+                if (have_s) {
+                    const double sn = ss[e];
+                    gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
+                }
+                if (JVP) {
+                    const double2 xv = Xs[e];
+                    dg[0] = fma(xv.x, g0, dg[0]); dg[1] = fma(xv.x, g1, dg[1]); dg[2] = fma(xv.x, g2, dg[2]);
+                    dg[3] = fma(xv.y, g0, dg[3]); dg[4] = fma(xv.y, g1, dg[4]); dg[5] = fma(xv.y, g2, dg[5]);
+                }
+            }
+            if constexpr (S::PSUM)
+                qp_tail<E, MODE>(a, RegQs{qv}, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx,
+                                 vy, vz, gs0, gs1, dg);
+            else
+                qp_tail<E, MODE>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy,
+                                 vz, gs0, gs1, dg);
+        }
+        __syncwarp();  // the stage (record, U, s) is consumed: refill it with the record two tiles ahead
+        if (l == 0) {
+            const int64_t nt = tile + 2 * vg;
+            if (nt < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[st], R::BYTES);
+                bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
+            }
+        }
+
+        // ---- per-node phase (+ gather of the next tile at q = Q/2) ----
+        const int64_t ntile = tile + vg;
+        const int nst = (it + 1) & 1;
+        Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
+        auto prefetch = [&]() {
+            if (ntile < a.ntiles) {
+                mbar_wait(&bar[nst], (uint32_t)(((it + 1) >> 1) & 1));
+                nxt = gather_load_c<E, MODE>(smem + nst * S::STAGE, a.U, a.surface, have_s, a.X);
+            }
+        };
+        double R0 = 0.0, R1 = 0.0, dR0 = 0.0, dR1 = 0.0;
+        double Jb[N / 2 + 1][2][2];
+        uint64_t srow = 0;
+        longlong2 rp = make_longlong2(0, 0);
+        if (CSR) csr_row_load(a, cell0 + c, gnode, act && c < nvalid, srow, rp, N, s);
+        if constexpr (S::PSUM) {
+            // partial sums over the (unused) GradBF region
+            double2 *P = reinterpret_cast<double2 *>(rg);
+            if (act) {
+                const double w = qv[5];
+                const double s00 = w * qv[0], s01 = w * qv[1], s02 = w * qv[2], s11 = w * qv[3], s12 = w * qv[4];
+#pragma unroll
+                for (int n = 0; n < N; ++n) {
+                    const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
+                    P[psum_idx<E>(c, n, s)] = make_double2(fma(qv[7], bq[n], fma(g2, s02, fma(g1, s01, g0 * s00))),
+                                                           fma(qv[8], bq[n], fma(g2, s12, fma(g1, s11, g0 * s01))));
+                }
+            }
+            __syncwarp();
+            prefetch();
+            if (act) {
+#pragma unroll
+                for (int k = 0; k < Q; ++k) {
+                    const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
+                    R0 += v.x;
+                    R1 += v.y;
+                }
+            }
+            if (JVP) {
+                __syncwarp();
+                if (act) {
+                    const double w = qv[5], gt = qv[14];
+                    const double d00 = fma(w, qv[9], gt * qv[0]), d01 = fma(w, qv[10], gt * qv[1]);
+                    const double d02 = fma(w, qv[11], gt * qv[2]), d11 = fma(w, qv[12], gt * qv[3]);
+                    const double d12 = fma(w, qv[13], gt * qv[4]);
+#pragma unroll
+                    for (int n = 0; n < N; ++n) {
+                        const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
+                        P[psum_idx<E>(c, n, s)] = make_double2(fma(g2, d02, fma(g1, d01, g0 * d00)),
+                                                               fma(g2, d12, fma(g1, d11, g0 * d01)));
+                    }
+                }
+                __syncwarp();
+                if (act) {
+#pragma unroll
+                    for (int k = 0; k < Q; ++k) {
+                        const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
+                        dR0 += v.x;
+                        dR1 += v.y;
+                    }
+                }
+            }
+        } else {
+            if (act) node_accumulate<E, MODE>(rg, qs, c, s, bfi, R0, R1, Jb, dR0, dR1, prefetch);
+            else prefetch();
+            if (forms_jac<MODE>()) ksplit_exchange<E>(Jb, c, s, act);
+        }
+        __syncwarp();  // every lane is done with G and qs
+        if (CSR) csr_scatter<E>(a.csr_vals, c, s, act && c < nvalid, srow, rp, Jb);
+        if (JAC) {
+            if (act) stage_J<E>(rg, c, s, Jb);
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (l == 0)
+                store_J<E>(a.J_cell, cell0, nvalid, reinterpret_cast<const char *>(rg), pol_stream,
+                           a.use_jmap ? &jmap : nullptr);
+        }
+        if (act && c < nvalid) {
+            if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, R0, R1);
+            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + c) * N + s) * 2) = make_double2(R0, R1);
+            if (JVP || MODE == M_DIAG) scatter_node(a.rem, a.remtab, a.Y, a.peers_y, gnode, dR0, dR1);
+        }
+        if (ntile < a.ntiles) gather_store_c<E, MODE>(smem + nst * S::STAGE, nxt);
     }
     if (JAC && l == 0) bulk_wait0();
 }

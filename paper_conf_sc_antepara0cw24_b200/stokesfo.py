@@ -20,7 +20,7 @@ NODES = {HEX8: 8, WEDGE6: 6}
 QPS = {HEX8: 8, WEDGE6: 6}
 ABI_VERSION = 1
 
-GEOMETRY = {"stored": 0, "on_the_fly": 1}
+GEOMETRY = {"stored": 0, "on_the_fly": 1, "compact": 2}
 STATUS = {0: "OK", 1: "EINVAL", 2: "EMESH", 3: "ECUDA", 4: "ENOMEM", 5: "EUNSUPPORTED"}
 
 

@@ -12,7 +12,7 @@ pytestmark = pytest.mark.gpu
 TOL = 1e-12
 
 
-@pytest.mark.parametrize("geometry", ["stored", "on_the_fly"])
+@pytest.mark.parametrize("geometry", ["stored", "on_the_fly", "compact"])
 @pytest.mark.parametrize("cfg", ["C3", "C4", "C5"])
 def test_fullsize_sampled_parity(cfg, geometry):
     import torch

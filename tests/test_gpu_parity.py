@@ -29,7 +29,7 @@ def _t(torch, a, dtype=None):
     return torch.from_numpy(a).to("cuda") if dtype is None else torch.from_numpy(a).to("cuda", dtype)
 
 
-GEOMS = ["stored", "on_the_fly"]
+GEOMS = ["stored", "on_the_fly", "compact"]
 
 
 def _setup(torch, elem="hex8", n=16, L=5, drop=0, kind="random", scalar_k=False, surface=True, geometry="stored"):

@@ -43,7 +43,7 @@ TOL = 1e-12
 RHO_G = 8.927
 DELTAS = [1e-10, 1e-6, 1.0]
 FIELDS = ["zero", "rigid", "linear", "scaled"]
-GEOMS = ["stored", "on_the_fly"]
+GEOMS = ["stored", "on_the_fly", "compact"]
 
 
 @pytest.fixture(scope="module")
