@@ -55,9 +55,8 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
         xy = 16
     if op == "jac_global":
         # jacobian (J_cell written) + pull assembly (DESIGN §6 NEXT-2): J_cell read again, per cell the
-        # slot row 8N and incidence 4N, per node rowptr pair 16 + incidence pointer 8, CSR values read + written;
-        # compact geometry = the fused launch (stokesfo_jacobian_global): the element matrices stay in L2
-        J = (0 if geometry == "compact" else 2 * 8 * (2 * N) ** 2) + 8 * N + 4 * N
+        # slot row 8N and incidence 4N, per node rowptr pair 16 + incidence pointer 8, CSR values read + written
+        J = 2 * 8 * (2 * N) ** 2 + 8 * N + 4 * N
         xy = 24
     vals = 16 * nnz if op in ("jac_csr", "jac_global") else 0
     if geometry == "on_the_fly":
@@ -418,8 +417,6 @@ def main():
             ctx.jacobian(Uc, J, R=Rc)
         elif args.op == "jac_csr":
             ctx.jacobian_csr(Uc, vals, R=Rc)
-        elif args.op == "jac_global" and args.geometry == "compact":   # one launch, J tiles through L2
-            ctx.jacobian_global(Uc, vals, R=Rc, J_scratch=J)
         elif args.op == "jac_global":   # element matrices, then the atomic-free pull assembly into CSR
             ctx.jacobian(Uc, J, R=Rc)
             ctx.scatter_assemble(J_cell=J, csr_vals=vals)
@@ -669,19 +666,16 @@ def main():
                                     "stored": "eval_kernel"}[args.geometry]
                          + ("<Hex8," if elem == "hex8" else "<Wedge6,")
                          + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>",
-                            "jac_global": ("M_GLOBAL>" if args.geometry == "compact"
-                                           else "M_JAC> + csr_gather_kernel")}[args.op]
+                            "jac_global": "M_JAC> + csr_gather_kernel"}[args.op]
                          + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
                             "jvp": " (stokesfo_jvp)", "jac_csr": " (stokesfo_jacobian_csr)",
-                            "jac_global": (" (stokesfo_jacobian_global: J tiles staged through L2, one launch)"
-                                           if args.geometry == "compact" else
-                                           " (stokesfo_jacobian + stokesfo_scatter_assemble, both timed)")}[args.op],
+                            "jac_global": " (stokesfo_jacobian + stokesfo_scatter_assemble, both timed)"}[args.op],
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src,
                          "live_copy_gbs": live_copy,
                          "note": "live_copy_gbs: torch device-to-device copy of 2 GiB on this box before the timed "
                                  "region (context for box-to-box variance; not the denominator)"},
             "achieved_hbm_gbs": achieved,
-            "gpu_launches": args.steps * ((2 if args.op == "jac_global" and args.geometry != "compact" else 1)
+            "gpu_launches": args.steps * ((2 if args.op == "jac_global" else 1)
                                           + (halo.launches_per_exchange * (2 if args.op == "jvp" else 1)
                                              if halo else 0)),
             "halo": halo_mode,

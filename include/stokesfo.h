@@ -225,25 +225,6 @@ int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots);
  * (+=); U, R: dev [num_nodes][2].  Summation order is unspecified (atomics). */
 int stokesfo_jacobian_csr(stokesfo_ctx *c, const double *U, double *csr_vals, double *R);
 
-/* NEXT-2 fused global matrix through L2 (COMPACT geometry mode, single GPU):
- * csr_vals += the assembled Jacobian and R += the residual (optional) in ONE
- * launch, without atomics on the matrix.  Element Jacobians are staged in L2:
- * every tile's J goes to J_scratch (dev [C][2N][2N], 128-B aligned; its content
- * is undefined afterwards), and the warp that completes the last tile around a
- * node pulls that node's two CSR rows from the J tiles (still in L2) and adds
- * them to csr_vals with plain read-modify-writes; consumed J tiles are discarded
- * from L2 (no write-back; STOKESFO_GLOBAL_DISCARD=0 keeps them).  Rows are
- * summed in ascending cell order, so the result is bitwise that of
- * stokesfo_jacobian + stokesfo_scatter_assemble.  Requires stokesfo_csr_slots
- * and a work buffer (caller-owned, 256-B aligned, work_size bytes) prepared
- * once by _setup (per-node / per-tile completion counters; reset from it at
- * every call).  EUNSUPPORTED for other geometry modes or nodes with more than
- * 64 neighbour nodes; EINVAL with a peer table attached. */
-int stokesfo_jacobian_global_work_size(stokesfo_ctx *c, size_t *bytes);
-int stokesfo_jacobian_global_setup(stokesfo_ctx *c, void *work);
-int stokesfo_jacobian_global(stokesfo_ctx *c, const double *U, double *J_scratch, double *csr_vals, double *R,
-                             void *work);
-
 /* Export the precomputed geometry in the canonical layout:
  * grad_bf dev [C][N][Q][3], w_measure dev [C][Q] (either may be NULL). */
 int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure);

@@ -27,7 +27,7 @@ struct stokesfo_ctx {
     char *recs;            // device records (full or light)
     double4 *xyz4;         // node coordinates (on-the-fly geometry mode)
     int mode;              // stokesfo_geometry_mode_t
-    int grid_resid, grid_jac, grid_jvp, grid_csr, grid_diag, grid_global = 0;
+    int grid_resid, grid_jac, grid_jvp, grid_csr, grid_diag;
     int rec_bytes;
     int nstage_resid, nstage_jac;  // TMA record ring depth of the eval kernels
     const int32_t *rem = nullptr;     // fused halo over peer memory (stokesfo_set_remote)
@@ -175,7 +175,6 @@ int create_impl(stokesfo_ctx *c) {
         if ((st = configure_compact<E, M_JVP>(&c->grid_jvp))) return st;
         if ((st = configure_compact<E, M_CSR>(&c->grid_csr))) return st;
         if ((st = configure_compact<E, M_DIAG>(&c->grid_diag))) return st;
-        if ((st = configure_compact<E, M_GLOBAL>(&c->grid_global))) return st;
     } else if (otf) {
         c->nstage_resid = c->nstage_jac = 0;
         st = configure_otf<E, M_RESID>(&c->grid_resid);
@@ -522,112 +521,6 @@ int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, d
 #define CALL(E) eval_impl<E, M_JVP>(c, U, nullptr, nullptr, R, nullptr, X, Y)
     return DISPATCH(c, CALL);
 #undef CALL
-}
-
-}  // extern "C"
-
-namespace {
-struct GlobalWork {
-    int32_t *node_cnt0, *tile_cnt0, *node_cnt, *tile_cnt;
-    int64_t bytes;
-};
-GlobalWork global_layout(const stokesfo_ctx *c, char *base) {
-    GlobalWork w{};
-    int64_t off = 0;
-    auto take = [&](int64_t n) {
-        int32_t *p = reinterpret_cast<int32_t *>(base + off);
-        off += round_up(std::max<int64_t>(n, 1) * 4, 256);
-        return p;
-    };
-    w.node_cnt0 = take(c->d.num_nodes);
-    w.tile_cnt0 = take(c->ntiles);
-    w.node_cnt = take(c->d.num_nodes);
-    w.tile_cnt = take(c->ntiles);
-    w.bytes = off;
-    return w;
-}
-
-template <class E>
-int global_impl(stokesfo_ctx *c, const double *U, double *J, double *vals, double *R, const GlobalWork &w) {
-    EvalArgs a{};
-    a.recs = c->recs;
-    a.kscal = c->d.k;
-    a.err = c->err;
-    a.ntiles = c->ntiles;
-    a.ncells = c->d.num_cells;
-    a.U = U;
-    a.surface = c->d.surface;
-    a.force_qp = c->d.force_qp;
-    a.rho_g = c->d.rho_g;
-    a.delta = c->d.delta;
-    a.R = R;
-    a.J_cell = J;
-    a.rowptr = c->rowptr;
-    a.slots = c->slots;
-    a.csr_vals = vals;
-    a.node_cnt = w.node_cnt;
-    a.tile_cnt = w.tile_cnt;
-    a.inc_ptr = c->inc_ptr;
-    a.inc = c->inc;
-    static const bool discard = !(getenv("STOKESFO_GLOBAL_DISCARD") && atoi(getenv("STOKESFO_GLOBAL_DISCARD")) == 0);
-    a.discard = discard ? 1 : 0;
-    a.use_jmap = wedge_jmap<E>(c, J) ? 1 : 0;
-    const CUtensorMap jm = a.use_jmap ? c->jmap : CUtensorMap{};
-    const int grid = (int)std::min<int64_t>(c->grid_global, c->ntiles);
-    eval_compact_kernel<E, M_GLOBAL><<<grid, 32, CompactSmem<E, M_GLOBAL>::BYTES, c->stream>>>(a, jm);
-    return cuda_status();
-}
-}  // namespace
-
-extern "C" {
-
-int stokesfo_jacobian_global_work_size(stokesfo_ctx *c, size_t *bytes) {
-    SFO_RANGE("stokesfo_jacobian_global_work_size");
-    if (!c || !bytes) return STOKESFO_EINVAL;
-    *bytes = (size_t)global_layout(c, nullptr).bytes;
-    return STOKESFO_OK;
-}
-
-int stokesfo_jacobian_global_setup(stokesfo_ctx *c, void *work) {
-    SFO_RANGE("stokesfo_jacobian_global_setup");
-    if (!c || !work || !aligned(work, 256)) return STOKESFO_EINVAL;
-    if (c->mode != STOKESFO_GEOMETRY_COMPACT) return STOKESFO_EUNSUPPORTED;
-    if (!c->slots || !c->inc || !c->rowptr) return STOKESFO_EINVAL;  // needs stokesfo_csr_slots
-    if (c->csr_maxdeg > CSR_GATHER_MAXDEG) return STOKESFO_EUNSUPPORTED;
-    GlobalWork w = global_layout(c, reinterpret_cast<char *>(work));
-    if (cudaMemsetAsync(w.node_cnt0, 0, (size_t)c->d.num_nodes * 4, c->stream) != cudaSuccess) return cuda_status();
-    if (c->ntiles > 0) {
-        const int bs = 128;
-        const unsigned g = (unsigned)((c->ntiles + bs - 1) / bs);
-        if (c->N == 8)
-            global_counts_kernel<8, Hex8::TC><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->ntiles, c->d.conn,
-                                                                       w.node_cnt0, w.tile_cnt0);
-        else
-            global_counts_kernel<6, Wedge6::TC><<<g, bs, 0, c->stream>>>(c->d.num_cells, c->ntiles, c->d.conn,
-                                                                         w.node_cnt0, w.tile_cnt0);
-    }
-    return cuda_status();
-}
-
-int stokesfo_jacobian_global(stokesfo_ctx *c, const double *U, double *J_scratch, double *csr_vals, double *R,
-                             void *work) {
-    SFO_RANGE("stokesfo_jacobian_global");
-    if (!c) return STOKESFO_EINVAL;
-    if (c->d.num_cells == 0) return STOKESFO_OK;
-    if (c->mode != STOKESFO_GEOMETRY_COMPACT) return STOKESFO_EUNSUPPORTED;
-    if (!c->slots || !c->inc || !c->rowptr || c->rem) return STOKESFO_EINVAL;
-    if (c->csr_maxdeg > CSR_GATHER_MAXDEG) return STOKESFO_EUNSUPPORTED;
-    if (!U || !J_scratch || !csr_vals || !work || !aligned(U, 16) || !aligned(J_scratch, 128) ||
-        !aligned(csr_vals, 16) || !aligned(work, 256) || (R && !aligned(R, 16)))
-        return STOKESFO_EINVAL;
-    GlobalWork w = global_layout(c, reinterpret_cast<char *>(work));
-    if (cudaMemcpyAsync(w.node_cnt, w.node_cnt0, (size_t)c->d.num_nodes * 4, cudaMemcpyDeviceToDevice, c->stream) !=
-            cudaSuccess ||
-        cudaMemcpyAsync(w.tile_cnt, w.tile_cnt0, (size_t)c->ntiles * 4, cudaMemcpyDeviceToDevice, c->stream) !=
-            cudaSuccess)
-        return cuda_status();
-    return c->N == 8 ? global_impl<Hex8>(c, U, J_scratch, csr_vals, R, w)
-                     : global_impl<Wedge6>(c, U, J_scratch, csr_vals, R, w);
 }
 
 int stokesfo_jacobian_diag(stokesfo_ctx *c, const double *U, double *diag, double *R) {

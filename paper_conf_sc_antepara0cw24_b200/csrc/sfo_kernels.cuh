@@ -314,13 +314,6 @@ struct EvalArgs {
     const uint64_t *slots;    // [C][N] rows of N uint8 slots (8-byte pitch)
     double *csr_vals;         // [nnz] (+=)
     int use_jmap;             // wedge6 M_JAC: J tile stored through the kernel's tensor-map parameter
-    // NEXT-2 fused global matrix (M_GLOBAL, compact geometry): J tiles pass through L2 (J_cell is scratch);
-    // the warp that completes the last tile around a node assembles that node's two CSR rows
-    int32_t *node_cnt;        // [nodes] tiles still to complete around each node (reset per call)
-    int32_t *tile_cnt;        // [ntiles] node assemblies still to read each tile's J (reset per call)
-    const int64_t *inc_ptr;   // [nodes + 1] node -> (cell N + i) incidence, ascending cells
-    const int32_t *inc;
-    int discard;              // discard consumed J tiles from L2 (no write-back of scratch)
 };
 
 constexpr int REM_MAX = 7;                 // remote copies of one node (<= 8 parts meet at a vertex)
@@ -364,14 +357,11 @@ __device__ __forceinline__ void scatter_node(const int32_t *rem, const int32_t *
 // M_DIAG: residual + the diagonal of the assembled Jacobian only (Jacobi
 // preconditioner of the Newton-Krylov driver): J[(i,a),(i,a)] of every cell
 // scatter-added into Y, no element matrices.
-// M_GLOBAL: residual + Jacobian assembled into the global CSR matrix with the
-// element matrices staged through L2 (eval_compact_kernel only; see
-// assemble_node_rows).
-enum { M_RESID = 0, M_JAC = 1, M_JVP = 2, M_CSR = 3, M_DIAG = 4, M_GLOBAL = 5 };
+enum { M_RESID = 0, M_JAC = 1, M_JVP = 2, M_CSR = 3, M_DIAG = 4 };
 // modes that form the tangent blocks (element matrices or CSR contributions)
 template <int MODE>
 __host__ __device__ constexpr bool forms_jac() {
-    return MODE == M_JAC || MODE == M_CSR || MODE == M_GLOBAL;
+    return MODE == M_JAC || MODE == M_CSR;
 }
 // per-(cell, qp) scalars: beta00 beta01 beta02 beta11 beta12, wmu2, gamma, wf0, wf1
 // (+ for M_JVP: dbeta00 dbeta01 dbeta02 dbeta11 dbeta12, gamma * tau)
@@ -1027,148 +1017,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
     if (JAC && l == 0) bulk_wait0();
 }
 
-// ---- NEXT-2 fused global matrix: assembly of one node's CSR rows from L2 ----
-// The warp pulls the two rows (i, 0), (i, 1) of every incident cell's element
-// Jacobian (node -> (cell, i) incidence, ascending cells) through the slot
-// table into a shared-memory row buffer and adds the buffer to the node's two
-// CSR rows with coalesced read-modify-writes: csr_gather_kernel's accumulation
-// for one node, in the same order (so the result is bitwise the two-kernel
-// path's).  The J rows are read with ld.global.cg: they were written by other
-// SMs' TMA stores in this launch.  Then every distinct incident tile's reader
-// count drops by one; the last reader discards the tile's J lines from L2
-// (`discard.global.L2`: J_cell is scratch, its write-back is skipped).
-template <int N, int TC>
-__device__ void assemble_node_rows(const EvalArgs &a, int64_t v, double *buf) {
-    constexpr int ND = 2 * N, LC = 2 * N, CPI = 32 / LC, BATCH = 8, NI = BATCH / CPI;
-    const int l = threadIdx.x & 31;
-    const int64_t r0 = __ldg(a.rowptr + 2 * v);
-    const int len = (int)(__ldg(a.rowptr + 2 * v + 2) - r0);  // both rows
-    const int64_t k0 = __ldg(a.inc_ptr + v);
-    const int cnt = (int)(__ldg(a.inc_ptr + v + 1) - k0);
-    const int32_t my = (l < cnt && l < BATCH) ? __ldg(a.inc + k0 + l) : 0;
-    for (int p = 2 * l; p < len; p += 64) *reinterpret_cast<double2 *>(&buf[p]) = make_double2(0.0, 0.0);
-    const int u = l / LC, ar = (l % LC) / N, j = l % N;
-    const bool lane_ok = l < CPI * LC;
-    const uint8_t *sb = reinterpret_cast<const uint8_t *>(a.slots);
-    double2 x[NI];
-    int sl[NI];
-#pragma unroll
-    for (int t = 0; t < NI; ++t) {
-        const int e = CPI * t + (u < CPI ? u : 0);
-        const int32_t ci = __shfl_sync(0xffffffffu, my, e);
-        const bool live = lane_ok && e < cnt;
-        const int64_t cell = ci / N;
-        const int i = ci - (int)(cell * N);
-        x[t] = live ? __ldcg(reinterpret_cast<const double2 *>(a.J_cell + (cell * ND + 2 * i + ar) * ND) + j)
-                    : make_double2(0.0, 0.0);
-        sl[t] = live ? (int)__ldg(sb + 8 * (int64_t)ci + j) : -1;
-    }
-    __syncwarp();
-    const int half = len >> 1;
-#pragma unroll
-    for (int t = 0; t < NI; ++t)
-#pragma unroll
-        for (int uu = 0; uu < CPI; ++uu) {
-            if (u == uu && sl[t] >= 0) {
-                double2 *p = reinterpret_cast<double2 *>(&buf[ar * half + 2 * sl[t]]);
-                double2 b = *p;
-                b.x += x[t].x;
-                b.y += x[t].y;
-                *p = b;
-            }
-            __syncwarp();
-        }
-    for (int64_t k = k0 + BATCH; k < k0 + cnt; ++k) {  // rare: more than BATCH incident cells
-        const int32_t ci = __ldg(a.inc + k);
-        const int64_t cell = ci / N;
-        const int i = ci - (int)(cell * N);
-        if (l < LC) {
-            const int s = (int)__ldg(sb + 8 * (int64_t)ci + j);
-            const double2 y = __ldcg(reinterpret_cast<const double2 *>(a.J_cell + (cell * ND + 2 * i + ar) * ND) + j);
-            buf[ar * half + 2 * s] += y.x;
-            buf[ar * half + 2 * s + 1] += y.y;
-        }
-        __syncwarp();
-    }
-    __syncwarp();
-    for (int p = 2 * l; p < len; p += 64) {
-        double2 *o = reinterpret_cast<double2 *>(a.csr_vals + r0 + p);
-        const double2 b = *reinterpret_cast<const double2 *>(&buf[p]);
-        double2 c = *o;
-        c.x += b.x;
-        c.y += b.y;
-        *o = c;
-    }
-    // this node no longer needs its incident tiles (its J loads have returned: their values are in
-    // the row buffer): drop their reader counts (distinct tiles: the incidence is in ascending cell
-    // order), discard a tile's J once nobody needs it
-    for (int base = 0; base < cnt; base += 32) {
-        const int k = base + l;
-        int32_t tile = -1, prev = -2;
-        if (k < cnt) tile = (int32_t)((__ldg(a.inc + k0 + k) / N) / TC);
-        if (k < cnt && k > 0) prev = (int32_t)((__ldg(a.inc + k0 + k - 1) / N) / TC);
-        bool last = false;
-        if (k < cnt && tile != prev) last = atomicSub(a.tile_cnt + tile, 1) == 1;
-        unsigned m = __ballot_sync(0xffffffffu, last && a.discard);
-        while (m) {
-            const int b = __ffs(m) - 1;
-            m &= m - 1;
-            const int32_t t = __shfl_sync(0xffffffffu, tile, b);
-            const int64_t c0 = (int64_t)t * TC;
-            const int64_t ncell = (a.ncells - c0 < TC) ? a.ncells - c0 : TC;
-            const int64_t lines = ncell * ND * ND * 8 / 128;
-            const char *jt = reinterpret_cast<const char *>(a.J_cell + c0 * ND * ND);
-            for (int64_t q = l; q < lines; q += 32)
-                asm volatile("discard.global.L2 [%0], 128;" ::"l"(jt + q * 128) : "memory");
-        }
-    }
-}
-
-// After tile `t`'s element Jacobians are complete in memory (the issuing lane waited for its bulk
-// store): each distinct node of the tile drops its count of incomplete incident tiles; the warp
-// assembles the nodes whose count reached zero, with `buf` (free shared memory) as row buffer.
-template <class E>
-__device__ __forceinline__ void signal_tile(const EvalArgs &a, int32_t g, bool valid, double *buf) {
-    const int l = threadIdx.x & 31;
-    const int key = valid ? g : -1 - l;
-    const unsigned peers = __match_any_sync(0xffffffffu, key);
-    bool done = false;
-    if (valid && (__ffs(peers) - 1) == l) done = atomicSub(a.node_cnt + g, 1) == 1;
-    unsigned m = __ballot_sync(0xffffffffu, done);
-    if (m) fence_acquire_gpu();  // every tile around these nodes is complete and visible
-    while (m) {
-        const int b = __ffs(m) - 1;
-        m &= m - 1;
-        const int32_t v = __shfl_sync(0xffffffffu, g, b);
-        assemble_node_rows<E::N, E::TC>(a, v, buf);
-        __syncwarp();
-    }
-}
-
-// Setup of the fused global-matrix counters (once per mesh): per tile the number
-// of distinct nodes of its cells (readers of its J tile), and per node the
-// number of distinct tiles around it (node_cnt0 zeroed by the caller).
-template <int N, int TC>
-__global__ void global_counts_kernel(int64_t ncells, int64_t ntiles, const int32_t *__restrict__ conn,
-                                     int32_t *__restrict__ node_cnt0, int32_t *__restrict__ tile_cnt0) {
-    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (t >= ntiles) return;
-    int32_t ids[TC * N];
-    int n = 0;
-    for (int c = 0; c < TC; ++c) {
-        const int64_t cell = t * TC + c;
-        if (cell >= ncells) break;
-        for (int k = 0; k < N; ++k) {
-            const int32_t g = conn[cell * N + k];
-            bool seen = false;
-            for (int m = 0; m < n; ++m) seen |= ids[m] == g;
-            if (!seen) ids[n++] = g;
-        }
-    }
-    tile_cnt0[t] = n;
-    for (int m = 0; m < n; ++m) atomicAdd(node_cnt0 + ids[m], 1);
-}
-
 // ---- G3/G4 with compact stored geometry (A_q = J_q^-T streamed per tile) ----
 // The stored kernel's TMA record ring and register gather, with the compact
 // record (RecC): the per-QP phase forms GradBF_n(q) = A_q grad_xi phi_n(xi_q)
@@ -1194,7 +1042,7 @@ struct CompactSmem {
     static constexpr int OFF_G = 2 * STAGE;
     static constexpr int OFF_QS = OFF_G + G_BYTES;                                 // double [NQS][TC][Q]
     static constexpr int QS_BYTES = PSUM ? 0 : nqs<MODE>() * TC * Q * 8;
-    static constexpr int J_BYTES = (MODE == M_JAC || MODE == M_GLOBAL) ? TC * E::JPITCH * 8 : 0;  // J staging over G + qs
+    static constexpr int J_BYTES = MODE == M_JAC ? TC * E::JPITCH * 8 : 0;         // J staging over G + qs
     static constexpr int TAIL = (G_BYTES + QS_BYTES > J_BYTES ? G_BYTES + QS_BYTES : J_BYTES);
     static constexpr int OFF_BAR = (int)round_up(OFF_G + TAIL, 8);
     static constexpr int BYTES = OFF_BAR + 2 * 8;
@@ -1237,8 +1085,7 @@ template <class E, int MODE>
 __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS : 16))
     eval_compact_kernel(EvalArgs a, const __grid_constant__ CUtensorMap jmap) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
-    constexpr bool GLOBAL = MODE == M_GLOBAL;
-    constexpr bool JAC = MODE == M_JAC || GLOBAL, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
+    constexpr bool JAC = MODE == M_JAC, JVP = MODE == M_JVP, CSR = MODE == M_CSR;
     static_assert(N == Q, "lane mappings assume N == Q");
     using R = RecC<E>;
     using S = CompactSmem<E, MODE>;
@@ -1252,10 +1099,9 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
     const int64_t vb = blockIdx.x, vg = gridDim.x;
 
-    uint64_t pol_stream = 0, pol_keep = 0;  // M_GLOBAL: J tiles are read back from L2 (evict_normal)
+    uint64_t pol_stream = 0;
     if (l == 0) {
         pol_stream = policy_evict_first();
-        if (GLOBAL) pol_keep = policy_evict_normal();
         for (int k = 0; k < 2; ++k) mbar_init(&bar[k], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         for (int k = 0; k < 2; ++k) {
@@ -1282,8 +1128,6 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS
         for (int n = 0; n < N; ++n) basis<E>(n, xq, yq, zq, bq[n], dx, dy, dz);
     }
 
-    int32_t gprev = 0;   // M_GLOBAL: this lane's node of the previous tile, signalled one tile late
-    bool vprev = false;
     int it = 0;
     for (int64_t tile = vb; tile < a.ntiles; tile += vg, ++it) {
         const int st = it & 1;
@@ -1432,22 +1276,8 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS
             fence_proxy_async_smem();
             __syncwarp();
             if (l == 0)
-                store_J<E>(a.J_cell, cell0, nvalid, reinterpret_cast<const char *>(rg),
-                           GLOBAL ? pol_keep : pol_stream, a.use_jmap ? &jmap : nullptr);
-        }
-        if (GLOBAL) {
-            // the previous tile's element Jacobians are complete (all but the newest bulk group); this
-            // tile's staging has been read, so its region is free as the assembly row buffer
-            if (l == 0) {
-                bulk_wait_read0();
-                bulk_wait1();
-                fence_proxy_async_global();
-                fence_release_gpu();
-            }
-            __syncwarp();
-            if (it > 0) signal_tile<E>(a, gprev, vprev, rg);
-            gprev = gnode;
-            vprev = act && c < nvalid;
+                store_J<E>(a.J_cell, cell0, nvalid, reinterpret_cast<const char *>(rg), pol_stream,
+                           a.use_jmap ? &jmap : nullptr);
         }
         if (act && c < nvalid) {
             if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, R0, R1);
@@ -1457,14 +1287,6 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS
         if (ntile < a.ntiles) gather_store_c<E, MODE>(smem + nst * S::STAGE, nxt);
     }
     if (JAC && l == 0) bulk_wait0();
-    if (GLOBAL && it > 0) {  // the last tile of this warp
-        if (l == 0) {
-            fence_proxy_async_global();
-            fence_release_gpu();
-        }
-        __syncwarp();
-        signal_tile<E>(a, gprev, vprev, rg);
-    }
 }
 
 // ---- G3/G4 with on-the-fly geometry ------------------------------------------

@@ -57,8 +57,7 @@ EXPORTS = [
     "stokesfo_set_remote", "stokesfo_set_remote_jvp", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
     "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
     "stokesfo_mesh_lateral_faces", "stokesfo_set_lateral", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
-    "stokesfo_jacobian_diag", "stokesfo_jacobian_global_work_size", "stokesfo_jacobian_global_setup",
-    "stokesfo_jacobian_global",
+    "stokesfo_jacobian_diag",
 ]
 
 
@@ -92,10 +91,6 @@ def _lib():
             L.stokesfo_jvp.argtypes = [P, P, P, P, P]
         if hasattr(L, "stokesfo_jacobian_diag"):
             L.stokesfo_jacobian_diag.argtypes = [P, P, P, P]
-        if hasattr(L, "stokesfo_jacobian_global"):
-            L.stokesfo_jacobian_global_work_size.argtypes = [P, ctypes.POINTER(ctypes.c_size_t)]
-            L.stokesfo_jacobian_global_setup.argtypes = [P, P]
-            L.stokesfo_jacobian_global.argtypes = [P, P, P, P, P, P]
         if hasattr(L, "stokesfo_basal_friction"):
             L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
         if hasattr(L, "stokesfo_lateral_pressure"):
@@ -359,26 +354,6 @@ class StokesFO:
         _dev(csr_vals, torch.float64, None, "csr_vals")
         _dev(R, torch.float64, (self.num_nodes, 2), "R")
         _check(_lib().stokesfo_jacobian_csr(self._h, _ptr(U), _ptr(csr_vals), _ptr(R)), "jacobian_csr")
-
-    def jacobian_global(self, U, csr_vals, R=None, J_scratch=None):
-        """csr_vals += assembled Jacobian (and R += residual) in one launch with the element matrices
-        staged through L2 (stokesfo_jacobian_global; compact geometry, after csr_slots).  J_scratch
-        ([C][2N][2N], content undefined afterwards) and the counter work buffer are allocated on first use."""
-        import torch
-        _dev(U, torch.float64, (self.num_nodes, 2), "U")
-        _dev(R, torch.float64, (self.num_nodes, 2), "R")
-        if getattr(self, "_global_work", None) is None:
-            n = ctypes.c_size_t(0)
-            _check(_lib().stokesfo_jacobian_global_work_size(self._h, ctypes.byref(n)), "jacobian_global_work_size")
-            self._global_work = torch.empty(int(n.value), dtype=torch.uint8, device=self.device)
-            _check(_lib().stokesfo_jacobian_global_setup(self._h, _ptr(self._global_work)), "jacobian_global_setup")
-        if J_scratch is None:
-            if getattr(self, "_global_J", None) is None:
-                N = self.N
-                self._global_J = torch.empty((self.num_cells, 2 * N, 2 * N), dtype=torch.float64, device=self.device)
-            J_scratch = self._global_J
-        _check(_lib().stokesfo_jacobian_global(self._h, _ptr(U), _ptr(J_scratch), _ptr(csr_vals), _ptr(R),
-                                               _ptr(self._global_work)), "jacobian_global")
 
     def scatter_assemble(self, R_cell=None, R=None, J_cell=None, csr_vals=None):
         _check(_lib().stokesfo_scatter_assemble(self._h, _ptr(R_cell), _ptr(R), _ptr(J_cell), _ptr(csr_vals)),

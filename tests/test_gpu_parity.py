@@ -485,43 +485,3 @@ def test_jacobian_diag_parity(torch, elem, drop, geometry):
     assert (np.abs(diag.cpu().numpy() - dref) <= TOL * dref).all()
     assert not diag.cpu().numpy()[~used].any()
     _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
-
-
-@pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 7)])
-def test_fused_global_matrix_through_l2(torch, elem, drop):
-    """NEXT-2 fused global matrix (stokesfo_jacobian_global, compact geometry): one
-    launch adds the assembled Jacobian to the CSR values with the element matrices
-    staged through L2 and pulled by the warp that completes each node's last tile.
-    It must equal the oracle's CSR scatter of its AD element Jacobians (element
-    tolerance), be bitwise the two-kernel path (jacobian + atomic-free pull
-    assembly: same rows, same ascending-cell summation order) and bitwise
-    reproducible, and give the oracle residual."""
-    ctx, orc = _setup(torch, elem, drop=drop, geometry="compact")
-    C, N = ctx.num_cells, ctx.N
-    rowptr, colidx = ctx.csr_pattern()
-    ctx.csr_slots()
-    rp2, ci2 = O.csr_pattern(orc["conn"], ctx.num_nodes)
-    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
-                     mode="jac")
-    v2, miss = O.scatter_csr(orc["e"], orc["conn"], ref["J_cell"], rp2, ci2)
-    cell_scale = np.abs(ref["J_cell"]).reshape(C, -1).max(1)[:, None, None] * np.ones_like(ref["J_cell"])
-    a2, _ = O.scatter_csr(orc["e"], orc["conn"], cell_scale, rp2, ci2)
-    assert miss == 0
-    U = _t(torch, orc["U"])
-    outs = []
-    for _ in range(2):
-        vals = torch.zeros(colidx.numel(), dtype=torch.float64, device="cuda")
-        R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
-        ctx.jacobian_global(U, vals, R=R)
-        ctx.sync()
-        outs.append((vals.clone(), R))
-    vals, R = outs[0]
-    assert torch.equal(outs[0][0], outs[1][0])
-    assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2).all()
-    _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
-    J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
-    ctx.jacobian(U, J)
-    vals_b = torch.zeros_like(vals)
-    ctx.scatter_assemble(J_cell=J, csr_vals=vals_b)
-    ctx.sync()
-    assert torch.equal(vals, vals_b)
