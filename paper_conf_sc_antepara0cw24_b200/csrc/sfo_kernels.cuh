@@ -185,7 +185,7 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
     if (!(det > 0.0)) atomicOr(err, ERR_DETJ);
     if (OUT == GEO_CHECK) return;
     const double idet = 1.0 / det;
-    if (OUT == GEO_COMPACT) {  // A = J^-T = cof / det
+    if constexpr (OUT == GEO_COMPACT) {  // A = J^-T = cof / det
 #pragma unroll
         for (int r = 0; r < 3; ++r)
 #pragma unroll
