@@ -1,6 +1,6 @@
 """Runs of every kernel variant for compute-sanitizer (memcheck / racecheck /
-synccheck / initcheck): hex8 + wedge6, stored + on-the-fly geometry, residual
-(partial-sum exchange), Jacobian, J.v, fused CSR, slot table + pull assembly,
+synccheck / initcheck): hex8 + wedge6, stored + on-the-fly + compact geometry, residual
+(partial-sum exchange), Jacobian, J.v, diagonal, fused CSR, slot table + pull assembly,
 ragged tiles, side sets, the NEXT-1 chain and a short Newton solve.  A second,
 larger mesh (more tiles than resident warps) exercises the persistent tile
 loop: record ring refills, next-tile gathers and the partial-sum overlay of a
@@ -19,7 +19,7 @@ def run(elem, n, L, drop, full):
     U, s, kc = M.fields(fp, L)
     kc = kc[:conn.shape[0]]
     C, N = conn.shape
-    for geo in ("stored", "on_the_fly"):
+    for geo in ("stored", "on_the_fly", "compact"):
         ctx = StokesFO(elem, torch.from_numpy(conn).cuda(), torch.from_numpy(coords).cuda(),
                        surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda(), geometry=geo)
         Ud = torch.from_numpy(U).cuda()
@@ -31,6 +31,7 @@ def run(elem, n, L, drop, full):
         ctx.jacobian(Ud, J, R_cell=Rc, R=R)
         ctx.viscosity_resid(Ud, mu_qp=mu, R_cell=Rc, R=R)
         ctx.jvp(Ud, Ud, Y, R=R)
+        ctx.jacobian_diag(Ud, Y, R=R)
         rp, ci = ctx.csr_pattern()
         ctx.csr_slots()
         vals = torch.zeros(ci.numel(), dtype=torch.float64, device="cuda")
@@ -50,7 +51,7 @@ def run(elem, n, L, drop, full):
         sd = torch.from_numpy(s).cuda()
         ctx.lateral_pressure(faces, sd, R)
         ctx.sync()
-        if geo == "stored":
+        if geo in ("stored", "compact"):
             ctx.set_lateral(faces, sd)
             Un = torch.ones_like(Ud)
             ctx.newton_solve(cells, beta, Un, max_newton=2, max_cg=20)
