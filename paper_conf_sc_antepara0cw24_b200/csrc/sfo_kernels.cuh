@@ -192,21 +192,22 @@ __global__ void geometry_kernel(int64_t ncells, int64_t nnodes, const int32_t *_
             for (int s2 = 0; s2 < 3; ++s2) ra[RC::a(3 * r + s2, q, c)] = cof[r][s2] * idet;
         rwm[RC::wm(q, c)] = wq * det;
         return;
-    }
+    } else {
 #pragma unroll
-    for (int n = 0; n < N; ++n)
+        for (int n = 0; n < N; ++n)
 #pragma unroll
-        for (int r = 0; r < 3; ++r) {
-            const double g = (cof[r][0] * dphi[n][0] + cof[r][1] * dphi[n][1] + cof[r][2] * dphi[n][2]) * idet;
-            if (OUT == GEO_RECORDS) {
-                rg[gidx<E>(n, q, r, c)] = g;
-            } else if (OUT == GEO_ALBANY) {
-                grad_bf[((int64_t)(n * Q + q) * 3 + r) * ncells + cell] = g;
-                grad_bf[((int64_t)(N * Q * 3) + (n * Q + q) * 3 + r) * ncells + cell] = g * (wq * det);
-            } else if (grad_bf) {
-                grad_bf[((cell * N + n) * Q + q) * 3 + r] = g;
+            for (int r = 0; r < 3; ++r) {
+                const double g = (cof[r][0] * dphi[n][0] + cof[r][1] * dphi[n][1] + cof[r][2] * dphi[n][2]) * idet;
+                if (OUT == GEO_RECORDS) {
+                    rg[gidx<E>(n, q, r, c)] = g;
+                } else if (OUT == GEO_ALBANY) {
+                    grad_bf[((int64_t)(n * Q + q) * 3 + r) * ncells + cell] = g;
+                    grad_bf[((int64_t)(N * Q * 3) + (n * Q + q) * 3 + r) * ncells + cell] = g * (wq * det);
+                } else if (grad_bf) {
+                    grad_bf[((cell * N + n) * Q + q) * 3 + r] = g;
+                }
             }
-        }
+    }
     if (OUT == GEO_ALBANY) {
 #pragma unroll
         for (int n = 0; n < N; ++n) {
