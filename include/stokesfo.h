@@ -281,13 +281,18 @@ int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid
  * (damped Newton, Jacobian at
  * every nonlinear step): per step, J dU = -F by Jacobi-preconditioned CG on the
  * matrix-free operator stokesfo_jvp + basal face term (J is SPD once basal
- * friction removes the rigid null space; Jacobi diagonal from stokesfo_jacobian
- * and the basal face matrices), then Armijo backtracking on ||F||.  Stops when
- * ||F|| <= max(atol, rtol ||F_0||) or after max_newton steps.  Single-GPU ctx
- * (a ctx with stokesfo_set_remote attached returns EINVAL).  U: dev [num_nodes][2], initial guess in, solution
- * out.  work: dev, stokesfo_newton_work_size bytes, 256-B aligned.  hist_F:
- * host [max_newton + 1] ||F|| per step; hist_cg: host [max_newton] CG
- * iterations (may be NULL); *iters = Newton steps taken. */
+ * friction removes the rigid null space; Jacobi diagonal from
+ * stokesfo_jacobian_diag and the basal face matrices), then Armijo backtracking
+ * on ||F||.  The CG scalars stay on the device and blocks of 8 CG iterations are
+ * replayed as one CUDA graph on a stream the solve creates (ordered after the
+ * ctx stream's prior work and before its later work); convergence is checked
+ * once per block.  Stops when ||F|| <= max(atol, rtol ||F_0||) or after
+ * max_newton steps.  Single-GPU ctx (a ctx with stokesfo_set_remote attached
+ * returns EINVAL).  Synchronous.  U: dev [num_nodes][2], initial guess in,
+ * solution out.  work: dev, stokesfo_newton_work_size bytes, 256-B aligned.
+ * hist_F: host [max_newton + 1] ||F|| per step; hist_cg: host [max_newton] CG
+ * iterations to reach rtol_cg per step (the block may run up to 7 more, which
+ * only refine the step; may be NULL); *iters = Newton steps taken. */
 typedef struct {
     int32_t max_newton;   /* e.g. 8 */
     int32_t max_cg;       /* CG iterations per Newton step */
