@@ -107,16 +107,22 @@ class P2PHalo:
         rem, remtab = part.remote_table()
         self.rem = torch.from_numpy(rem).to(device)
         self.remtab = torch.from_numpy(remtab).to(device)
-        handles = [S.ipc_get_handle(b) for b in self.buf]
+        # an allocation CUDA IPC cannot export (e.g. torch expandable segments) -> every rank falls back
+        try:
+            handles = [S.ipc_get_handle(b) for b in self.buf]
+        except Exception:
+            handles = None
         allh = [None] * self.world
         dist.all_gather_object(allh, handles)
         nns = [None] * self.world      # node counts: the field stride of each peer's buffer
         dist.all_gather_object(nns, int(nn))
         self.opened = []
-        ok = 1
+        ok = 1 if all(h is not None for h in allh) else 0
         ptrs = [[[0] * self.world for _ in range(fields)] for _ in range(2)]
         bases = {}   # one mapping per distinct peer allocation (handles may repeat)
         try:
+            if not ok:
+                raise RuntimeError("a rank could not export its buffers")
             for b in range(2):
                 for f in range(fields):
                     ptrs[b][f][self.rank] = self.buf[b].data_ptr() + f * nn * 16
