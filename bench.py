@@ -54,11 +54,12 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
         J = 8 * N
         xy = 16
     if op == "jac_global":
-        # jacobian (J_cell written) + pull assembly (DESIGN §6 NEXT-2): J_cell read again, per cell the
-        # slot row 8N and incidence 4N, per node rowptr pair 16 + incidence pointer 8, CSR values read + written
+        # jacobian (J_cell written) + pull assembly overwriting the CSR values (DESIGN §6 NEXT-2): J_cell read
+        # again, per cell the slot row 8N and incidence 4N, per node rowptr pair 16 + incidence pointer 8,
+        # every CSR value written once (8 nnz)
         J = 2 * 8 * (2 * N) ** 2 + 8 * N + 4 * N
         xy = 24
-    vals = 16 * nnz if op in ("jac_csr", "jac_global") else 0
+    vals = {"jac_csr": 16 * nnz, "jac_global": 8 * nnz}.get(op, 0)
     if geometry == "on_the_fly":
         return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32 + xy) + vals
     if geometry == "compact":   # A_q = J_q^-T (9 doubles) + wM per QP instead of GradBF
@@ -417,9 +418,9 @@ def main():
             ctx.jacobian(Uc, J, R=Rc)
         elif args.op == "jac_csr":
             ctx.jacobian_csr(Uc, vals, R=Rc)
-        elif args.op == "jac_global":   # element matrices, then the atomic-free pull assembly into CSR
+        elif args.op == "jac_global":   # element matrices, then the atomic-free pull assembly overwriting CSR
             ctx.jacobian(Uc, J, R=Rc)
-            ctx.scatter_assemble(J_cell=J, csr_vals=vals)
+            ctx.assemble_csr(J, vals, accumulate=False)
         elif args.op == "jvp":
             ctx.jvp(Uc, Xd, Yc, R=Rc)
         else:
@@ -427,7 +428,7 @@ def main():
 
     def step(i=None):
         Rc, Yc = begin()
-        if vals is not None:
+        if vals is not None and args.op == "jac_csr":   # jac_global overwrites every CSR value
             vals.zero_()
         if i is not None:
             k0[i].record(stream)
@@ -505,7 +506,7 @@ def main():
         s0.record(stream)
         for i in range(n_sus):
             Rc, Yc = begin()
-            if vals is not None:
+            if vals is not None and args.op == "jac_csr":
                 vals.zero_()
             ks0[i].record(stream)
             evaluate(U, Rc, Yc)
@@ -559,7 +560,7 @@ def main():
                 Rc.zero_()
                 if Yc is not None:
                     Yc.zero_()
-            if vals is not None:
+            if vals is not None and args.op == "jac_csr":
                 vals.zero_()
             evaluate(Ub[b], Rc, Yc)
             finish(Rc, Yc)
@@ -669,7 +670,7 @@ def main():
                             "jac_global": "M_JAC> + csr_gather_kernel"}[args.op]
                          + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
                             "jvp": " (stokesfo_jvp)", "jac_csr": " (stokesfo_jacobian_csr)",
-                            "jac_global": " (stokesfo_jacobian + stokesfo_scatter_assemble, both timed)"}[args.op],
+                            "jac_global": " (stokesfo_jacobian + stokesfo_assemble_csr overwriting, both timed)"}[args.op],
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src,
                          "live_copy_gbs": live_copy,
                          "note": "live_copy_gbs: torch device-to-device copy of 2 GiB on this box before the timed "

@@ -196,6 +196,17 @@ int stokesfo_set_lateral(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, 
 int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R,
                               const double *J_cell, double *csr_vals);
 
+/* NEXT-2 global matrix from element matrices with the atomic-free pull
+ * assembly (requires stokesfo_csr_slots; nodes with at most 64 neighbour nodes,
+ * else EUNSUPPORTED): a warp owns a node's two CSR rows and sums the rows of
+ * every incident cell's J_cell in ascending cell order (bitwise reproducible).
+ * accumulate != 0: csr_vals += assembled J (as stokesfo_scatter_assemble);
+ * accumulate == 0: csr_vals = assembled J -- every entry of the pattern is
+ * written, so the caller needs no zeroing pass and the kernel never reads
+ * csr_vals (15 GB less traffic per C4 fill).  J_cell: dev [C][2N][2N];
+ * csr_vals: dev [nnz]. */
+int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_vals, int accumulate);
+
 /* CSR pattern over dofs (rows = 2*num_nodes; columns of a row = sorted dofs of
  * every node sharing a cell with the row's node).  Size query: pass rowptr =
  * colidx = NULL to get *nnz.  Fill: rowptr dev [2*num_nodes+1] int64, colidx

@@ -629,6 +629,26 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
     return cuda_status();
 }
 
+int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_vals, int accumulate) {
+    SFO_RANGE("stokesfo_assemble_csr");
+    if (!c || !J_cell || !csr_vals || !aligned(J_cell, 16) || !aligned(csr_vals, 16)) return STOKESFO_EINVAL;
+    if (!c->slots || !c->inc || !c->rowptr) return STOKESFO_EINVAL;  // needs stokesfo_csr_slots
+    if (c->csr_maxdeg > CSR_GATHER_MAXDEG) return STOKESFO_EUNSUPPORTED;
+    const int64_t NN = c->d.num_nodes;
+    if (NN == 0) return STOKESFO_OK;
+    const int64_t per_block = (int64_t)CSR_GATHER_WARPS * CSR_GATHER_NPW;
+    const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
+    const int bt = 32 * CSR_GATHER_WARPS;
+    if (c->N == 8) {
+        if (accumulate) csr_gather_kernel<8, true><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+        else csr_gather_kernel<8, false><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+    } else {
+        if (accumulate) csr_gather_kernel<6, true><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+        else csr_gather_kernel<6, false><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+    }
+    return cuda_status();
+}
+
 int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure) {
     SFO_RANGE("stokesfo_geometry");
     if (!c) return STOKESFO_EINVAL;

@@ -1829,7 +1829,8 @@ __global__ void scatter_csr_slots_kernel(int64_t ncells, const int32_t *__restri
 constexpr int CSR_GATHER_MAXDEG = 64;   // neighbour nodes per node (else the atomic kernel)
 constexpr int CSR_GATHER_WARPS = 8;
 constexpr int CSR_GATHER_NPW = 2;       // nodes per warp
-template <int N>
+// ACC = false: the rows are overwritten (vals = assembled J; no prior zeroing, no read of vals).
+template <int N, bool ACC = true>
 __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
     csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
                       const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
@@ -1854,10 +1855,12 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
         cnt[n] = ok ? (int)(__ldg(inc_ptr + v + 1) - k0[n]) : 0;
     }
     // pull the rows' vals lines into L2 now: the final read-modify-write then hits L2
+    if (ACC) {
 #pragma unroll
-    for (int n = 0; n < NPW; ++n)
-        for (int p = 16 * l; p < len[n]; p += 16 * 32)
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(vals + r0[n] + p));
+        for (int n = 0; n < NPW; ++n)
+            for (int p = 16 * l; p < len[n]; p += 16 * 32)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(vals + r0[n] + p));
+    }
     // incidence: lane n LPN + t holds entry t (< BATCH) of node n
     const int ln = l / LPN, lt = l % LPN;
     int32_t my = 0;
@@ -1924,10 +1927,14 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
         for (int p = 2 * l; p < len[n]; p += 64) {
             double2 *o = reinterpret_cast<double2 *>(vals + r0[n] + p);
             const double2 b = *reinterpret_cast<const double2 *>(&buf[w][n][p]);
-            double2 c = *o;
-            c.x += b.x;
-            c.y += b.y;
-            *o = c;
+            if (ACC) {
+                double2 c = *o;
+                c.x += b.x;
+                c.y += b.y;
+                *o = c;
+            } else {
+                __stcs(o, b);  // streamed: the assembled matrix is not re-read by this kernel
+            }
         }
 }
 

@@ -57,7 +57,7 @@ EXPORTS = [
     "stokesfo_set_remote", "stokesfo_set_remote_jvp", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
     "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
     "stokesfo_mesh_lateral_faces", "stokesfo_set_lateral", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
-    "stokesfo_jacobian_diag",
+    "stokesfo_jacobian_diag", "stokesfo_assemble_csr",
 ]
 
 
@@ -91,6 +91,8 @@ def _lib():
             L.stokesfo_jvp.argtypes = [P, P, P, P, P]
         if hasattr(L, "stokesfo_jacobian_diag"):
             L.stokesfo_jacobian_diag.argtypes = [P, P, P, P]
+        if hasattr(L, "stokesfo_assemble_csr"):
+            L.stokesfo_assemble_csr.argtypes = [P, P, P, ctypes.c_int]
         if hasattr(L, "stokesfo_basal_friction"):
             L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
         if hasattr(L, "stokesfo_lateral_pressure"):
@@ -354,6 +356,12 @@ class StokesFO:
         _dev(csr_vals, torch.float64, None, "csr_vals")
         _dev(R, torch.float64, (self.num_nodes, 2), "R")
         _check(_lib().stokesfo_jacobian_csr(self._h, _ptr(U), _ptr(csr_vals), _ptr(R)), "jacobian_csr")
+
+    def assemble_csr(self, J_cell, csr_vals, accumulate=False):
+        """csr_vals (+)= the global matrix assembled from element matrices (stokesfo_assemble_csr;
+        pull assembly, after csr_slots); accumulate=False overwrites every entry."""
+        _check(_lib().stokesfo_assemble_csr(self._h, _ptr(J_cell), _ptr(csr_vals), 1 if accumulate else 0),
+               "assemble_csr")
 
     def scatter_assemble(self, R_cell=None, R=None, J_cell=None, csr_vals=None):
         _check(_lib().stokesfo_scatter_assemble(self._h, _ptr(R_cell), _ptr(R), _ptr(J_cell), _ptr(csr_vals)),

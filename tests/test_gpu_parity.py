@@ -427,6 +427,15 @@ def test_csr_slots_and_fused_assembly(torch, elem, geometry):
     ctx.scatter_assemble(J_cell=J, csr_vals=vals2)
     ctx.sync()
     assert torch.equal(vals, vals2)
+    # overwrite mode (stokesfo_assemble_csr, accumulate = 0): every entry of the pattern is written
+    # (a NaN prefill must disappear) and equals the accumulated assembly bitwise; accumulate = 1 adds
+    vals3 = torch.full_like(vals, float("nan"))
+    ctx.assemble_csr(J, vals3, accumulate=False)
+    ctx.sync()
+    assert torch.equal(vals3, vals)
+    ctx.assemble_csr(J, vals3, accumulate=True)
+    ctx.sync()
+    assert torch.equal(vals3, 2 * vals)
     # fused: residual + Jacobian straight into CSR
     vals.zero_()
     R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
