@@ -47,7 +47,8 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
     N = 8 if elem == "hex8" else 6
     Q = N
     J = 8 * (2 * N) ** 2 if op == "jacobian" else 0
-    xy = (16 + 32) if op == "jvp" else 0  # X gather, Y read+write
+    xy = (16 + 32) if op in ("jvp", "jvp_y") else 0  # X gather, Y read+write
+    rb = 0 if op == "jvp_y" else 32                   # R read + write (jvp_y: the Krylov apply, no residual)
     if op == "jac_csr":
         # NEXT-2 fused CSR: no J_cell; per cell the slot row 8N, per node the
         # rowptr pair 16, and every CSR value read + written once (16 nnz)
@@ -61,11 +62,11 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
         xy = 24
     vals = {"jac_csr": 16 * nnz, "jac_global": 8 * nnz}.get(op, 0)
     if geometry == "on_the_fly":
-        return cells * (4 * N + 8 + J) + nodes * (16 + 8 + 32 + 32 + xy) + vals
+        return cells * (4 * N + 8 + J) + nodes * (16 + 8 + rb + 32 + xy) + vals
     if geometry == "compact":   # A_q = J_q^-T (9 doubles) + wM per QP instead of GradBF
-        return cells * (4 * N + 72 * Q + 8 * Q + 8 + J) + nodes * (16 + 8 + 32 + xy) + vals
+        return cells * (4 * N + 72 * Q + 8 * Q + 8 + J) + nodes * (16 + 8 + rb + xy) + vals
     per_cell = 4 * N + 24 * N * Q + 8 * Q + 8 + J
-    return cells * per_cell + nodes * (16 + 8 + 32 + xy) + vals
+    return cells * per_cell + nodes * (16 + 8 + rb + xy) + vals
 
 
 MESH_SIZES = {"C4": (8431650, 9313304), "C5": (16863300, 9313304), "C3": (2033100, 2274459),
@@ -301,7 +302,7 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly", "compact"])
-    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jac_csr", "jac_global"],
+    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jvp_y", "jac_csr", "jac_global"],
                     help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
                          "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
     ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
@@ -356,15 +357,16 @@ def main():
     N = conn.shape[1]
     stream = torch.cuda.current_stream(dev)
     ctx = StokesFO(elem, conn, coords, surface=surface, flow_factor=kc, stream=stream, geometry=args.geometry)
-    if world > 1 and args.op in ("jac_csr", "jac_global"):
-        sys.stderr.write("bench.py: the global-matrix ops are single-GPU (no CSR row exchange)\n")
+    if world > 1 and args.op in ("jac_csr", "jac_global", "jvp_y"):
+        sys.stderr.write("bench.py: --op jac_csr / jac_global / jvp_y are single-GPU lines\n")
         return 2
     J = torch.empty((C, 2 * N, 2 * N) if args.op in ("jacobian", "jac_global") else (0,), dtype=torch.float64,
                     device=dev)
     # J.v direction: one global seeded field, restricted to this rank's nodes (consistent across ranks)
-    x_global = np.random.default_rng(5).normal(0, 10.0, (coords_g.shape[0], 2)) if args.op == "jvp" else None
-    Xd = torch.from_numpy(np.ascontiguousarray(x_global[gids])).to(dev) if args.op == "jvp" else None
-    Yd = torch.zeros((NN, 2), dtype=torch.float64, device=dev) if args.op == "jvp" else None
+    JV = args.op in ("jvp", "jvp_y")
+    x_global = np.random.default_rng(5).normal(0, 10.0, (coords_g.shape[0], 2)) if JV else None
+    Xd = torch.from_numpy(np.ascontiguousarray(x_global[gids])).to(dev) if JV else None
+    Yd = torch.zeros((NN, 2), dtype=torch.float64, device=dev) if JV else None
     R = torch.zeros((NN, 2), dtype=torch.float64, device=dev)
     nnz, vals = 0, None
     if args.op in ("jac_csr", "jac_global"):   # NEXT-2: pattern + slot table once per mesh (untimed)
@@ -423,6 +425,8 @@ def main():
             ctx.assemble_csr(J, vals, accumulate=False)
         elif args.op == "jvp":
             ctx.jvp(Uc, Xd, Yc, R=Rc)
+        elif args.op == "jvp_y":   # the Krylov operator apply: Y += J(U) X only
+            ctx.jvp(Uc, Xd, Yc)
         else:
             ctx.viscosity_resid(Uc, R=Rc)
 
@@ -640,6 +644,8 @@ def main():
             "metric": {"jacobian": METRIC,
                        "resid": "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s",
                        "jvp": "Stokes-FO matrix-free J(U)X + residual (stokesfo_jvp) cells/s and achieved HBM GB/s",
+                       "jvp_y": "Stokes-FO matrix-free J(U)X only (stokesfo_jvp, the Krylov operator apply) cells/s "
+                                "and achieved HBM GB/s",
                        "jac_csr": "Stokes-FO residual + Jacobian assembled into global CSR (stokesfo_jacobian_csr) "
                                   "cells/s and achieved HBM GB/s",
                        "jac_global": "Stokes-FO residual + Jacobian assembled into global CSR (stokesfo_jacobian + "
@@ -666,10 +672,12 @@ def main():
                          "kernel": {"on_the_fly": "eval_otf_kernel", "compact": "eval_compact_kernel",
                                     "stored": "eval_kernel"}[args.geometry]
                          + ("<Hex8," if elem == "hex8" else "<Wedge6,")
-                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jac_csr": "M_CSR>",
+                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jvp_y": "M_JVP>",
+                            "jac_csr": "M_CSR>",
                             "jac_global": "M_JAC> + csr_gather_kernel"}[args.op]
                          + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
-                            "jvp": " (stokesfo_jvp)", "jac_csr": " (stokesfo_jacobian_csr)",
+                            "jvp": " (stokesfo_jvp)", "jvp_y": " (stokesfo_jvp, R = NULL)",
+                            "jac_csr": " (stokesfo_jacobian_csr)",
                             "jac_global": " (stokesfo_jacobian + stokesfo_assemble_csr overwriting, both timed)"}[args.op],
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src,
                          "live_copy_gbs": live_copy,

@@ -958,25 +958,32 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
         if constexpr (S::PSUM) {
             // partial sums over the GradBF region of this stage (its reads are done: __syncwarp above)
             double2 *P = reinterpret_cast<double2 *>(stage + R::G_OFF);
-            if (act) {
-                const double w = qv[5];
-                const double s00 = w * qv[0], s01 = w * qv[1], s02 = w * qv[2], s11 = w * qv[3], s12 = w * qv[4];
+            // J.v without a residual output (the Newton-Krylov operator apply): skip the residual's exchange
+            const bool resid_out = !JVP || a.R != nullptr || a.R_cell != nullptr;
+            if (resid_out) {
+                if (act) {
+                    const double w = qv[5];
+                    const double s00 = w * qv[0], s01 = w * qv[1], s02 = w * qv[2], s11 = w * qv[3], s12 = w * qv[4];
 #pragma unroll
-                for (int n = 0; n < N; ++n) {
-                    const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
-                    P[psum_idx<E>(c, n, s)] = make_double2(fma(qv[7], bq[n], fma(g2, s02, fma(g1, s01, g0 * s00))),
-                                                           fma(qv[8], bq[n], fma(g2, s12, fma(g1, s11, g0 * s01))));
+                    for (int n = 0; n < N; ++n) {
+                        const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
+                        P[psum_idx<E>(c, n, s)] =
+                            make_double2(fma(qv[7], bq[n], fma(g2, s02, fma(g1, s01, g0 * s00))),
+                                         fma(qv[8], bq[n], fma(g2, s12, fma(g1, s11, g0 * s01))));
+                    }
                 }
-            }
-            __syncwarp();
-            prefetch();
-            if (act) {
+                __syncwarp();
+                prefetch();
+                if (act) {
 #pragma unroll
-                for (int k = 0; k < Q; ++k) {
-                    const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
-                    R0 += v.x;
-                    R1 += v.y;
+                    for (int k = 0; k < Q; ++k) {
+                        const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
+                        R0 += v.x;
+                        R1 += v.y;
+                    }
                 }
+            } else {
+                prefetch();
             }
             if (JVP) {
                 __syncwarp();
@@ -1240,25 +1247,32 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS
         if constexpr (S::PSUM) {
             // partial sums over the (unused) GradBF region
             double2 *P = reinterpret_cast<double2 *>(rg);
-            if (act) {
-                const double w = qv[5];
-                const double s00 = w * qv[0], s01 = w * qv[1], s02 = w * qv[2], s11 = w * qv[3], s12 = w * qv[4];
+            // J.v without a residual output (the Newton-Krylov operator apply): skip the residual's exchange
+            const bool resid_out = !JVP || a.R != nullptr || a.R_cell != nullptr;
+            if (resid_out) {
+                if (act) {
+                    const double w = qv[5];
+                    const double s00 = w * qv[0], s01 = w * qv[1], s02 = w * qv[2], s11 = w * qv[3], s12 = w * qv[4];
 #pragma unroll
-                for (int n = 0; n < N; ++n) {
-                    const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
-                    P[psum_idx<E>(c, n, s)] = make_double2(fma(qv[7], bq[n], fma(g2, s02, fma(g1, s01, g0 * s00))),
-                                                           fma(qv[8], bq[n], fma(g2, s12, fma(g1, s11, g0 * s01))));
+                    for (int n = 0; n < N; ++n) {
+                        const double g0 = gq[n][0], g1 = gq[n][1], g2 = gq[n][2];
+                        P[psum_idx<E>(c, n, s)] =
+                            make_double2(fma(qv[7], bq[n], fma(g2, s02, fma(g1, s01, g0 * s00))),
+                                         fma(qv[8], bq[n], fma(g2, s12, fma(g1, s11, g0 * s01))));
+                    }
                 }
-            }
-            __syncwarp();
-            prefetch();
-            if (act) {
+                __syncwarp();
+                prefetch();
+                if (act) {
 #pragma unroll
-                for (int k = 0; k < Q; ++k) {
-                    const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
-                    R0 += v.x;
-                    R1 += v.y;
+                    for (int k = 0; k < Q; ++k) {
+                        const double2 v = P[psum_idx<E>(c, s, (k + s) % Q)];
+                        R0 += v.x;
+                        R1 += v.y;
+                    }
                 }
+            } else {
+                prefetch();
             }
             if (JVP) {
                 __syncwarp();
