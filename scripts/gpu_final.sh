@@ -14,7 +14,7 @@ timeout 900 python bench.py --impl reference --steps 5 --warmup 3 > $OUT/bench_r
 for A in "--config C3" "--config C5" "--config C4p" "--config C4 --op resid" "--config C5 --op resid" \
          "--config C4 --op jvp" "--config C4 --geometry compact" "--config C4 --op jvp --geometry compact" \
          "--config C5 --geometry compact" "--config C4 --geometry on_the_fly" "--config C4 --op jac_global" \
-         "--config C4 --op jac_csr" "--config C1"; do
+         "--config C4 --op jac_csr" "--config C4 --op jvp_y" "--config C4 --op jvp_y --geometry compact" "--config C1"; do
   timeout 900 python bench.py $A --no-cpu-baseline >> $OUT/bench_lines.jsonl 2>> $OUT/bench_lines.err
 done
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
@@ -23,7 +23,8 @@ bash scripts/gpu_prof.sh $TAG "c4jac|C4:hex8:jacobian:stored|--config C4" "c5jac
    "c4jvp|C4:hex8:jvp:stored|--config C4 --op jvp" "c4res|C4:hex8:resid:stored|--config C4 --op resid" \
    "c5res|C5:wedge6:resid:stored|--config C5 --op resid" "c4cmp|C4:hex8:jacobian:compact|--config C4 --geometry compact" \
    "c4otf|C4:hex8:jacobian:on_the_fly|--config C4 --geometry on_the_fly" "c3jac|C3:hex8:jacobian:stored|--config C3" \
-   "c4pjac|C4p:hex8:jacobian:stored|--config C4p" > $OUT/prof.log 2>&1
+   "c4pjac|C4p:hex8:jacobian:stored|--config C4p" "c4jvpy|C4:hex8:jvp_y:stored|--config C4 --op jvp_y" \
+   "c5cmp|C5:wedge6:jacobian:compact|--config C5 --geometry compact" > $OUT/prof.log 2>&1
 python - <<PY > $OUT/summary.txt
 import json
 for f in ["$OUT/bench_C4.json", "$OUT/bench_reference.json", "$OUT/bench_lines.jsonl"]:

@@ -84,7 +84,7 @@ def test_traffic_entries_are_keyed_to_this_build_and_plausible():
     for key, e in tr.items():
         assert "rev" in e and "tag" in e, key
         cfg, elem, op, geo = key.split(":")
-        if e["rev"] != rev or op not in ("jacobian", "resid", "jvp") or cfg not in sizes:
+        if e["rev"] != rev or op not in ("jacobian", "resid", "jvp", "jvp_y") or cfg not in sizes:
             continue
         cells, nodes = sizes[cfg]
         algo = bench.bytes_per_launch(elem, cells, nodes, geo, op)
