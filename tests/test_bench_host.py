@@ -93,3 +93,21 @@ def test_traffic_entries_are_keyed_to_this_build_and_plausible():
         assert got == e["dram_bytes_per_launch"] and e["tag"] in src
     # a stale or foreign entry is never reported
     assert bench.lookup_traffic("C4", "hex8", "jacobian", "stored", 2)[0] is None
+
+
+def test_gpus_n_relaunch_refuses_without_enough_gpus(monkeypatch, capsys):
+    """`python bench.py --gpus N` without a torchrun environment re-launches itself with N
+    ranks, one per GPU (r1 verdict: it timed one GPU and reported n_gpus = 1); with fewer
+    visible GPUs than N (and the NCCL backend) it refuses instead of oversubscribing."""
+    import torch
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    monkeypatch.setenv("STOKESFO_BENCH_BACKEND", "nccl")
+    monkeypatch.setattr(torch.cuda, "device_count", lambda: 1)
+    assert bench.relaunch(2) == 2
+    assert "needs 2 visible GPUs" in capsys.readouterr().err
+    # under torchrun, --gpus must equal WORLD_SIZE
+    monkeypatch.setenv("WORLD_SIZE", "3")
+    monkeypatch.setenv("RANK", "0")
+    monkeypatch.setattr("sys.argv", ["bench.py", "--gpus", "2", "--no-cpu-baseline"])
+    assert bench.main() == 2
+    assert "WORLD_SIZE = 3" in capsys.readouterr().err
