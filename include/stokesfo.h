@@ -84,7 +84,8 @@ typedef enum {
     STOKESFO_EMESH = 2,        /* det J <= 0, conn out of range, CSR entry missing */
     STOKESFO_ECUDA = 3,        /* a CUDA runtime error */
     STOKESFO_ENOMEM = 4,       /* workspace too small */
-    STOKESFO_EUNSUPPORTED = 5  /* e.g. glen_n != 3 */
+    STOKESFO_EUNSUPPORTED = 5, /* e.g. glen_n != 3 */
+    STOKESFO_ENONFINITE = 6    /* NaN / Inf in an output (only with STOKESFO_CHECK_FINITE=1) */
 } stokesfo_status_t;
 
 typedef struct {
@@ -272,8 +273,14 @@ int stokesfo_ipc_get_handle(const void *dev_ptr, void *handle, int64_t *offset);
 int stokesfo_ipc_open_handle(const void *handle, void **dev_ptr);
 int stokesfo_ipc_close(void *dev_ptr);
 
+/* Failure detection: with the environment variable STOKESFO_CHECK_FINITE=1 set
+ * when the ctx is created, viscosity_resid / jacobian / jvp / jacobian_diag scan
+ * the outputs they wrote for NaN / Inf (one extra read of each output) and raise
+ * a sticky flag that stokesfo_sync reports as STOKESFO_ENONFINITE. */
+
 /* Synchronise the ctx stream; returns ECUDA on a CUDA error, else EMESH if a
- * device-side error flag was raised since create, else OK. */
+ * mesh error flag (det J <= 0, conn out of range, CSR entry missing) was raised
+ * since create, else ENONFINITE if the finite check flagged an output, else OK. */
 int stokesfo_sync(stokesfo_ctx *c);
 
 /* Static string for a status code. */

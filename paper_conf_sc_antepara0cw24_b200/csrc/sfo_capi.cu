@@ -52,6 +52,7 @@ struct stokesfo_ctx {
     CUtensorMap jmap;
     const double *jmap_ptr = nullptr;
     bool jmap_ok = false;
+    bool check_finite = false;  // STOKESFO_CHECK_FINITE=1 at create: scan outputs for NaN / Inf
 };
 
 namespace {
@@ -77,6 +78,14 @@ struct NvtxRange {
 #define SFO_RANGE(name) NvtxRange sfo_nvtx_range_(name)
 
 bool aligned(const void *p, size_t a) { return (reinterpret_cast<uintptr_t>(p) % a) == 0; }
+
+// STOKESFO_CHECK_FINITE=1: scan an output (n doubles) for NaN / Inf after the call that wrote it
+void check_finite(const stokesfo_ctx *c, const double *p, int64_t n) {
+    if (!c->check_finite || !p || n <= 0) return;
+    const int bs = 256;
+    const unsigned g = (unsigned)std::min<int64_t>((n + bs - 1) / bs, 148 * 16);
+    finite_check_kernel<<<g, bs, 0, c->stream>>>(n, p, c->err);
+}
 
 int cuda_status() {
     cudaError_t e = cudaGetLastError();
@@ -341,6 +350,7 @@ const char *stokesfo_strerror(int s) {
         case STOKESFO_ECUDA: return "CUDA runtime error";
         case STOKESFO_ENOMEM: return "workspace too small";
         case STOKESFO_EUNSUPPORTED: return "unsupported configuration (glen_n must be 3)";
+        case STOKESFO_ENONFINITE: return "non-finite value in an output (STOKESFO_CHECK_FINITE=1)";
         default: return "unknown status";
     }
 }
@@ -378,6 +388,7 @@ int stokesfo_create(const stokesfo_desc_t *d, stokesfo_ctx **out) {
     if (!c) return STOKESFO_ENOMEM;
     c->d = *d;
     c->stream = reinterpret_cast<cudaStream_t>(d->stream);
+    if (const char *e = getenv("STOKESFO_CHECK_FINITE")) c->check_finite = atoi(e) == 1;
     c->err = reinterpret_cast<int *>(d->workspace);
     c->mode = d->geometry_mode;
     char *ws = reinterpret_cast<char *>(d->workspace);
@@ -435,8 +446,14 @@ int stokesfo_viscosity_resid(stokesfo_ctx *c, const double *U, double *mu_qp, do
     for (const void *p : ps)
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
 #define CALL(E) eval_impl<E, M_RESID>(c, U, mu_qp, R_cell, R, nullptr)
-    return DISPATCH(c, CALL);
+    const int st = DISPATCH(c, CALL);
 #undef CALL
+    if (st == STOKESFO_OK) {
+        check_finite(c, mu_qp, c->d.num_cells * c->Q);
+        check_finite(c, R_cell, c->d.num_cells * c->N * 2);
+        check_finite(c, R, c->d.num_nodes * 2);
+    }
+    return st == STOKESFO_OK ? cuda_status() : st;
 }
 
 int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *R_cell, double *R) {
@@ -448,8 +465,14 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
     for (const void *p : ps)
         if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
 #define CALL(E) eval_impl<E, M_JAC>(c, U, nullptr, R_cell, R, J_cell)
-    return DISPATCH(c, CALL);
+    const int st = DISPATCH(c, CALL);
 #undef CALL
+    if (st == STOKESFO_OK) {
+        check_finite(c, J_cell, c->d.num_cells * 4 * c->N * c->N);
+        check_finite(c, R_cell, c->d.num_cells * c->N * 2);
+        check_finite(c, R, c->d.num_nodes * 2);
+    }
+    return st == STOKESFO_OK ? cuda_status() : st;
 }
 
 int stokesfo_jacobian_csr(stokesfo_ctx *c, const double *U, double *csr_vals, double *R) {
@@ -519,8 +542,13 @@ int stokesfo_jvp(stokesfo_ctx *c, const double *U, const double *X, double *Y, d
         return STOKESFO_EINVAL;
     if (c->rem && !c->peers_y) return STOKESFO_EINVAL;  // Y would miss the peers' boundary contributions
 #define CALL(E) eval_impl<E, M_JVP>(c, U, nullptr, nullptr, R, nullptr, X, Y)
-    return DISPATCH(c, CALL);
+    const int st = DISPATCH(c, CALL);
 #undef CALL
+    if (st == STOKESFO_OK) {
+        check_finite(c, Y, c->d.num_nodes * 2);
+        check_finite(c, R, c->d.num_nodes * 2);
+    }
+    return st == STOKESFO_OK ? cuda_status() : st;
 }
 
 int stokesfo_jacobian_diag(stokesfo_ctx *c, const double *U, double *diag, double *R) {
@@ -530,8 +558,13 @@ int stokesfo_jacobian_diag(stokesfo_ctx *c, const double *U, double *diag, doubl
     if (!U || !diag || !aligned(U, 16) || !aligned(diag, 16) || (R && !aligned(R, 16))) return STOKESFO_EINVAL;
     if (c->rem && !c->peers_y) return STOKESFO_EINVAL;  // diag would miss the peers' boundary contributions
 #define CALL(E) eval_impl<E, M_DIAG>(c, U, nullptr, nullptr, R, nullptr, nullptr, diag)
-    return DISPATCH(c, CALL);
+    const int st = DISPATCH(c, CALL);
 #undef CALL
+    if (st == STOKESFO_OK) {
+        check_finite(c, diag, c->d.num_nodes * 2);
+        check_finite(c, R, c->d.num_nodes * 2);
+    }
+    return st == STOKESFO_OK ? cuda_status() : st;
 }
 
 int stokesfo_basal_friction(stokesfo_ctx *c, const int32_t *basal_cells, int64_t nfaces, const double *beta,
@@ -770,7 +803,8 @@ int stokesfo_sync(stokesfo_ctx *c) {
     if (cudaStreamSynchronize(c->stream) != cudaSuccess) return cuda_status();
     int h = 0;
     if (cudaMemcpy(&h, c->err, sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess) return cuda_status();
-    return h ? STOKESFO_EMESH : STOKESFO_OK;
+    if (h & (ERR_DETJ | ERR_CONN | ERR_CSR)) return STOKESFO_EMESH;
+    return h ? STOKESFO_ENONFINITE : STOKESFO_OK;
 }
 
 int stokesfo_launch_info(stokesfo_ctx *c, int32_t *cells_per_tile, int32_t *grid_resid, int32_t *grid_jac,

@@ -126,7 +126,7 @@ struct RecC {
 
 // Workspace: [0, 256) header (error flag), then ntiles records.
 constexpr int64_t WS_HEADER = 256;
-enum : int { ERR_DETJ = 1, ERR_CONN = 2, ERR_CSR = 4 };
+enum : int { ERR_DETJ = 1, ERR_CONN = 2, ERR_CSR = 4, ERR_NONFINITE = 8 };
 
 // ---------------------------------------------------------------------------
 // PTX helpers (sm_90+/sm_100a): mbarrier + 1-D bulk async copies (TMA engine)

@@ -1953,6 +1953,17 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
 }
 
 // ---------------------------------------------------------------------------
+// Failure detection (STOKESFO_CHECK_FINITE=1): any non-finite value in an
+// output raises the sticky ERR_NONFINITE flag (one atomic per warp).
+// ---------------------------------------------------------------------------
+__global__ void finite_check_kernel(int64_t n, const double *__restrict__ p, int *__restrict__ err) {
+    bool bad = false;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        bad |= !isfinite(__ldcs(p + i));
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(err, ERR_NONFINITE);
+}
+
+// ---------------------------------------------------------------------------
 // G7: halo pack / unpack-add.
 // ---------------------------------------------------------------------------
 __global__ void halo_pack_kernel(int64_t n, const int32_t *__restrict__ nodes, const double2 *__restrict__ R,

@@ -21,7 +21,7 @@ QPS = {HEX8: 8, WEDGE6: 6}
 ABI_VERSION = 1
 
 GEOMETRY = {"stored": 0, "on_the_fly": 1, "compact": 2}
-STATUS = {0: "OK", 1: "EINVAL", 2: "EMESH", 3: "ECUDA", 4: "ENOMEM", 5: "EUNSUPPORTED"}
+STATUS = {0: "OK", 1: "EINVAL", 2: "EMESH", 3: "ECUDA", 4: "ENOMEM", 5: "EUNSUPPORTED", 6: "ENONFINITE"}
 
 
 class StokesFOError(RuntimeError):

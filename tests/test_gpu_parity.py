@@ -494,3 +494,28 @@ def test_jacobian_diag_parity(torch, elem, drop, geometry):
     assert (np.abs(diag.cpu().numpy() - dref) <= TOL * dref).all()
     assert not diag.cpu().numpy()[~used].any()
     _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
+
+
+@pytest.mark.parametrize("geometry", GEOMS)
+def test_check_finite_flags_nan_outputs(torch, geometry, monkeypatch):
+    """Failure detection: with STOKESFO_CHECK_FINITE=1 at create, a NaN
+    in U propagates to R / J and stokesfo_sync reports ENONFINITE; finite inputs stay OK,
+    and without the switch nothing is scanned."""
+    from paper_conf_sc_antepara0cw24_b200 import StokesFOError
+    monkeypatch.setenv("STOKESFO_CHECK_FINITE", "1")
+    ctx, orc = _setup(torch, "hex8", n=6, L=3, geometry=geometry)
+    C, nn = ctx.num_cells, ctx.num_nodes
+    J = torch.empty((C, 16, 16), dtype=torch.float64, device="cuda")
+    R = torch.zeros((nn, 2), dtype=torch.float64, device="cuda")
+    U = _t(torch, orc["U"])
+    ctx.jacobian(U, J, R=R)
+    ctx.sync()   # finite: OK
+    Ubad = U.clone()
+    Ubad[nn // 2, 0] = float("nan")
+    ctx.jacobian(Ubad, J, R=R)
+    with pytest.raises(StokesFOError, match="ENONFINITE"):
+        ctx.sync()
+    monkeypatch.setenv("STOKESFO_CHECK_FINITE", "0")
+    ctx2, _ = _setup(torch, "hex8", n=6, L=3, geometry=geometry)
+    ctx2.jacobian(Ubad, J, R=R)
+    ctx2.sync()   # not scanned
