@@ -53,6 +53,7 @@ struct stokesfo_ctx {
     const double *jmap_ptr = nullptr;
     bool jmap_ok = false;
     bool check_finite = false;  // STOKESFO_CHECK_FINITE=1 at create: scan outputs for NaN / Inf
+    bool jac_mma = false;       // hex8 stored-geometry Jacobian on the fp64 tensor cores (eval_mma_kernel)
 };
 
 namespace {
@@ -167,6 +168,19 @@ int configure_eval(int *grid) {
     return STOKESFO_OK;
 }
 
+int configure_mma(int *grid) {
+    auto fn = eval_mma_kernel<2>;
+    constexpr int bytes = MmaSmem<2>::BYTES;
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
+        return cuda_status();
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, bytes) != cudaSuccess) return cuda_status();
+    *grid = std::max(1, sms * std::max(1, per_sm));
+    return STOKESFO_OK;
+}
+
 template <class E>
 int create_impl(stokesfo_ctx *c) {
     c->N = E::N;
@@ -208,6 +222,12 @@ int create_impl(stokesfo_ctx *c) {
         st = c->nstage_jac == 3 ? configure_eval<E, M_JAC, 3>(&c->grid_jac)
                                 : configure_eval<E, M_JAC, 2>(&c->grid_jac);
         if (st) return st;
+        // hex8 Jacobian on the fp64 tensor cores (default; STOKESFO_JAC_MMA=0: the vector kernel)
+        if (E::N == 8) {
+            const char *e = getenv("STOKESFO_JAC_MMA");
+            c->jac_mma = !(e && atoi(e) == 0);
+            if (c->jac_mma && (st = configure_mma(&c->grid_jac))) return st;
+        }
         st = configure_eval<E, M_JVP, 2>(&c->grid_jvp);
         if (st) return st;
         st = configure_eval<E, M_CSR, 2>(&c->grid_csr);
@@ -328,6 +348,8 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
                                         c->stream>>>(a, jm);
     else if (otf)
         eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
+    else if (E::N == 8 && MODE == M_JAC && c->jac_mma)
+        eval_mma_kernel<2><<<(int)std::min<int64_t>(g, c->ntiles), 32, MmaSmem<2>::BYTES, c->stream>>>(a);
     else if (MODE != M_CSR && ns == 3)
         eval_kernel<E, MODE, 3><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 3>(), c->stream>>>(a, jm);
     else

@@ -25,10 +25,16 @@ struct Hex8 {
     __host__ __device__ static constexpr int lane_cell(int l) { return l / N; }
     __host__ __device__ static constexpr int lane_sub(int l) { return l % N; }
     __host__ __device__ static constexpr int lane_of(int c, int sub) { return c * N + sub; }
-    // slot of (cell c, node n) in the slab of qp q: both the per-QP loads (fixed n,
-    // lanes over (c,q)) and the per-node loads (fixed q, lanes over (c,j)) hit 16
-    // distinct bank pairs per half-warp
-    __host__ __device__ static constexpr int slot(int c, int n, int q) { return c * N + (n + q) % N; }
+    // slot of (cell c, node n) in the slab of qp q (a slab is 32 doubles = 2 x 16 bank pairs):
+    // 16 (c >> 1) + a 4-bit bank-pair index linear over GF(2) in the bits of (c, n, q),
+    //   b0 = q0 ^ n1, b1 = q1 ^ n2, b2 = q2 ^ n0, b3 = c0 ^ n1,
+    // chosen so that three access patterns each hit 16 distinct bank pairs per half-warp:
+    // the per-QP loads (fixed n, lanes over (c, q)), the vector per-node loads (fixed q, lanes
+    // over (c, j)) and the DMMA operand loads (fixed c, lanes over (n = l >> 2, q = l & 3 (+4)))
+    __host__ __device__ static constexpr int slot(int c, int n, int q) {
+        return 16 * (c >> 1) + (((q ^ (n >> 1)) & 1) | (((q >> 1) ^ (n >> 2)) & 1) << 1 |
+                                (((q >> 2) ^ n) & 1) << 2 | ((c ^ (n >> 1)) & 1) << 3);
+    }
     // gathered U/s per (cell, node) in shared memory: node slot rotated by the cell, (n + c) mod 8, so
     // that the per-QP phase's broadcast reads of one node (one address per cell) hit 4 distinct bank
     // groups: 1 wavefront per LDS.128 / LDS.64 instead of 4 / 2 (cell pitch 128 B put every cell's

@@ -1044,6 +1044,223 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
     if (JAC && l == 0) bulk_wait0();
 }
 
+// ---- G4 on the fp64 tensor cores (hex8, stored geometry, residual + element Jacobians) ----
+// The per-node phase of a cell is a dense contraction over its QPs (reading Z5):
+//   J[(i,a),(j,b)] = sum_q wmu2 G_i^T B_ab G_j + gamma h_(i,a) h_(j,b),  h_(i,a) = G_i . beta_a,
+// B_00 = diag(2, 1/2, 1/2), B_11 = diag(1/2, 2, 1/2), B_01 = [[0,1,0],[1/2,0,0],[0,0,0]], B_10 = B_01^T.
+// With S_dd = sum_q wmu2 G[d] G[d]^T and Gam_ab = sum_q gamma h_a h_b^T (8 x 8 over node pairs):
+//   J_00 = 2 S_00 + (S_11 + S_22) / 2 + Gam_00,  J_11 = 2 S_11 + (S_00 + S_22) / 2 + Gam_11,
+//   J_01 = sum_q wmu2 (G[1] G[0]^T / 2 + G[0] G[1]^T) + Gam_01,  J_10 = J_01^T.
+// Each 8 x 8 product over 8 QPs is two m8n8k4 DMMAs (k = 4 QPs); both operands of every DMMA are the
+// lane's own values in the layout lane l <-> (node i = l >> 2, qp q = (l & 3) + 4 kc), so a cell is 16
+// DMMAs + ~50 vector FP64 ops per lane (the vector form: ~160 FP64 instructions per lane and cell).
+// The C fragments hold J rows (2i, 2i+1), columns 4 (l & 3) .. +3 after one transposing shuffle of J_01:
+// two 256-bit stores per lane and cell straight to J_cell (no staging, no shared-memory round trip).
+// The per-QP phase (lane <-> (cell, qp)) and the record ring are the stored kernel's.
+__device__ __forceinline__ void dmma884(double (&d)[2], double a, double b) {
+    asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+        : "+d"(d[0]), "+d"(d[1])
+        : "d"(a), "d"(b));
+}
+__device__ __forceinline__ void st_v4_hint(double *p, double x, double y, double z, double w, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v4.f64 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "d"(x), "d"(y), "d"(z),
+                 "d"(w), "l"(pol)
+                 : "memory");
+}
+// per-QP scalars of the DMMA kernel: [NQS][TC][Q] with the QP pair (q, q + 4) adjacent (one LDS.128 per
+// field gives a lane both of its QPs); the per-QP phase's stores stay 32 consecutive doubles per field
+struct QsMma {
+    double *p;
+    __device__ __forceinline__ static int idx(int f, int c, int q) {
+        return (f * Hex8::TC + c) * Hex8::Q + 2 * (q & 3) + (q >> 2);
+    }
+    __device__ __forceinline__ double &operator()(int f, int c, int q) const { return p[idx(f, c, q)]; }
+    __device__ __forceinline__ double2 pair(int f, int c, int qq) const {
+        return *reinterpret_cast<const double2 *>(p + idx(f, c, qq));
+    }
+};
+#ifndef SFO_MMA_JAC_WARPS
+#define SFO_MMA_JAC_WARPS 12
+#endif
+template <int NSTAGE>
+struct MmaSmem {
+    using E = Hex8;
+    static constexpr int REC = Rec<E>::BYTES;
+    static constexpr int U_OFF = (int)round_up(REC, 16);
+    static constexpr int S_OFF = U_OFF + E::TC * E::UPITCH * 16;
+    static constexpr int STAGE = (int)round_up(S_OFF + E::TC * E::UPITCH * 8, 128);
+    static constexpr int OFF_QS = NSTAGE * STAGE;
+    static constexpr int OFF_BAR = OFF_QS + NQS * E::TC * E::Q * 8;
+    static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
+    static_assert(U_OFF == EvalSmem<E, M_JAC, NSTAGE>::U_OFF && S_OFF == EvalSmem<E, M_JAC, NSTAGE>::S_OFF,
+                  "gather_store / gather_load share the stored kernel's stage layout");
+};
+
+template <int NSTAGE>
+__global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_mma_kernel(EvalArgs a) {
+    using E = Hex8;
+    constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    using R = Rec<E>;
+    using S = MmaSmem<NSTAGE>;
+    extern __shared__ __align__(128) char smem[];
+    const int64_t vb = blockIdx.x, vg = gridDim.x;
+    const QsMma qs{reinterpret_cast<double *>(smem + S::OFF_QS)};
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
+    const int l = threadIdx.x & 31;
+    const int c = l >> 3, s = l & 7;    // per-QP phase: (cell, qp)
+    const int ni = l >> 2, qq = l & 3;  // DMMA fragments: (node, qp quad)
+    const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
+
+    const uint64_t pol_stream = policy_evict_first();
+    if (l == 0) {
+        for (int k = 0; k < NSTAGE; ++k) mbar_init(&bar[k], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (int k = 0; k < NSTAGE; ++k) {
+            const int64_t tile = vb + (int64_t)k * vg;
+            if (tile < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[k], R::BYTES);
+                bulk_g2s(smem + k * S::STAGE, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[k], pol_stream);
+            }
+        }
+    }
+    __syncwarp();
+    if (vb < a.ntiles) {
+        mbar_wait(&bar[0], 0);
+        gather_store<E, M_JAC>(smem, gather_load<E, M_JAC>(smem, a.U, a.surface, have_s, nullptr));
+    }
+    // phi_ni at this lane's two QPs (the body-force rows)
+    double phi[2];
+    {
+        double x, y, z, w, dx, dy, dz;
+#pragma unroll
+        for (int kc = 0; kc < 2; ++kc) {
+            qp_coords<E>(qq + 4 * kc, x, y, z, w);
+            basis<E>(ni, x, y, z, phi[kc], dx, dy, dz);
+        }
+    }
+
+    int it = 0;
+    for (int64_t tile = vb; tile < a.ntiles; tile += vg, ++it) {
+        const int st = it % NSTAGE;
+        char *stage = smem + st * S::STAGE;
+        const int32_t *rconn = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF);
+        const double *rkc = reinterpret_cast<const double *>(stage + R::KC_OFF);
+        const double *rwm = reinterpret_cast<const double *>(stage + R::WM_OFF);
+        const double *rg = reinterpret_cast<const double *>(stage + R::G_OFF);
+        const double2 *Us = reinterpret_cast<const double2 *>(stage + S::U_OFF);
+        const double *ss = reinterpret_cast<const double *>(stage + S::S_OFF);
+        const int64_t cell0 = tile * TC;
+        const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
+
+        __syncwarp();  // this tile's gathered U, s are visible
+
+        // ---- per-QP phase: lane <-> (cell c, qp s), as in eval_kernel ----
+        {
+            const int q = s;
+            double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+#pragma unroll
+            for (int n = 0; n < N; ++n) {
+                const double g0 = rg[gidx<E>(n, q, 0, c)];
+                const double g1 = rg[gidx<E>(n, q, 1, c)];
+                const double g2 = rg[gidx<E>(n, q, 2, c)];
+                const int e = E::uidx(c, n);
+                const double2 uv = Us[e];
+                ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
+                vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
+                if (have_s) {
+                    const double sn = ss[e];
+                    gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
+                }
+            }
+            qp_tail<E, M_JAC>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy, vz,
+                              gs0, gs1);
+        }
+        __syncwarp();
+
+        // ---- per-node phase on the tensor cores, one cell at a time ----
+        const int32_t gnode = rconn[R::conn(ni, qq)];  // this lane scatters R of (cell qq, node ni)
+        const int64_t ntile = tile + vg;
+        const int nst = (it + 1) % NSTAGE;
+        Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
+        double Rm0 = 0.0, Rm1 = 0.0;
+#pragma unroll 1
+        for (int cc = 0; cc < TC; ++cc) {
+            if (cc == TC / 2 && ntile < a.ntiles) {  // the next tile's gather, half a tile of latency slack
+                mbar_wait(&bar[nst], (uint32_t)(((it + 1) / NSTAGE) & 1));
+                nxt = gather_load<E, M_JAC>(smem + nst * S::STAGE, a.U, a.surface, have_s, nullptr);
+            }
+            double S00[2] = {0, 0}, S11[2] = {0, 0}, S22[2] = {0, 0}, X01[2] = {0, 0}, G00[2] = {0, 0},
+                   G11[2] = {0, 0};
+            double r0 = 0.0, r1 = 0.0;
+            const double2 b00 = qs.pair(0, cc, qq), b01 = qs.pair(1, cc, qq), b02 = qs.pair(2, cc, qq);
+            const double2 b11 = qs.pair(3, cc, qq), b12 = qs.pair(4, cc, qq), wv = qs.pair(5, cc, qq);
+            const double2 gv = qs.pair(6, cc, qq), f0 = qs.pair(7, cc, qq), f1 = qs.pair(8, cc, qq);
+#pragma unroll
+            for (int kc = 0; kc < 2; ++kc) {
+                const int q = qq + 4 * kc;
+                const double g0 = rg[gidx<E>(ni, q, 0, cc)];
+                const double g1 = rg[gidx<E>(ni, q, 1, cc)];
+                const double g2 = rg[gidx<E>(ni, q, 2, cc)];
+                const double B00 = kc ? b00.y : b00.x, B01 = kc ? b01.y : b01.x, B02 = kc ? b02.y : b02.x;
+                const double B11 = kc ? b11.y : b11.x, B12 = kc ? b12.y : b12.x;
+                const double w = kc ? wv.y : wv.x, gam = kc ? gv.y : gv.x;
+                const double wf0 = kc ? f0.y : f0.x, wf1 = kc ? f1.y : f1.x;
+                const double h0 = fma(g2, B02, fma(g1, B01, g0 * B00));
+                const double h1 = fma(g2, B12, fma(g1, B11, g0 * B01));
+                r0 = fma(wf0, phi[kc], fma(w, h0, r0));
+                r1 = fma(wf1, phi[kc], fma(w, h1, r1));
+                const double wg0 = w * g0, wg1 = w * g1;
+                dmma884(S00, g0, wg0);
+                dmma884(S11, g1, wg1);
+                dmma884(S22, g2, w * g2);
+                dmma884(X01, g1, 0.5 * wg0);
+                dmma884(X01, g0, wg1);
+                const double gh1 = gam * h1;
+                dmma884(G00, h0, gam * h0);
+                dmma884(G11, h1, gh1);
+                dmma884(X01, h0, gh1);
+            }
+            // residual rows of (cc, ni): sum over the 4 lanes of the node's QP quads
+            r0 += __shfl_xor_sync(0xffffffffu, r0, 1);
+            r1 += __shfl_xor_sync(0xffffffffu, r1, 1);
+            r0 += __shfl_xor_sync(0xffffffffu, r0, 2);
+            r1 += __shfl_xor_sync(0xffffffffu, r1, 2);
+            if (qq == cc) {
+                Rm0 = r0;
+                Rm1 = r1;
+            }
+            // J_10[ni][2qq + e] = J_01[2qq + e][ni]: lane (2qq + e, ni >> 1), element ni & 1
+            const int src0 = 8 * qq + (ni >> 1), src1 = src0 + 4;
+            const double t00 = __shfl_sync(0xffffffffu, X01[0], src0), t01 = __shfl_sync(0xffffffffu, X01[1], src0);
+            const double t10 = __shfl_sync(0xffffffffu, X01[0], src1), t11 = __shfl_sync(0xffffffffu, X01[1], src1);
+            const double j10a = (ni & 1) ? t01 : t00, j10b = (ni & 1) ? t11 : t10;
+            if (cc < nvalid) {
+                double *Jr = a.J_cell + (cell0 + cc) * (4 * N * N) + (2 * ni) * (2 * N) + 4 * qq;
+                const double j00a = fma(2.0, S00[0], fma(0.5, S11[0] + S22[0], G00[0]));
+                const double j00b = fma(2.0, S00[1], fma(0.5, S11[1] + S22[1], G00[1]));
+                const double j11a = fma(2.0, S11[0], fma(0.5, S00[0] + S22[0], G11[0]));
+                const double j11b = fma(2.0, S11[1], fma(0.5, S00[1] + S22[1], G11[1]));
+                st_v4_hint(Jr, j00a, X01[0], j00b, X01[1], pol_stream);
+                st_v4_hint(Jr + 2 * N, j10a, j11a, j10b, j11b, pol_stream);
+            }
+        }
+        __syncwarp();  // every lane is done with this stage's record and per-QP scalars
+
+        if (l == 0) {
+            const int64_t nt = tile + (int64_t)NSTAGE * vg;
+            if (nt < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[st], R::BYTES);
+                bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
+            }
+        }
+        if (qq < nvalid) {
+            if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, Rm0, Rm1);
+            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + qq) * N + ni) * 2) = make_double2(Rm0, Rm1);
+        }
+        if (ntile < a.ntiles) gather_store<E, M_JAC>(smem + nst * S::STAGE, nxt);
+    }
+}
+
 // ---- G3/G4 with compact stored geometry (A_q = J_q^-T streamed per tile) ----
 // The stored kernel's TMA record ring and register gather, with the compact
 // record (RecC): the per-QP phase forms GradBF_n(q) = A_q grad_xi phi_n(xi_q)
