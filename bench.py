@@ -36,8 +36,36 @@ WORKLOADS = {
 }
 
 
+def jac_mma(elem: str, geometry: str, packed: bool = False) -> bool:
+    """The element Jacobians run on the fp64 tensor cores (eval_mma_kernel / eval_compact_mma_kernel): stored
+    or compact geometry; STOKESFO_JAC_MMA (read by stokesfo_create) unset: hex8 only, 1: both elements, 0:
+    neither. The packed form (stokesfo_jacobian_packed) always comes from them unless STOKESFO_JAC_MMA=0."""
+    v = os.environ.get("STOKESFO_JAC_MMA")
+    if geometry == "on_the_fly" or v == "0":
+        return False
+    return packed or v == "1" or elem == "hex8"
+
+
+def kernel_name(elem: str, geometry: str, op: str, packed: bool = False) -> str:
+    E = "Hex8" if elem == "hex8" else "Wedge6"
+    if op in ("jacobian", "jac_global") and (packed or jac_mma(elem, geometry)):
+        k = ("eval_compact_mma_kernel<" if geometry == "compact" else "eval_mma_kernel<") + E + ">"
+        if op == "jacobian":
+            return k + " (stokesfo_jacobian)"
+        if packed:
+            return k + " (stokesfo_jacobian_packed) + csr_gather_kernel<packed> (stokesfo_assemble_csr_packed " \
+                       "overwriting, both timed)"
+        return k + " (stokesfo_jacobian) + csr_gather_kernel (stokesfo_assemble_csr overwriting, both timed)"
+    k = {"on_the_fly": "eval_otf_kernel", "compact": "eval_compact_kernel", "stored": "eval_kernel"}[geometry]
+    k += "<" + E + "," + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jvp_y": "M_JVP>",
+                         "jac_csr": "M_CSR>", "jac_global": "M_JAC> + csr_gather_kernel"}[op]
+    return k + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
+                "jvp": " (stokesfo_jvp)", "jvp_y": " (stokesfo_jvp, R = NULL)", "jac_csr": " (stokesfo_jacobian_csr)",
+                "jac_global": " (stokesfo_jacobian + stokesfo_assemble_csr overwriting, both timed)"}[op]
+
+
 def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored", op: str = "jacobian",
-                     nnz: int = 0) -> int:
+                     nnz: int = 0, packed: bool = False) -> int:
     """Algorithmic (compulsory) HBM bytes of one stokesfo_jacobian launch with
     assembled R.
     stored:     per cell conn 4N + GradBF 24NQ + wMeasure 8Q + k_c 8 + J_cell 8(2N)^2;
@@ -58,7 +86,8 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
         # jacobian (J_cell written) + pull assembly overwriting the CSR values (DESIGN §6 NEXT-2): J_cell read
         # again, per cell the slot row 8N and incidence 4N, per node rowptr pair 16 + incidence pointer 8,
         # every CSR value written once (8 nnz)
-        J = 2 * 8 * (2 * N) ** 2 + 8 * N + 4 * N
+        # packed: the N(N+1)/2 upper 2 x 2 node blocks (symmetric J) written and read instead of (2N)^2 entries
+        J = 2 * 8 * (4 * N * (N + 1) // 2 if packed else (2 * N) ** 2) + 8 * N + 4 * N
         xy = 24
     vals = {"jac_csr": 16 * nnz, "jac_global": 8 * nnz}.get(op, 0)
     if geometry == "on_the_fly":
@@ -302,6 +331,9 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly", "compact"])
+    ap.add_argument("--global-format", default="packed", choices=["packed", "full"],
+                    help="--op jac_global: element matrices in symmetric block-packed form (tensor-core kernels) "
+                         "or full [C][2N][2N]")
     ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jvp_y", "jac_csr", "jac_global"],
                     help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
                          "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
@@ -360,7 +392,9 @@ def main():
     if world > 1 and args.op in ("jac_csr", "jac_global", "jvp_y"):
         sys.stderr.write("bench.py: --op jac_csr / jac_global / jvp_y are single-GPU lines\n")
         return 2
-    J = torch.empty((C, 2 * N, 2 * N) if args.op in ("jacobian", "jac_global") else (0,), dtype=torch.float64,
+    packed = args.op == "jac_global" and args.global_format == "packed" and jac_mma(elem, args.geometry, True)   # NEXT-2 through symmetric block-packed J
+    J = torch.empty((C, N * (N + 1) // 2, 2, 2) if packed else
+                    ((C, 2 * N, 2 * N) if args.op in ("jacobian", "jac_global") else (0,)), dtype=torch.float64,
                     device=dev)
     # J.v direction: one global seeded field, restricted to this rank's nodes (consistent across ranks)
     JV = args.op in ("jvp", "jvp_y")
@@ -420,6 +454,9 @@ def main():
             ctx.jacobian(Uc, J, R=Rc)
         elif args.op == "jac_csr":
             ctx.jacobian_csr(Uc, vals, R=Rc)
+        elif args.op == "jac_global" and packed:   # packed element matrices, then the pull assembly
+            ctx.jacobian_packed(Uc, J, R=Rc)
+            ctx.assemble_csr_packed(J, vals, accumulate=False)
         elif args.op == "jac_global":   # element matrices, then the atomic-free pull assembly overwriting CSR
             ctx.jacobian(Uc, J, R=Rc)
             ctx.assemble_csr(J, vals, accumulate=False)
@@ -636,7 +673,7 @@ def main():
 
     if rank == 0:
         peak, peak_src = load_peaks()
-        bpl = bytes_per_launch(elem, C, NN, args.geometry, args.op, nnz)
+        bpl = bytes_per_launch(elem, C, NN, args.geometry, args.op, nnz, packed)
         achieved = bpl / (kern_ms_max * 1e-3) / 1e9
         traffic, traffic_src = lookup_traffic(args.config, elem, args.op, args.geometry, world)
         l2_bytes = 126 * 2 ** 20
@@ -648,8 +685,8 @@ def main():
                                 "and achieved HBM GB/s",
                        "jac_csr": "Stokes-FO residual + Jacobian assembled into global CSR (stokesfo_jacobian_csr) "
                                   "cells/s and achieved HBM GB/s",
-                       "jac_global": "Stokes-FO residual + Jacobian assembled into global CSR (stokesfo_jacobian + "
-                                     "stokesfo_scatter_assemble) cells/s and achieved HBM GB/s"}[args.op],
+                       "jac_global": "Stokes-FO residual + Jacobian assembled into global CSR (element matrices + "
+                                     "pull assembly) cells/s and achieved HBM GB/s"}[args.op],
             "value": total_cells / (ms_step * 1e-3),
             "unit": "cells/s",
             "n_gpus": world,
@@ -669,16 +706,7 @@ def main():
                        "launch": ctx.launch_info()},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
-                         "kernel": {"on_the_fly": "eval_otf_kernel", "compact": "eval_compact_kernel",
-                                    "stored": "eval_kernel"}[args.geometry]
-                         + ("<Hex8," if elem == "hex8" else "<Wedge6,")
-                         + {"jacobian": "M_JAC>", "resid": "M_RESID>", "jvp": "M_JVP>", "jvp_y": "M_JVP>",
-                            "jac_csr": "M_CSR>",
-                            "jac_global": "M_JAC> + csr_gather_kernel"}[args.op]
-                         + {"jacobian": " (stokesfo_jacobian)", "resid": " (stokesfo_viscosity_resid)",
-                            "jvp": " (stokesfo_jvp)", "jvp_y": " (stokesfo_jvp, R = NULL)",
-                            "jac_csr": " (stokesfo_jacobian_csr)",
-                            "jac_global": " (stokesfo_jacobian + stokesfo_assemble_csr overwriting, both timed)"}[args.op],
+                         "kernel": kernel_name(elem, args.geometry, args.op, packed),
                          "kernel_ms": kern_ms_max, "algorithmic_bytes_per_launch": bpl, "peak_source": peak_src,
                          "live_copy_gbs": live_copy,
                          "note": "live_copy_gbs: torch device-to-device copy of 2 GiB on this box before the timed "

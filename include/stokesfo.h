@@ -208,6 +208,23 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R,
  * csr_vals: dev [nnz]. */
 int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_vals, int accumulate);
 
+/* NEXT-2 element Jacobians in symmetric block-packed form.  The element tangent
+ * is the Hessian of the cell's quadrature energy sum_q wM Psi(eps_e^2) (Glen's law
+ * is a potential flow law; section III-A; reading Z5), so
+ * J_cell[c] is symmetric and its N(N+1)/2 upper 2 x 2 node blocks determine it:
+ * Jp dev [C][N(N+1)/2][2][2], block (i, j >= i) at index i N - i (i - 1) / 2 +
+ * (j - i), entries [a][b] = J[(i,a),(j,b)] (hex8 1,152 B per cell instead of
+ * 2,048; wedge6 672 instead of 1,152).  Jp must be 32-B aligned.  R_cell and R
+ * as stokesfo_jacobian.  Written by the fp64 tensor-core kernels (stored or
+ * compact geometry): on-the-fly geometry or STOKESFO_JAC_MMA=0 at create return
+ * EUNSUPPORTED. */
+int stokesfo_jacobian_packed(stokesfo_ctx *c, const double *U, double *Jp, double *R_cell, double *R);
+
+/* stokesfo_assemble_csr from the packed form: row (i, a) of cell c is block
+ * (i, j) for j >= i and the transpose of block (j, i) for j < i.  Same
+ * requirements, ordering and accumulate semantics as stokesfo_assemble_csr. */
+int stokesfo_assemble_csr_packed(stokesfo_ctx *c, const double *Jp, double *csr_vals, int accumulate);
+
 /* CSR pattern over dofs (rows = 2*num_nodes; columns of a row = sorted dofs of
  * every node sharing a cell with the row's node).  Size query: pass rowptr =
  * colidx = NULL to get *nnz.  Fill: rowptr dev [2*num_nodes+1] int64, colidx

@@ -53,7 +53,9 @@ struct stokesfo_ctx {
     const double *jmap_ptr = nullptr;
     bool jmap_ok = false;
     bool check_finite = false;  // STOKESFO_CHECK_FINITE=1 at create: scan outputs for NaN / Inf
-    bool jac_mma = false;       // hex8 stored-geometry Jacobian on the fp64 tensor cores (eval_mma_kernel)
+    bool jac_mma = false;       // Jacobian on the fp64 tensor cores (eval_mma_kernel / eval_compact_mma_kernel)
+    bool mma_ok = false;        // the DMMA kernels are configured (stokesfo_jacobian_packed)
+    int grid_mma = 0;           // their persistent grid
 };
 
 namespace {
@@ -168,9 +170,10 @@ int configure_eval(int *grid) {
     return STOKESFO_OK;
 }
 
+template <class E>
 int configure_mma(int *grid) {
-    auto fn = eval_mma_kernel<2>;
-    constexpr int bytes = MmaSmem<2>::BYTES;
+    auto fn = eval_mma_kernel<E, 2>;
+    constexpr int bytes = MmaSmem<E, 2>::BYTES;
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
         return cuda_status();
     int dev = 0, sms = 0, per_sm = 0;
@@ -179,6 +182,34 @@ int configure_mma(int *grid) {
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, bytes) != cudaSuccess) return cuda_status();
     *grid = std::max(1, sms * std::max(1, per_sm));
     return STOKESFO_OK;
+}
+
+template <class E>
+int configure_compact_mma(int *grid) {
+    auto fn = eval_compact_mma_kernel<E>;
+    constexpr int bytes = CompactMmaSmem<E>::BYTES;
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
+        return cuda_status();
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, bytes) != cudaSuccess) return cuda_status();
+    *grid = std::max(1, sms * std::max(1, per_sm));
+    return STOKESFO_OK;
+}
+
+// Element Jacobians on the fp64 tensor cores. STOKESFO_JAC_MMA unset: hex8 (the DMMA kernels cost the same per
+// cell for both elements, which beats the vector kernel for hex8's 8 x 8 node blocks but not for wedge6's
+// padded 6 x 6); 1: both elements; 0: neither (and no packed form). The DMMA kernels are configured
+// unless 0: stokesfo_jacobian_packed always runs on them.
+inline int jac_mma_env() {
+    const char *e = getenv("STOKESFO_JAC_MMA");
+    return e ? atoi(e) : -1;
+}
+template <class E>
+bool want_jac_mma() {
+    const int v = jac_mma_env();
+    return v == 1 || (v < 0 && E::N == 8);
 }
 
 template <class E>
@@ -195,6 +226,9 @@ int create_impl(stokesfo_ctx *c) {
         c->nstage_resid = c->nstage_jac = 2;
         if ((st = configure_compact<E, M_RESID>(&c->grid_resid))) return st;
         if ((st = configure_compact<E, M_JAC>(&c->grid_jac))) return st;
+        c->jac_mma = want_jac_mma<E>();
+        c->mma_ok = jac_mma_env() != 0;
+        if (c->mma_ok && (st = configure_compact_mma<E>(&c->grid_mma))) return st;
         if ((st = configure_compact<E, M_JVP>(&c->grid_jvp))) return st;
         if ((st = configure_compact<E, M_CSR>(&c->grid_csr))) return st;
         if ((st = configure_compact<E, M_DIAG>(&c->grid_diag))) return st;
@@ -222,12 +256,9 @@ int create_impl(stokesfo_ctx *c) {
         st = c->nstage_jac == 3 ? configure_eval<E, M_JAC, 3>(&c->grid_jac)
                                 : configure_eval<E, M_JAC, 2>(&c->grid_jac);
         if (st) return st;
-        // hex8 Jacobian on the fp64 tensor cores (default; STOKESFO_JAC_MMA=0: the vector kernel)
-        if (E::N == 8) {
-            const char *e = getenv("STOKESFO_JAC_MMA");
-            c->jac_mma = !(e && atoi(e) == 0);
-            if (c->jac_mma && (st = configure_mma(&c->grid_jac))) return st;
-        }
+        c->jac_mma = want_jac_mma<E>();
+        c->mma_ok = jac_mma_env() != 0;
+        if (c->mma_ok && (st = configure_mma<E>(&c->grid_mma))) return st;
         st = configure_eval<E, M_JVP, 2>(&c->grid_jvp);
         if (st) return st;
         st = configure_eval<E, M_CSR, 2>(&c->grid_csr);
@@ -304,7 +335,7 @@ bool wedge_jmap(stokesfo_ctx *c, const double *J_cell) {
 
 template <class E, int MODE>
 int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, double *R, double *J_cell,
-              const double *X = nullptr, double *Y = nullptr, double *csr_vals = nullptr) {
+              const double *X = nullptr, double *Y = nullptr, double *csr_vals = nullptr, bool packed = false) {
     if (c->ntiles == 0) return STOKESFO_OK;
     EvalArgs a;
     a.recs = c->recs;
@@ -333,23 +364,30 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     a.rowptr = c->rowptr;
     a.slots = c->slots;
     a.csr_vals = csr_vals;
+    a.packed = packed ? 1 : 0;
     const int g = MODE == M_JAC ? c->grid_jac
                 : MODE == M_JVP ? c->grid_jvp
                 : MODE == M_CSR ? c->grid_csr
                 : MODE == M_DIAG ? c->grid_diag : c->grid_resid;
     const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
-    a.use_jmap = (!otf && MODE == M_JAC && wedge_jmap<E>(c, J_cell)) ? 1 : 0;
+    // the DMMA kernels store J with 32-B vector stores (16-B aligned J_cell: the vector kernels)
+    const bool mma = MODE == M_JAC && !otf && c->mma_ok && (c->jac_mma || packed) && aligned(J_cell, 32);
+    if (packed && !mma) return STOKESFO_EUNSUPPORTED;  // the packed form comes from the DMMA kernels only
+    a.use_jmap = (!otf && !mma && MODE == M_JAC && wedge_jmap<E>(c, J_cell)) ? 1 : 0;
     const CUtensorMap jm = a.use_jmap ? c->jmap : CUtensorMap{};
     constexpr int WPC = warps_per_cta<E, MODE>();  // eval_kernel only (the on-the-fly kernel: 1)
     const int grid = (int)std::min<int64_t>(g, otf ? c->ntiles : (c->ntiles + WPC - 1) / WPC);
     const int ns = MODE == M_JAC ? c->nstage_jac : (MODE == M_RESID ? c->nstage_resid : 2);
-    if (c->mode == STOKESFO_GEOMETRY_COMPACT)
+    const int gm = (int)std::min<int64_t>(c->grid_mma, c->ntiles);
+    if (mma && c->mode == STOKESFO_GEOMETRY_COMPACT)
+        eval_compact_mma_kernel<E><<<gm, 32, CompactMmaSmem<E>::BYTES, c->stream>>>(a);
+    else if (c->mode == STOKESFO_GEOMETRY_COMPACT)
         eval_compact_kernel<E, MODE><<<(int)std::min<int64_t>(g, c->ntiles), 32, CompactSmem<E, MODE>::BYTES,
                                         c->stream>>>(a, jm);
     else if (otf)
         eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
-    else if (E::N == 8 && MODE == M_JAC && c->jac_mma)
-        eval_mma_kernel<2><<<(int)std::min<int64_t>(g, c->ntiles), 32, MmaSmem<2>::BYTES, c->stream>>>(a);
+    else if (mma)
+        eval_mma_kernel<E, 2><<<gm, 32, MmaSmem<E, 2>::BYTES, c->stream>>>(a);
     else if (MODE != M_CSR && ns == 3)
         eval_kernel<E, MODE, 3><<<grid, 32 * WPC, eval_smem_bytes<E, MODE, 3>(), c->stream>>>(a, jm);
     else
@@ -371,7 +409,9 @@ const char *stokesfo_strerror(int s) {
         case STOKESFO_EMESH: return "mesh error (det J <= 0, conn out of range or CSR entry missing)";
         case STOKESFO_ECUDA: return "CUDA runtime error";
         case STOKESFO_ENOMEM: return "workspace too small";
-        case STOKESFO_EUNSUPPORTED: return "unsupported configuration (glen_n must be 3)";
+        case STOKESFO_EUNSUPPORTED:
+            return "unsupported configuration (glen_n != 3, a node degree beyond the CSR kernels, or a packed "
+                   "Jacobian without the tensor-core kernels)";
         case STOKESFO_ENONFINITE: return "non-finite value in an output (STOKESFO_CHECK_FINITE=1)";
         default: return "unknown status";
     }
@@ -491,6 +531,25 @@ int stokesfo_jacobian(stokesfo_ctx *c, const double *U, double *J_cell, double *
 #undef CALL
     if (st == STOKESFO_OK) {
         check_finite(c, J_cell, c->d.num_cells * 4 * c->N * c->N);
+        check_finite(c, R_cell, c->d.num_cells * c->N * 2);
+        check_finite(c, R, c->d.num_nodes * 2);
+    }
+    return st == STOKESFO_OK ? cuda_status() : st;
+}
+
+int stokesfo_jacobian_packed(stokesfo_ctx *c, const double *U, double *Jp, double *R_cell, double *R) {
+    SFO_RANGE("stokesfo_jacobian_packed");
+    if (!c) return STOKESFO_EINVAL;
+    if (c->d.num_cells == 0) return STOKESFO_OK;
+    if (!U || !Jp || !aligned(U, 16) || !aligned(Jp, 32)) return STOKESFO_EINVAL;
+    const void *ps[] = {R_cell, R};
+    for (const void *p : ps)
+        if (p && !aligned(p, 16)) return STOKESFO_EINVAL;
+#define CALL(E) eval_impl<E, M_JAC>(c, U, nullptr, R_cell, R, Jp, nullptr, nullptr, nullptr, true)
+    const int st = DISPATCH(c, CALL);
+#undef CALL
+    if (st == STOKESFO_OK) {
+        check_finite(c, Jp, c->d.num_cells * 2 * c->N * (c->N + 1));
         check_finite(c, R_cell, c->d.num_cells * c->N * 2);
         check_finite(c, R, c->d.num_nodes * 2);
     }
@@ -684,8 +743,9 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
     return cuda_status();
 }
 
-int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_vals, int accumulate) {
-    SFO_RANGE("stokesfo_assemble_csr");
+}  // extern "C"
+template <bool PACKED>
+static int assemble_csr_impl(stokesfo_ctx *c, const double *J_cell, double *csr_vals, int accumulate) {
     if (!c || !J_cell || !csr_vals || !aligned(J_cell, 16) || !aligned(csr_vals, 16)) return STOKESFO_EINVAL;
     if (!c->slots || !c->inc || !c->rowptr) return STOKESFO_EINVAL;  // needs stokesfo_csr_slots
     if (c->csr_maxdeg > CSR_GATHER_MAXDEG) return STOKESFO_EUNSUPPORTED;
@@ -695,13 +755,25 @@ int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_val
     const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
     const int bt = 32 * CSR_GATHER_WARPS;
     if (c->N == 8) {
-        if (accumulate) csr_gather_kernel<8, true><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
-        else csr_gather_kernel<8, false><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+        if (accumulate) csr_gather_kernel<8, true, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+        else csr_gather_kernel<8, false, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
     } else {
-        if (accumulate) csr_gather_kernel<6, true><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
-        else csr_gather_kernel<6, false><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+        if (accumulate) csr_gather_kernel<6, true, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+        else csr_gather_kernel<6, false, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
     }
     return cuda_status();
+}
+
+extern "C" {
+
+int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_vals, int accumulate) {
+    SFO_RANGE("stokesfo_assemble_csr");
+    return assemble_csr_impl<false>(c, J_cell, csr_vals, accumulate);
+}
+
+int stokesfo_assemble_csr_packed(stokesfo_ctx *c, const double *Jp, double *csr_vals, int accumulate) {
+    SFO_RANGE("stokesfo_assemble_csr_packed");
+    return assemble_csr_impl<true>(c, Jp, csr_vals, accumulate);
 }
 
 int stokesfo_geometry(stokesfo_ctx *c, double *grad_bf, double *w_measure) {

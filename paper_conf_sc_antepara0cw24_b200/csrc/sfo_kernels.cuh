@@ -315,7 +315,19 @@ struct EvalArgs {
     const uint64_t *slots;    // [C][N] rows of N uint8 slots (8-byte pitch)
     double *csr_vals;         // [nnz] (+=)
     int use_jmap;             // wedge6 M_JAC: J tile stored through the kernel's tensor-map parameter
+    int packed;               // M_JAC on the DMMA kernels: J_cell holds the symmetric block-packed form
 };
+
+// Symmetric block-packed element matrix (stokesfo_jacobian_packed): the N(N+1)/2 upper 2 x 2 node blocks
+// (i, j >= i) of J_cell[c], block index i N - i (i - 1) / 2 + (j - i), entries [a][b] = J[(i,a),(j,b)].
+template <int N>
+__host__ __device__ __forceinline__ constexpr int pk_block(int i, int j) {
+    return i * N - i * (i - 1) / 2 + (j - i);
+}
+template <int N>
+__host__ __device__ constexpr int pk_blocks() {
+    return N * (N + 1) / 2;
+}
 
 constexpr int REM_MAX = 7;                 // remote copies of one node (<= 8 parts meet at a vertex)
 constexpr int REM_ROW = 1 + 2 * REM_MAX;
@@ -1044,19 +1056,28 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
     if (JAC && l == 0) bulk_wait0();
 }
 
-// ---- G4 on the fp64 tensor cores (hex8, stored geometry, residual + element Jacobians) ----
+// ---- G4 on the fp64 tensor cores (residual + element Jacobians; hex8 and wedge6) ----
 // The per-node phase of a cell is a dense contraction over its QPs (reading Z5):
 //   J[(i,a),(j,b)] = sum_q wmu2 G_i^T B_ab G_j + gamma h_(i,a) h_(j,b),  h_(i,a) = G_i . beta_a,
 // B_00 = diag(2, 1/2, 1/2), B_11 = diag(1/2, 2, 1/2), B_01 = [[0,1,0],[1/2,0,0],[0,0,0]], B_10 = B_01^T.
-// With S_dd = sum_q wmu2 G[d] G[d]^T and Gam_ab = sum_q gamma h_a h_b^T (8 x 8 over node pairs):
+// With S_dd = sum_q wmu2 G[d] G[d]^T and Gam_ab = sum_q gamma h_a h_b^T (N x N over node pairs):
 //   J_00 = 2 S_00 + (S_11 + S_22) / 2 + Gam_00,  J_11 = 2 S_11 + (S_00 + S_22) / 2 + Gam_11,
 //   J_01 = sum_q wmu2 (G[1] G[0]^T / 2 + G[0] G[1]^T) + Gam_01,  J_10 = J_01^T.
-// Each 8 x 8 product over 8 QPs is two m8n8k4 DMMAs (k = 4 QPs); both operands of every DMMA are the
+// Each N x N product over Q QPs is two m8n8k4 DMMAs (k = 4 QPs); both operands of every DMMA are the
 // lane's own values in the layout lane l <-> (node i = l >> 2, qp q = (l & 3) + 4 kc), so a cell is 16
 // DMMAs + ~50 vector FP64 ops per lane (the vector form: ~160 FP64 instructions per lane and cell).
+// wedge6 pads the 6 x 6 node blocks to 8 x 8 and its 6 QPs to 8 (zero operands: lanes i >= 6, and
+// q >= 6 in the second k step), the same 16 DMMAs per cell.
 // The C fragments hold J rows (2i, 2i+1), columns 4 (l & 3) .. +3 after one transposing shuffle of J_01:
-// two 256-bit stores per lane and cell straight to J_cell (no staging, no shared-memory round trip).
+// two 256-bit stores per lane and cell straight to J_cell (no staging, no shared-memory round trip;
+// J_cell 32-B aligned, else the vector kernels run).
 // The per-QP phase (lane <-> (cell, qp)) and the record ring are the stored kernel's.
+#ifndef SFO_MMA_SPLIT
+#define SFO_MMA_SPLIT 1
+#endif
+#ifndef SFO_MMA_UNROLL
+#define SFO_MMA_UNROLL 1
+#endif
 __device__ __forceinline__ void dmma884(double (&d)[2], double a, double b) {
     asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
         : "+d"(d[0]), "+d"(d[1])
@@ -1067,48 +1088,184 @@ __device__ __forceinline__ void st_v4_hint(double *p, double x, double y, double
                  "d"(w), "l"(pol)
                  : "memory");
 }
-// per-QP scalars of the DMMA kernel: [NQS][TC][Q] with the QP pair (q, q + 4) adjacent (one LDS.128 per
-// field gives a lane both of its QPs); the per-QP phase's stores stay 32 consecutive doubles per field
+// per-QP scalars of the DMMA kernels: [NQS][TC][8] with the QP pair (q, q + 4) adjacent (one LDS.128 per
+// field gives a lane both of its QPs); wedge6's slots of q = 6, 7 are never written (the readers zero them)
+template <class E>
 struct QsMma {
     double *p;
-    __device__ __forceinline__ static int idx(int f, int c, int q) {
-        return (f * Hex8::TC + c) * Hex8::Q + 2 * (q & 3) + (q >> 2);
-    }
+    __device__ __forceinline__ static int idx(int f, int c, int q) { return (f * E::TC + c) * 8 + 2 * (q & 3) + (q >> 2); }
     __device__ __forceinline__ double &operator()(int f, int c, int q) const { return p[idx(f, c, q)]; }
     __device__ __forceinline__ double2 pair(int f, int c, int qq) const {
         return *reinterpret_cast<const double2 *>(p + idx(f, c, qq));
     }
 };
+template <class E>
+constexpr int qs_mma_bytes() {
+    return NQS * E::TC * 8 * 8;
+}
+
+// phi_ni at the lane's two DMMA QPs (qq, qq + 4): the body-force rows (0 on padding lanes / QPs)
+template <class E>
+__device__ __forceinline__ void mma_phi(int ni, int qq, double (&phi)[2]) {
+    double x, y, z, w, dx, dy, dz;
+#pragma unroll
+    for (int kc = 0; kc < 2; ++kc) {
+        const int q = qq + 4 * kc;
+        phi[kc] = 0.0;
+        if (ni < E::N && q < E::Q) {
+            qp_coords<E>(q, x, y, z, w);
+            basis<E>(ni, x, y, z, phi[kc], dx, dy, dz);
+        }
+    }
+}
+
+// The DMMA per-node phase of one tile: GradBF rg in the record slot layout (Rec<E>::g), per-QP scalars in
+// the QsMma layout; lane (ni, qq) returns the residual rows of (cell qq, node ni) in Rm[0] (and, wedge6's
+// fifth cell, of (cell 4, node ni) in Rm[1] on the lanes qq == 0) and writes the element Jacobians of the
+// tile's valid cells straight to J_cell.  pf() is called once, before cell TC / 2.
+template <class E, class PF>
+__device__ __forceinline__ void mma_node_phase(double *__restrict__ J_cell, const double *rg, const QsMma<E> &qs,
+                                               const double (&phi)[2], int64_t cell0, int nvalid, int ni, int qq,
+                                               uint64_t pol, double (&Rm)[2][2], bool packed, PF pf) {
+    constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    static_assert(N <= 8 && Q <= 8 && Q > 4 && TC <= 5, "two k steps of 4 QPs, 8 x 8 node blocks");
+    const bool node_ok = N == 8 || ni < N;
+#if SFO_MMA_UNROLL == 2
+#pragma unroll 2
+#else
+#pragma unroll 1
+#endif
+    for (int cc = 0; cc < TC; ++cc) {
+        if (cc == TC / 2) pf();
+        double S00[2] = {0, 0}, S11[2] = {0, 0}, S22[2] = {0, 0}, X01[2] = {0, 0}, G00[2] = {0, 0},
+               G11[2] = {0, 0};
+        // J_01's three products in independent accumulators (dependent DMMA chains of 2, not 6; SFO_MMA_SPLIT)
+        double Xb[2] = {0, 0}, Xc[2] = {0, 0};
+        double r0 = 0.0, r1 = 0.0;
+        const double2 b00 = qs.pair(0, cc, qq), b01 = qs.pair(1, cc, qq), b02 = qs.pair(2, cc, qq);
+        const double2 b11 = qs.pair(3, cc, qq), b12 = qs.pair(4, cc, qq), wv = qs.pair(5, cc, qq);
+        const double2 gv = qs.pair(6, cc, qq), f0 = qs.pair(7, cc, qq), f1 = qs.pair(8, cc, qq);
+#pragma unroll
+        for (int kc = 0; kc < 2; ++kc) {
+            const int q = qq + 4 * kc;
+            const bool q_ok = Q == 8 || q < Q;  // wedge6: QPs 6, 7 of the second k step are padding
+            const bool ok = node_ok && q_ok;
+            const double g0 = ok ? rg[gidx<E>(ni, q, 0, cc)] : 0.0;
+            const double g1 = ok ? rg[gidx<E>(ni, q, 1, cc)] : 0.0;
+            const double g2 = ok ? rg[gidx<E>(ni, q, 2, cc)] : 0.0;
+            const double B00 = kc ? b00.y : b00.x, B01 = kc ? b01.y : b01.x, B02 = kc ? b02.y : b02.x;
+            const double B11 = kc ? b11.y : b11.x, B12 = kc ? b12.y : b12.x;
+            const double w = q_ok ? (kc ? wv.y : wv.x) : 0.0, gam = q_ok ? (kc ? gv.y : gv.x) : 0.0;
+            const double wf0 = q_ok ? (kc ? f0.y : f0.x) : 0.0, wf1 = q_ok ? (kc ? f1.y : f1.x) : 0.0;
+            const double h0 = q_ok ? fma(g2, B02, fma(g1, B01, g0 * B00)) : 0.0;
+            const double h1 = q_ok ? fma(g2, B12, fma(g1, B11, g0 * B01)) : 0.0;
+            r0 = fma(wf0, phi[kc], fma(w, h0, r0));
+            r1 = fma(wf1, phi[kc], fma(w, h1, r1));
+            const double wg0 = w * g0, wg1 = w * g1;
+            dmma884(S00, g0, wg0);
+            dmma884(S11, g1, wg1);
+            dmma884(S22, g2, w * g2);
+            dmma884(X01, g1, 0.5 * wg0);
+            dmma884(SFO_MMA_SPLIT ? Xb : X01, g0, wg1);
+            const double gh1 = gam * h1;
+            dmma884(G00, h0, gam * h0);
+            dmma884(G11, h1, gh1);
+            dmma884(SFO_MMA_SPLIT ? Xc : X01, h0, gh1);
+        }
+        if (SFO_MMA_SPLIT) {
+            X01[0] += Xb[0] + Xc[0];
+            X01[1] += Xb[1] + Xc[1];
+        }
+        // residual rows of (cc, ni): sum over the 4 lanes of the node's QP quads
+        r0 += __shfl_xor_sync(0xffffffffu, r0, 1);
+        r1 += __shfl_xor_sync(0xffffffffu, r1, 1);
+        r0 += __shfl_xor_sync(0xffffffffu, r0, 2);
+        r1 += __shfl_xor_sync(0xffffffffu, r1, 2);
+        if (qq == cc) {
+            Rm[0][0] = r0;
+            Rm[0][1] = r1;
+        }
+        if (TC > 4 && cc == 4 && qq == 0) {
+            Rm[1][0] = r0;
+            Rm[1][1] = r1;
+        }
+        // J_10[ni][2qq + e] = J_01[2qq + e][ni]: lane (2qq + e, ni >> 1), element ni & 1
+        const int src0 = 8 * qq + (ni >> 1), src1 = src0 + 4;
+        const double t00 = __shfl_sync(0xffffffffu, X01[0], src0), t01 = __shfl_sync(0xffffffffu, X01[1], src0);
+        const double t10 = __shfl_sync(0xffffffffu, X01[0], src1), t11 = __shfl_sync(0xffffffffu, X01[1], src1);
+        const double j10a = (ni & 1) ? t01 : t00, j10b = (ni & 1) ? t11 : t10;
+        if (cc < nvalid && node_ok && (N == 8 || 2 * qq < N)) {
+            double *Jr = J_cell + (cell0 + cc) * (4 * N * N) + (2 * ni) * (2 * N) + 4 * qq;
+            const double j00a = fma(2.0, S00[0], fma(0.5, S11[0] + S22[0], G00[0]));
+            const double j00b = fma(2.0, S00[1], fma(0.5, S11[1] + S22[1], G00[1]));
+            const double j11a = fma(2.0, S11[0], fma(0.5, S00[0] + S22[0], G11[0]));
+            const double j11b = fma(2.0, S11[1], fma(0.5, S00[1] + S22[1], G11[1]));
+            if (!packed) {
+                st_v4_hint(Jr, j00a, X01[0], j00b, X01[1], pol);
+                st_v4_hint(Jr + 2 * N, j10a, j11a, j10b, j11b, pol);
+            } else {  // the lane's blocks (ni, 2qq), (ni, 2qq + 1) that lie in the upper block triangle
+                double *Jb = J_cell + (cell0 + cc) * (4 * pk_blocks<N>());
+                const int j0 = 2 * qq, j1 = j0 + 1;
+                if (j0 >= ni) st_v4_hint(Jb + 4 * pk_block<N>(ni, j0), j00a, X01[0], j10a, j11a, pol);
+                if (j1 >= ni) st_v4_hint(Jb + 4 * pk_block<N>(ni, j1), j00b, X01[1], j10b, j11b, pol);
+            }
+        }
+    }
+}
+
+// residual scatter of a DMMA tile: lane (ni, qq) owns (cell qq, node ni) and, wedge6, (cell 4, node ni)
+template <class E>
+__device__ __forceinline__ void mma_scatter_r(const EvalArgs &a, const int32_t (&gnode)[2], const double (&Rm)[2][2],
+                                              int64_t cell0, int nvalid, int ni, int qq) {
+    constexpr int N = E::N;
+    if (ni >= N) return;
+#pragma unroll
+    for (int k = 0; k < (E::TC > 4 ? 2 : 1); ++k) {
+        const int cc = k ? 4 : qq;
+        if ((k == 0 || qq == 0) && cc < nvalid) {
+            if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode[k], Rm[k][0], Rm[k][1]);
+            if (a.R_cell)
+                *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + cc) * N + ni) * 2) = make_double2(Rm[k][0], Rm[k][1]);
+        }
+    }
+}
+// node ids the lane scatters to (read from the tile's record before its stage is refilled)
+template <class E, class RR>
+__device__ __forceinline__ void mma_gnodes(const int32_t *rconn, int ni, int qq, int32_t (&gnode)[2]) {
+    const int n = ni < E::N ? ni : 0;
+    gnode[0] = rconn[RR::conn(n, qq < E::TC ? qq : 0)];
+    gnode[1] = E::TC > 4 ? rconn[RR::conn(n, 4 < E::TC ? 4 : 0)] : 0;
+}
+
 #ifndef SFO_MMA_JAC_WARPS
 #define SFO_MMA_JAC_WARPS 12
 #endif
-template <int NSTAGE>
+template <class E, int NSTAGE>
 struct MmaSmem {
-    using E = Hex8;
     static constexpr int REC = Rec<E>::BYTES;
     static constexpr int U_OFF = (int)round_up(REC, 16);
     static constexpr int S_OFF = U_OFF + E::TC * E::UPITCH * 16;
     static constexpr int STAGE = (int)round_up(S_OFF + E::TC * E::UPITCH * 8, 128);
     static constexpr int OFF_QS = NSTAGE * STAGE;
-    static constexpr int OFF_BAR = OFF_QS + NQS * E::TC * E::Q * 8;
+    static constexpr int OFF_BAR = OFF_QS + qs_mma_bytes<E>();
     static constexpr int BYTES = OFF_BAR + NSTAGE * 8;
     static_assert(U_OFF == EvalSmem<E, M_JAC, NSTAGE>::U_OFF && S_OFF == EvalSmem<E, M_JAC, NSTAGE>::S_OFF,
                   "gather_store / gather_load share the stored kernel's stage layout");
 };
 
-template <int NSTAGE>
+template <class E, int NSTAGE>
 __global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_mma_kernel(EvalArgs a) {
-    using E = Hex8;
-    constexpr int N = E::N, Q = E::Q, TC = E::TC;
+    constexpr int N = E::N, TC = E::TC;
     using R = Rec<E>;
-    using S = MmaSmem<NSTAGE>;
+    using S = MmaSmem<E, NSTAGE>;
     extern __shared__ __align__(128) char smem[];
     const int64_t vb = blockIdx.x, vg = gridDim.x;
-    const QsMma qs{reinterpret_cast<double *>(smem + S::OFF_QS)};
+    const QsMma<E> qs{reinterpret_cast<double *>(smem + S::OFF_QS)};
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
     const int l = threadIdx.x & 31;
-    const int c = l >> 3, s = l & 7;    // per-QP phase: (cell, qp)
-    const int ni = l >> 2, qq = l & 3;  // DMMA fragments: (node, qp quad)
+    const bool act = l < TC * N;
+    const int c = act ? E::lane_cell(l) : 0, s = act ? E::lane_sub(l) : 0;  // per-QP phase: (cell, qp)
+    const int ni = l >> 2, qq = l & 3;                                      // DMMA fragments: (node, qp quad)
     const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
 
     const uint64_t pol_stream = policy_evict_first();
@@ -1128,16 +1285,8 @@ __global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_mma_kernel(EvalArg
         mbar_wait(&bar[0], 0);
         gather_store<E, M_JAC>(smem, gather_load<E, M_JAC>(smem, a.U, a.surface, have_s, nullptr));
     }
-    // phi_ni at this lane's two QPs (the body-force rows)
     double phi[2];
-    {
-        double x, y, z, w, dx, dy, dz;
-#pragma unroll
-        for (int kc = 0; kc < 2; ++kc) {
-            qp_coords<E>(qq + 4 * kc, x, y, z, w);
-            basis<E>(ni, x, y, z, phi[kc], dx, dy, dz);
-        }
-    }
+    mma_phi<E>(ni, qq, phi);
 
     int it = 0;
     for (int64_t tile = vb; tile < a.ntiles; tile += vg, ++it) {
@@ -1155,7 +1304,7 @@ __global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_mma_kernel(EvalArg
         __syncwarp();  // this tile's gathered U, s are visible
 
         // ---- per-QP phase: lane <-> (cell c, qp s), as in eval_kernel ----
-        {
+        if (act) {
             const int q = s;
             double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
 #pragma unroll
@@ -1178,72 +1327,18 @@ __global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_mma_kernel(EvalArg
         __syncwarp();
 
         // ---- per-node phase on the tensor cores, one cell at a time ----
-        const int32_t gnode = rconn[R::conn(ni, qq)];  // this lane scatters R of (cell qq, node ni)
+        int32_t gnode[2];
+        mma_gnodes<E, R>(rconn, ni, qq, gnode);
         const int64_t ntile = tile + vg;
         const int nst = (it + 1) % NSTAGE;
         Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
-        double Rm0 = 0.0, Rm1 = 0.0;
-#pragma unroll 1
-        for (int cc = 0; cc < TC; ++cc) {
-            if (cc == TC / 2 && ntile < a.ntiles) {  // the next tile's gather, half a tile of latency slack
+        double Rm[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
+        mma_node_phase<E>(a.J_cell, rg, qs, phi, cell0, nvalid, ni, qq, pol_stream, Rm, a.packed != 0, [&]() {
+            if (ntile < a.ntiles) {  // the next tile's gather, half a tile of latency slack
                 mbar_wait(&bar[nst], (uint32_t)(((it + 1) / NSTAGE) & 1));
                 nxt = gather_load<E, M_JAC>(smem + nst * S::STAGE, a.U, a.surface, have_s, nullptr);
             }
-            double S00[2] = {0, 0}, S11[2] = {0, 0}, S22[2] = {0, 0}, X01[2] = {0, 0}, G00[2] = {0, 0},
-                   G11[2] = {0, 0};
-            double r0 = 0.0, r1 = 0.0;
-            const double2 b00 = qs.pair(0, cc, qq), b01 = qs.pair(1, cc, qq), b02 = qs.pair(2, cc, qq);
-            const double2 b11 = qs.pair(3, cc, qq), b12 = qs.pair(4, cc, qq), wv = qs.pair(5, cc, qq);
-            const double2 gv = qs.pair(6, cc, qq), f0 = qs.pair(7, cc, qq), f1 = qs.pair(8, cc, qq);
-#pragma unroll
-            for (int kc = 0; kc < 2; ++kc) {
-                const int q = qq + 4 * kc;
-                const double g0 = rg[gidx<E>(ni, q, 0, cc)];
-                const double g1 = rg[gidx<E>(ni, q, 1, cc)];
-                const double g2 = rg[gidx<E>(ni, q, 2, cc)];
-                const double B00 = kc ? b00.y : b00.x, B01 = kc ? b01.y : b01.x, B02 = kc ? b02.y : b02.x;
-                const double B11 = kc ? b11.y : b11.x, B12 = kc ? b12.y : b12.x;
-                const double w = kc ? wv.y : wv.x, gam = kc ? gv.y : gv.x;
-                const double wf0 = kc ? f0.y : f0.x, wf1 = kc ? f1.y : f1.x;
-                const double h0 = fma(g2, B02, fma(g1, B01, g0 * B00));
-                const double h1 = fma(g2, B12, fma(g1, B11, g0 * B01));
-                r0 = fma(wf0, phi[kc], fma(w, h0, r0));
-                r1 = fma(wf1, phi[kc], fma(w, h1, r1));
-                const double wg0 = w * g0, wg1 = w * g1;
-                dmma884(S00, g0, wg0);
-                dmma884(S11, g1, wg1);
-                dmma884(S22, g2, w * g2);
-                dmma884(X01, g1, 0.5 * wg0);
-                dmma884(X01, g0, wg1);
-                const double gh1 = gam * h1;
-                dmma884(G00, h0, gam * h0);
-                dmma884(G11, h1, gh1);
-                dmma884(X01, h0, gh1);
-            }
-            // residual rows of (cc, ni): sum over the 4 lanes of the node's QP quads
-            r0 += __shfl_xor_sync(0xffffffffu, r0, 1);
-            r1 += __shfl_xor_sync(0xffffffffu, r1, 1);
-            r0 += __shfl_xor_sync(0xffffffffu, r0, 2);
-            r1 += __shfl_xor_sync(0xffffffffu, r1, 2);
-            if (qq == cc) {
-                Rm0 = r0;
-                Rm1 = r1;
-            }
-            // J_10[ni][2qq + e] = J_01[2qq + e][ni]: lane (2qq + e, ni >> 1), element ni & 1
-            const int src0 = 8 * qq + (ni >> 1), src1 = src0 + 4;
-            const double t00 = __shfl_sync(0xffffffffu, X01[0], src0), t01 = __shfl_sync(0xffffffffu, X01[1], src0);
-            const double t10 = __shfl_sync(0xffffffffu, X01[0], src1), t11 = __shfl_sync(0xffffffffu, X01[1], src1);
-            const double j10a = (ni & 1) ? t01 : t00, j10b = (ni & 1) ? t11 : t10;
-            if (cc < nvalid) {
-                double *Jr = a.J_cell + (cell0 + cc) * (4 * N * N) + (2 * ni) * (2 * N) + 4 * qq;
-                const double j00a = fma(2.0, S00[0], fma(0.5, S11[0] + S22[0], G00[0]));
-                const double j00b = fma(2.0, S00[1], fma(0.5, S11[1] + S22[1], G00[1]));
-                const double j11a = fma(2.0, S11[0], fma(0.5, S00[0] + S22[0], G11[0]));
-                const double j11b = fma(2.0, S11[1], fma(0.5, S00[1] + S22[1], G11[1]));
-                st_v4_hint(Jr, j00a, X01[0], j00b, X01[1], pol_stream);
-                st_v4_hint(Jr + 2 * N, j10a, j11a, j10b, j11b, pol_stream);
-            }
-        }
+        });
         __syncwarp();  // every lane is done with this stage's record and per-QP scalars
 
         if (l == 0) {
@@ -1253,10 +1348,7 @@ __global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_mma_kernel(EvalArg
                 bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
             }
         }
-        if (qq < nvalid) {
-            if (a.R) scatter_node(a.rem, a.remtab, a.R, a.peers, gnode, Rm0, Rm1);
-            if (a.R_cell) *reinterpret_cast<double2 *>(a.R_cell + ((cell0 + qq) * N + ni) * 2) = make_double2(Rm0, Rm1);
-        }
+        mma_scatter_r<E>(a, gnode, Rm, cell0, nvalid, ni, qq);
         if (ntile < a.ntiles) gather_store<E, M_JAC>(smem + nst * S::STAGE, nxt);
     }
 }
@@ -1538,6 +1630,132 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_COMPACT_JAC_WARPS
         if (ntile < a.ntiles) gather_store_c<E, MODE>(smem + nst * S::STAGE, nxt);
     }
     if (JAC && l == 0) bulk_wait0();
+}
+
+// ---- G4 with compact stored geometry on the fp64 tensor cores (hex8, wedge6) ----
+// The compact kernel's record ring (A_q = J_q^-T) and register gather, the per-QP phase forming
+// GradBF = A_q grad_xi phi into the per-warp GradBF region (record slot layout), and the DMMA per-node phase
+// of eval_mma_kernel (mma_node_phase: J written straight from the accumulator fragments, no staging). The
+// record stage is refilled right after the per-QP phase (GradBF lives in the per-warp region), so the TMA
+// lead is 1.5 tiles. Shared memory per warp: 2 record stages + GradBF + per-QP scalars (hex8 15.6 KB).
+template <class E>
+struct CompactMmaSmem {
+    using C = CompactSmem<E, M_JAC>;
+    static constexpr int STAGE = C::STAGE;  // RecC + gathered U, s (gather_store_c's layout)
+    static constexpr int OFF_G = 2 * STAGE;
+    static constexpr int OFF_QS = OFF_G + E::Q * 3 * E::SLAB * 8;
+    static constexpr int OFF_BAR = OFF_QS + qs_mma_bytes<E>();
+    static constexpr int BYTES = OFF_BAR + 2 * 8;
+    static_assert(OFF_G % 128 == 0 && OFF_QS % 16 == 0, "alignment");
+};
+
+template <class E>
+__global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_compact_mma_kernel(EvalArgs a) {
+    constexpr int N = E::N, TC = E::TC;
+    using R = RecC<E>;
+    using S = CompactMmaSmem<E>;
+    extern __shared__ __align__(128) char smem[];
+    double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
+    const QsMma<E> qs{reinterpret_cast<double *>(smem + S::OFF_QS)};
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem + S::OFF_BAR);
+    const int64_t vb = blockIdx.x, vg = gridDim.x;
+    const int l = threadIdx.x & 31;
+    const bool act = l < TC * N;
+    const int c = act ? E::lane_cell(l) : 0, s = act ? E::lane_sub(l) : 0;  // per-QP phase: (cell, qp)
+    const int ni = l >> 2, qq = l & 3;                                      // DMMA fragments: (node, qp quad)
+    const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
+
+    const uint64_t pol_stream = policy_evict_first();
+    if (l == 0) {
+        for (int k = 0; k < 2; ++k) mbar_init(&bar[k], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (int k = 0; k < 2; ++k) {
+            const int64_t tile = vb + (int64_t)k * vg;
+            if (tile < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[k], R::BYTES);
+                bulk_g2s(smem + k * S::STAGE, a.recs + tile * (int64_t)R::BYTES, R::BYTES, &bar[k], pol_stream);
+            }
+        }
+    }
+    __syncwarp();
+    if (vb < a.ntiles) {
+        mbar_wait(&bar[0], 0);
+        gather_store_c<E, M_JAC>(smem, gather_load_c<E, M_JAC>(smem, a.U, a.surface, have_s, nullptr));
+    }
+    double xq, yq, zq, wq;  // this lane's QP (per-QP phase)
+    qp_coords<E>(s, xq, yq, zq, wq);
+    double phi[2];
+    mma_phi<E>(ni, qq, phi);
+
+    int it = 0;
+    for (int64_t tile = vb; tile < a.ntiles; tile += vg, ++it) {
+        const int st = it & 1;
+        char *stage = smem + st * S::STAGE;
+        const int32_t *rconn = reinterpret_cast<const int32_t *>(stage + R::CONN_OFF);
+        const double *rkc = reinterpret_cast<const double *>(stage + R::KC_OFF);
+        const double *rwm = reinterpret_cast<const double *>(stage + R::WM_OFF);
+        const double *ra = reinterpret_cast<const double *>(stage + R::A_OFF);
+        const double2 *Us = reinterpret_cast<const double2 *>(stage + S::C::U_OFF);
+        const double *ss = reinterpret_cast<const double *>(stage + S::C::S_OFF);
+        const int64_t cell0 = tile * TC;
+        const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
+
+        __syncwarp();  // this tile's gathered U, s are visible; the previous node phase is done with G and qs
+        int32_t gnode[2];
+        mma_gnodes<E, R>(rconn, ni, qq, gnode);
+
+        // ---- per-QP phase: lane <-> (cell c, qp s); GradBF = A grad_xi phi in registers -> G region ----
+        if (act) {
+            const int q = s;
+            double A[9];
+#pragma unroll
+            for (int k = 0; k < 9; ++k) A[k] = ra[R::a(k, q, c)];
+            double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+#pragma unroll
+            for (int n = 0; n < N; ++n) {
+                double ph, d0, d1, d2;
+                basis<E>(n, xq, yq, zq, ph, d0, d1, d2);
+                const double g0 = fma(A[0], d0, fma(A[1], d1, A[2] * d2));
+                const double g1 = fma(A[3], d0, fma(A[4], d1, A[5] * d2));
+                const double g2 = fma(A[6], d0, fma(A[7], d1, A[8] * d2));
+                rg[gidx<E>(n, q, 0, c)] = g0;
+                rg[gidx<E>(n, q, 1, c)] = g1;
+                rg[gidx<E>(n, q, 2, c)] = g2;
+                const int e = E::uidx(c, n);
+                const double2 uv = Us[e];
+                ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
+                vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
+                if (have_s) {
+                    const double sn = ss[e];
+                    gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
+                }
+            }
+            qp_tail<E, M_JAC>(a, qs, c, q, nvalid, cell0, have_s, rkc[c], rwm[R::wm(q, c)], ux, uy, uz, vx, vy, vz,
+                              gs0, gs1);
+        }
+        __syncwarp();  // the stage (record, U, s) is consumed: refill it with the record two tiles ahead
+        if (l == 0) {
+            const int64_t nt = tile + 2 * vg;
+            if (nt < a.ntiles) {
+                mbar_arrive_expect_tx(&bar[st], R::BYTES);
+                bulk_g2s(stage, a.recs + nt * (int64_t)R::BYTES, R::BYTES, &bar[st], pol_stream);
+            }
+        }
+
+        // ---- per-node phase on the tensor cores (+ gather of the next tile before cell TC / 2) ----
+        const int64_t ntile = tile + vg;
+        const int nst = (it + 1) & 1;
+        Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
+        double Rm[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
+        mma_node_phase<E>(a.J_cell, rg, qs, phi, cell0, nvalid, ni, qq, pol_stream, Rm, a.packed != 0, [&]() {
+            if (ntile < a.ntiles) {
+                mbar_wait(&bar[nst], (uint32_t)(((it + 1) >> 1) & 1));
+                nxt = gather_load_c<E, M_JAC>(smem + nst * S::STAGE, a.U, a.surface, have_s, nullptr);
+            }
+        });
+        mma_scatter_r<E>(a, gnode, Rm, cell0, nvalid, ni, qq);
+        if (ntile < a.ntiles) gather_store_c<E, M_JAC>(smem + nst * S::STAGE, nxt);
+    }
 }
 
 // ---- G3/G4 with on-the-fly geometry ------------------------------------------
@@ -2061,12 +2279,22 @@ constexpr int CSR_GATHER_MAXDEG = 64;   // neighbour nodes per node (else the at
 constexpr int CSR_GATHER_WARPS = 8;
 constexpr int CSR_GATHER_NPW = 2;       // nodes per warp
 // ACC = false: the rows are overwritten (vals = assembled J; no prior zeroing, no read of vals).
-template <int N, bool ACC = true>
+// row pair (2 i + a, columns 2 j, 2 j + 1) of cell `cell`'s element matrix: full [C][2N][2N] (streamed
+// once) or symmetric block-packed (block (i, j) or the transpose of block (j, i); each off-diagonal
+// block is read by two node warps, so the packed reads keep the default L2 policy)
+template <int N, bool PACKED>
+__device__ __forceinline__ double2 jrow2(const double *__restrict__ Jc, int64_t cell, int i, int a, int j) {
+    if (!PACKED) return __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * 2 * N + 2 * i + a) * 2 * N) + j);
+    const double *b = Jc + cell * (4 * pk_blocks<N>());
+    if (j >= i) return __ldg(reinterpret_cast<const double2 *>(b + 4 * pk_block<N>(i, j) + 2 * a));
+    const double *t = b + 4 * pk_block<N>(j, i);
+    return make_double2(__ldg(t + a), __ldg(t + 2 + a));
+}
+template <int N, bool ACC = true, bool PACKED = false>
 __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
     csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
                       const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
                       const uint64_t *__restrict__ slots, double *__restrict__ vals) {
-    constexpr int ND = 2 * N;
     constexpr int LC = 2 * N;            // lanes per cell: each loads one (j, b = 0..1) pair of one row
     constexpr int CPI = 32 / LC;         // cells per load instruction (2 for hex8 and wedge6)
     constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW, NI = BATCH / CPI;
@@ -2116,8 +2344,7 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
             const bool live = lane_ok && e < cnt[n];
             const int64_t cell = ci / N;
             const int i = ci - (int)(cell * N);
-            x[n][t] = live ? __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j)
-                           : make_double2(0.0, 0.0);
+            x[n][t] = live ? jrow2<N, PACKED>(Jc, cell, i, a, j) : make_double2(0.0, 0.0);
             sl[n][t] = live ? (int)__ldg(sb + 8 * (int64_t)ci + j) : -1;
         }
     __syncwarp();
@@ -2145,7 +2372,7 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
             const int i = ci - (int)(cell * N);
             if (l < LC) {
                 const int s = (int)__ldg(sb + 8 * (int64_t)ci + j);
-                const double2 y = __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j);
+                const double2 y = jrow2<N, PACKED>(Jc, cell, i, a, j);
                 buf[w][n][a * half + 2 * s] += y.x;
                 buf[w][n][a * half + 2 * s + 1] += y.y;
             }

@@ -57,7 +57,7 @@ EXPORTS = [
     "stokesfo_set_remote", "stokesfo_set_remote_jvp", "stokesfo_ipc_get_handle", "stokesfo_ipc_open_handle", "stokesfo_ipc_close",
     "stokesfo_newton_work_size", "stokesfo_newton_solve", "stokesfo_lateral_pressure",
     "stokesfo_mesh_lateral_faces", "stokesfo_set_lateral", "stokesfo_csr_slots_size", "stokesfo_csr_slots", "stokesfo_jacobian_csr",
-    "stokesfo_jacobian_diag", "stokesfo_assemble_csr",
+    "stokesfo_jacobian_diag", "stokesfo_assemble_csr", "stokesfo_jacobian_packed", "stokesfo_assemble_csr_packed",
 ]
 
 
@@ -93,6 +93,9 @@ def _lib():
             L.stokesfo_jacobian_diag.argtypes = [P, P, P, P]
         if hasattr(L, "stokesfo_assemble_csr"):
             L.stokesfo_assemble_csr.argtypes = [P, P, P, ctypes.c_int]
+        if hasattr(L, "stokesfo_jacobian_packed"):
+            L.stokesfo_jacobian_packed.argtypes = [P, P, P, P, P]
+            L.stokesfo_assemble_csr_packed.argtypes = [P, P, P, ctypes.c_int]
         if hasattr(L, "stokesfo_basal_friction"):
             L.stokesfo_basal_friction.argtypes = [P, P, I64, P, P, P, P]
         if hasattr(L, "stokesfo_lateral_pressure"):
@@ -362,6 +365,25 @@ class StokesFO:
         pull assembly, after csr_slots); accumulate=False overwrites every entry."""
         _check(_lib().stokesfo_assemble_csr(self._h, _ptr(J_cell), _ptr(csr_vals), 1 if accumulate else 0),
                "assemble_csr")
+
+    @property
+    def packed_blocks(self):
+        """N(N+1)/2: upper 2 x 2 node blocks per cell of the symmetric block-packed element matrix."""
+        return self.N * (self.N + 1) // 2
+
+    def jacobian_packed(self, U, Jp, R_cell=None, R=None):
+        """Element Jacobians in symmetric block-packed form Jp [C][N(N+1)/2][2][2] (stokesfo_jacobian_packed)."""
+        import torch
+        _dev(U, torch.float64, (self.num_nodes, 2), "U")
+        _dev(Jp, torch.float64, (self.num_cells, self.packed_blocks, 2, 2), "Jp")
+        _dev(R_cell, torch.float64, (self.num_cells, self.N, 2), "R_cell")
+        _dev(R, torch.float64, (self.num_nodes, 2), "R")
+        _check(_lib().stokesfo_jacobian_packed(self._h, _ptr(U), _ptr(Jp), _ptr(R_cell), _ptr(R)), "jacobian_packed")
+
+    def assemble_csr_packed(self, Jp, csr_vals, accumulate=False):
+        """csr_vals (+)= the global matrix assembled from packed element matrices (stokesfo_assemble_csr_packed)."""
+        _check(_lib().stokesfo_assemble_csr_packed(self._h, _ptr(Jp), _ptr(csr_vals), 1 if accumulate else 0),
+               "assemble_csr_packed")
 
     def scatter_assemble(self, R_cell=None, R=None, J_cell=None, csr_vals=None):
         _check(_lib().stokesfo_scatter_assemble(self._h, _ptr(R_cell), _ptr(R), _ptr(J_cell), _ptr(csr_vals)),

@@ -445,6 +445,77 @@ def test_csr_slots_and_fused_assembly(torch, elem, geometry):
     _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
 
 
+def _unpack_blocks(Jp, N):
+    """Full [C][2N][2N] element matrices from the symmetric block-packed form (header: block (i, j >= i) at
+    index i N - i (i - 1) / 2 + (j - i), entries [a][b] = J[(i,a),(j,b)]; block (j, i) = block (i, j)^T)."""
+    C = Jp.shape[0]
+    J = np.empty((C, 2 * N, 2 * N))
+    k = 0
+    for i in range(N):
+        for j in range(i, N):
+            J[:, 2 * i:2 * i + 2, 2 * j:2 * j + 2] = Jp[:, k]
+            J[:, 2 * j:2 * j + 2, 2 * i:2 * i + 2] = np.transpose(Jp[:, k], (0, 2, 1))
+            k += 1
+    return J
+
+
+@pytest.mark.parametrize("geometry", ["stored", "compact"])
+@pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 0), ("wedge6", 11)])
+def test_jacobian_packed_and_assembly(torch, elem, drop, geometry):
+    """NEXT-2 symmetric block-packed element matrices (stokesfo_jacobian_packed): unpacked, they match the
+    oracle's dual-number J at 1e-12 (the oracle's J is symmetric to rounding: a transposed operand or a
+    wrong block index in the packing fails this), R_cell / R as the full path; no write past the last
+    cell; the pull assembly from the packed form (stokesfo_assemble_csr_packed) matches the oracle's CSR
+    scatter, overwrites every entry and is bitwise reproducible."""
+    ctx, orc = _setup(torch, elem, n=6, L=3, drop=drop, geometry=geometry)
+    C, N = ctx.num_cells, ctx.N
+    NB = N * (N + 1) // 2
+    conn = orc["conn"]
+    ref = O.evaluate(orc["e"], conn, orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"], mode="jac")
+    U = _t(torch, orc["U"])
+    buf = torch.full(((C + 2) * NB * 4,), 7.0, dtype=torch.float64, device="cuda")
+    Jp = buf[:C * NB * 4].view(C, NB, 2, 2)
+    Rc = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
+    R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+    ctx.jacobian_packed(U, Jp, R_cell=Rc, R=R)
+    ctx.sync()
+    assert (buf[C * NB * 4:] == 7.0).all()
+    Jpn = Jp.cpu().numpy()
+    assert np.isfinite(Jpn).all()
+    assert _cell_rel(_unpack_blocks(Jpn, N), ref["J_cell"]) <= TOL
+    assert _cell_rel(Rc.cpu().numpy(), ref["R_cell"]) <= TOL
+    _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
+    # pull assembly from the packed form
+    rowptr, colidx = ctx.csr_pattern()
+    rp2, ci2 = O.csr_pattern(conn, ctx.num_nodes)
+    ctx.csr_slots()
+    v2, miss = O.scatter_csr(orc["e"], conn, ref["J_cell"], rp2, ci2)
+    cell_scale = np.abs(ref["J_cell"]).reshape(C, -1).max(1)[:, None, None] * np.ones_like(ref["J_cell"])
+    a2, _ = O.scatter_csr(orc["e"], conn, cell_scale, rp2, ci2)
+    assert miss == 0
+    vals = torch.full((colidx.numel(),), float("nan"), dtype=torch.float64, device="cuda")
+    ctx.assemble_csr_packed(Jp, vals, accumulate=False)
+    ctx.sync()
+    assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2).all()
+    vals2 = torch.zeros_like(vals)
+    ctx.assemble_csr_packed(Jp, vals2, accumulate=True)
+    ctx.sync()
+    assert torch.equal(vals, vals2)
+
+
+def test_jacobian_packed_unsupported(torch, monkeypatch):
+    """The packed form comes from the tensor-core kernels only: on-the-fly geometry, or STOKESFO_JAC_MMA=0
+    at create, returns EUNSUPPORTED (a loud error, no silent fallback)."""
+    from paper_conf_sc_antepara0cw24_b200.stokesfo import StokesFOError
+    for geometry, mma in (("on_the_fly", "1"), ("stored", "0")):
+        monkeypatch.setenv("STOKESFO_JAC_MMA", mma)
+        ctx, orc = _setup(torch, "hex8", n=4, L=2, geometry=geometry)
+        C, N = ctx.num_cells, ctx.N
+        Jp = torch.empty((C, N * (N + 1) // 2, 2, 2), dtype=torch.float64, device="cuda")
+        with pytest.raises(StokesFOError, match="unsupported|EUNSUPPORTED"):
+            ctx.jacobian_packed(_t(torch, orc["U"]), Jp)
+
+
 @pytest.mark.parametrize("drop", [0, 11])
 def test_wedge_tensor_map_store(torch, drop, monkeypatch):
     """wedge6 J tiles leave the kernel as ONE 2-D TMA tensor store of the padded
@@ -452,6 +523,7 @@ def test_wedge_tensor_map_store(torch, drop, monkeypatch):
     result must be bitwise the per-cell bulk-copy path's (STOKESFO_JMAP=0), and
     neither the padding columns nor the box rows past the last cell may land in
     memory: a sentinel after J[C-1] (ragged last tile for drop=11) stays intact."""
+    monkeypatch.setenv("STOKESFO_JAC_MMA", "0")  # the vector kernel (the DMMA kernel stores J directly)
     ctx, orc = _setup(torch, "wedge6", drop=drop)
     C, N = ctx.num_cells, ctx.N
     U = _t(torch, orc["U"])
@@ -468,6 +540,42 @@ def test_wedge_tensor_map_store(torch, drop, monkeypatch):
     ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
                      mode="jac")
     assert _cell_rel(a[:C], ref["J_cell"]) <= TOL
+
+
+@pytest.mark.parametrize("geometry", ["stored", "compact"])
+@pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 0), ("wedge6", 11)])
+def test_jacobian_tensor_core_vs_vector(torch, elem, drop, geometry, monkeypatch):
+    """The element Jacobians on the fp64 tensor cores (eval_mma_kernel / eval_compact_mma_kernel; default for
+    hex8, STOKESFO_JAC_MMA=1 forces them for wedge6 too) and on the vector pipes (STOKESFO_JAC_MMA=0) both
+    match the oracle at 1e-12; a J_cell that is only
+    16-B aligned (the ABI's requirement) takes the vector kernel on a DMMA context; the DMMA kernels write
+    no byte past the last cell (ragged last tile: sentinel cells after J[C-1] stay intact)."""
+    outs = {}
+    for mma in ("1", "0"):
+        monkeypatch.setenv("STOKESFO_JAC_MMA", mma)
+        ctx, orc = _setup(torch, elem, drop=drop, geometry=geometry)
+        C, N = ctx.num_cells, ctx.N
+        U = _t(torch, orc["U"])
+        buf = torch.full(((C + 3) * 4 * N * N + 2,), 7.0, dtype=torch.float64, device="cuda")
+        for off in (0, 2):  # 32-B aligned, then 16-B aligned only
+            J = buf[off:off + C * 4 * N * N].view(C, 2 * N, 2 * N)
+            Rc = torch.empty((C, N, 2), dtype=torch.float64, device="cuda")
+            R = torch.zeros((ctx.num_nodes, 2), dtype=torch.float64, device="cuda")
+            ctx.jacobian(U, J, R_cell=Rc, R=R)
+            ctx.sync()
+            b = buf.cpu().numpy()
+            assert (b[off + C * 4 * N * N:] == 7.0).all()
+            outs[(mma, off)] = (J.cpu().numpy().copy(), Rc.cpu().numpy(), R.cpu().numpy())
+            buf.fill_(7.0)
+    ref = O.evaluate(orc["e"], orc["conn"], orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"],
+                     mode="jac")
+    for key, (J, Rc, R) in outs.items():
+        assert np.isfinite(J).all(), key
+        assert _cell_rel(J, ref["J_cell"]) <= TOL, key
+        assert _cell_rel(Rc, ref["R_cell"]) <= TOL, key
+        _assembled_check(R, orc, ref["R_cell"])
+    # the misaligned call on the DMMA context ran the vector kernel: bitwise the JAC_MMA=0 result
+    assert np.array_equal(outs[("1", 2)][0], outs[("0", 0)][0])
 
 
 @pytest.mark.parametrize("geometry", GEOMS)
