@@ -221,8 +221,10 @@ int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_val
 int stokesfo_jacobian_packed(stokesfo_ctx *c, const double *U, double *Jp, double *R_cell, double *R);
 
 /* stokesfo_assemble_csr from the packed form: row (i, a) of cell c is block
- * (i, j) for j >= i and the transpose of block (j, i) for j < i.  Same
- * requirements, ordering and accumulate semantics as stokesfo_assemble_csr. */
+ * (i, j) for j >= i and the transpose of block (j, i) for j < i (one 32-B
+ * load per block).  Jp dev [C][N(N+1)/2][2][2], 32-B aligned (else EINVAL);
+ * otherwise the same requirements, ordering and accumulate semantics as
+ * stokesfo_assemble_csr. */
 int stokesfo_assemble_csr_packed(stokesfo_ctx *c, const double *Jp, double *csr_vals, int accumulate);
 
 /* CSR pattern over dofs (rows = 2*num_nodes; columns of a row = sorted dofs of

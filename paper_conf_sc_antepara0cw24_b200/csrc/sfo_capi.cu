@@ -754,13 +754,24 @@ static int assemble_csr_impl(stokesfo_ctx *c, const double *J_cell, double *csr_
     const int64_t per_block = (int64_t)CSR_GATHER_WARPS * CSR_GATHER_NPW;
     const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
     const int bt = 32 * CSR_GATHER_WARPS;
-    if (c->N == 8) {
-        if (accumulate) csr_gather_kernel<8, true, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
-        else csr_gather_kernel<8, false, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+#define PULL(K, NN_, ACC_) K<NN_, ACC_><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals)
+    if (PACKED) {
+        if (!aligned(J_cell, 32)) return STOKESFO_EINVAL;
+        if (c->N == 8) {
+            if (accumulate) PULL(csr_gather_packed_kernel, 8, true);
+            else PULL(csr_gather_packed_kernel, 8, false);
+        } else {
+            if (accumulate) PULL(csr_gather_packed_kernel, 6, true);
+            else PULL(csr_gather_packed_kernel, 6, false);
+        }
+    } else if (c->N == 8) {
+        if (accumulate) PULL(csr_gather_kernel, 8, true);
+        else PULL(csr_gather_kernel, 8, false);
     } else {
-        if (accumulate) csr_gather_kernel<6, true, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
-        else csr_gather_kernel<6, false, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals);
+        if (accumulate) PULL(csr_gather_kernel, 6, true);
+        else PULL(csr_gather_kernel, 6, false);
     }
+#undef PULL
     return cuda_status();
 }
 

@@ -1075,8 +1075,13 @@ __global__ void __launch_bounds__(32 * warps_per_cta<E, MODE>(), (warps_per_sm<E
 #ifndef SFO_MMA_SPLIT
 #define SFO_MMA_SPLIT 1
 #endif
-#ifndef SFO_MMA_UNROLL
-#define SFO_MMA_UNROLL 1
+// cells of a tile unrolled in the DMMA node phase: stored kernel 1 (2: -7% same box, it is at its HBM bound
+// and the extra registers cost), compact kernel 2 (+3%, latency-bound; profiles/r2_samebox_mma_unroll.txt)
+#ifndef SFO_MMA_UNROLL_STORED
+#define SFO_MMA_UNROLL_STORED 1
+#endif
+#ifndef SFO_MMA_UNROLL_COMPACT
+#define SFO_MMA_UNROLL_COMPACT 2
 #endif
 __device__ __forceinline__ void dmma884(double (&d)[2], double a, double b) {
     asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
@@ -1123,18 +1128,14 @@ __device__ __forceinline__ void mma_phi(int ni, int qq, double (&phi)[2]) {
 // the QsMma layout; lane (ni, qq) returns the residual rows of (cell qq, node ni) in Rm[0] (and, wedge6's
 // fifth cell, of (cell 4, node ni) in Rm[1] on the lanes qq == 0) and writes the element Jacobians of the
 // tile's valid cells straight to J_cell.  pf() is called once, before cell TC / 2.
-template <class E, class PF>
+template <class E, int UNROLL, class PF>
 __device__ __forceinline__ void mma_node_phase(double *__restrict__ J_cell, const double *rg, const QsMma<E> &qs,
                                                const double (&phi)[2], int64_t cell0, int nvalid, int ni, int qq,
                                                uint64_t pol, double (&Rm)[2][2], bool packed, PF pf) {
     constexpr int N = E::N, Q = E::Q, TC = E::TC;
     static_assert(N <= 8 && Q <= 8 && Q > 4 && TC <= 5, "two k steps of 4 QPs, 8 x 8 node blocks");
     const bool node_ok = N == 8 || ni < N;
-#if SFO_MMA_UNROLL == 2
-#pragma unroll 2
-#else
-#pragma unroll 1
-#endif
+#pragma unroll(UNROLL)
     for (int cc = 0; cc < TC; ++cc) {
         if (cc == TC / 2) pf();
         double S00[2] = {0, 0}, S11[2] = {0, 0}, S22[2] = {0, 0}, X01[2] = {0, 0}, G00[2] = {0, 0},
@@ -1333,7 +1334,7 @@ __global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_mma_kernel(EvalArg
         const int nst = (it + 1) % NSTAGE;
         Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
         double Rm[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
-        mma_node_phase<E>(a.J_cell, rg, qs, phi, cell0, nvalid, ni, qq, pol_stream, Rm, a.packed != 0, [&]() {
+        mma_node_phase<E, SFO_MMA_UNROLL_STORED>(a.J_cell, rg, qs, phi, cell0, nvalid, ni, qq, pol_stream, Rm, a.packed != 0, [&]() {
             if (ntile < a.ntiles) {  // the next tile's gather, half a tile of latency slack
                 mbar_wait(&bar[nst], (uint32_t)(((it + 1) / NSTAGE) & 1));
                 nxt = gather_load<E, M_JAC>(smem + nst * S::STAGE, a.U, a.surface, have_s, nullptr);
@@ -1747,7 +1748,7 @@ __global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_compact_mma_kernel
         const int nst = (it + 1) & 1;
         Gathered nxt{make_double2(0.0, 0.0), 0.0, make_double2(0.0, 0.0)};
         double Rm[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
-        mma_node_phase<E>(a.J_cell, rg, qs, phi, cell0, nvalid, ni, qq, pol_stream, Rm, a.packed != 0, [&]() {
+        mma_node_phase<E, SFO_MMA_UNROLL_COMPACT>(a.J_cell, rg, qs, phi, cell0, nvalid, ni, qq, pol_stream, Rm, a.packed != 0, [&]() {
             if (ntile < a.ntiles) {
                 mbar_wait(&bar[nst], (uint32_t)(((it + 1) >> 1) & 1));
                 nxt = gather_load_c<E, M_JAC>(smem + nst * S::STAGE, a.U, a.surface, have_s, nullptr);
@@ -2279,22 +2280,12 @@ constexpr int CSR_GATHER_MAXDEG = 64;   // neighbour nodes per node (else the at
 constexpr int CSR_GATHER_WARPS = 8;
 constexpr int CSR_GATHER_NPW = 2;       // nodes per warp
 // ACC = false: the rows are overwritten (vals = assembled J; no prior zeroing, no read of vals).
-// row pair (2 i + a, columns 2 j, 2 j + 1) of cell `cell`'s element matrix: full [C][2N][2N] (streamed
-// once) or symmetric block-packed (block (i, j) or the transpose of block (j, i); each off-diagonal
-// block is read by two node warps, so the packed reads keep the default L2 policy)
-template <int N, bool PACKED>
-__device__ __forceinline__ double2 jrow2(const double *__restrict__ Jc, int64_t cell, int i, int a, int j) {
-    if (!PACKED) return __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * 2 * N + 2 * i + a) * 2 * N) + j);
-    const double *b = Jc + cell * (4 * pk_blocks<N>());
-    if (j >= i) return __ldg(reinterpret_cast<const double2 *>(b + 4 * pk_block<N>(i, j) + 2 * a));
-    const double *t = b + 4 * pk_block<N>(j, i);
-    return make_double2(__ldg(t + a), __ldg(t + 2 + a));
-}
-template <int N, bool ACC = true, bool PACKED = false>
+template <int N, bool ACC = true>
 __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
     csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
                       const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
                       const uint64_t *__restrict__ slots, double *__restrict__ vals) {
+    constexpr int ND = 2 * N;
     constexpr int LC = 2 * N;            // lanes per cell: each loads one (j, b = 0..1) pair of one row
     constexpr int CPI = 32 / LC;         // cells per load instruction (2 for hex8 and wedge6)
     constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW, NI = BATCH / CPI;
@@ -2344,7 +2335,8 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
             const bool live = lane_ok && e < cnt[n];
             const int64_t cell = ci / N;
             const int i = ci - (int)(cell * N);
-            x[n][t] = live ? jrow2<N, PACKED>(Jc, cell, i, a, j) : make_double2(0.0, 0.0);
+            x[n][t] = live ? __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j)
+                           : make_double2(0.0, 0.0);
             sl[n][t] = live ? (int)__ldg(sb + 8 * (int64_t)ci + j) : -1;
         }
     __syncwarp();
@@ -2372,7 +2364,7 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
             const int i = ci - (int)(cell * N);
             if (l < LC) {
                 const int s = (int)__ldg(sb + 8 * (int64_t)ci + j);
-                const double2 y = jrow2<N, PACKED>(Jc, cell, i, a, j);
+                const double2 y = __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j);
                 buf[w][n][a * half + 2 * s] += y.x;
                 buf[w][n][a * half + 2 * s + 1] += y.y;
             }
@@ -2392,6 +2384,141 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
                 *o = c;
             } else {
                 __stcs(o, b);  // streamed: the assembled matrix is not re-read by this kernel
+            }
+        }
+}
+
+// Pull assembly from the symmetric block-packed element matrices: lane <-> (incident cell u, column node j)
+// loads the whole 2 x 2 block (i, j) -- or block (j, i), transposed in registers -- with one 256-bit load
+// (a full 32-B sector; the row-pair mapping of csr_gather_kernel needs two scalar loads for every transposed
+// block: C4 5.46 vs 5.04 ms, ncu r2g), and adds both of its rows to the node's two CSR rows in shared memory.
+__device__ __forceinline__ double4 ld_v4_nc(const double *p) {
+    double4 v;
+    asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w) : "l"(p));
+    return v;
+}
+template <int N, bool ACC = true>
+__global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
+    csr_gather_packed_kernel(int64_t nnodes, const double *__restrict__ Jp, const int64_t *__restrict__ rowptr,
+                             const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
+                             const uint64_t *__restrict__ slots, double *__restrict__ vals) {
+    constexpr int CPI = 32 / N;  // cells per load instruction (hex8 4, wedge6 5)
+    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW, NI = (BATCH + CPI - 1) / CPI;
+    constexpr int NB = pk_blocks<N>();
+    __shared__ __align__(16) double buf[CSR_GATHER_WARPS][NPW][4 * CSR_GATHER_MAXDEG];
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    const int64_t v0 = (blockIdx.x * (int64_t)CSR_GATHER_WARPS + w) * NPW;
+    if (v0 >= nnodes) return;  // uniform per warp
+    int64_t r0[NPW], k0[NPW];
+    int len[NPW], cnt[NPW];
+#pragma unroll
+    for (int n = 0; n < NPW; ++n) {
+        const bool ok = v0 + n < nnodes;
+        const int64_t v = ok ? v0 + n : v0;
+        r0[n] = __ldg(rowptr + 2 * v);
+        len[n] = ok ? (int)(__ldg(rowptr + 2 * v + 2) - r0[n]) : 0;  // both rows: 4 deg entries
+        k0[n] = __ldg(inc_ptr + v);
+        cnt[n] = ok ? (int)(__ldg(inc_ptr + v + 1) - k0[n]) : 0;
+    }
+    if (ACC) {
+#pragma unroll
+        for (int n = 0; n < NPW; ++n)
+            for (int p = 16 * l; p < len[n]; p += 16 * 32)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(vals + r0[n] + p));
+    }
+    const int ln = l / LPN, lt = l % LPN;
+    int32_t my = 0;
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+        if (ln == n && lt < cnt[n] && lt < BATCH) my = __ldg(inc + k0[n] + lt);
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+        for (int p = 2 * l; p < len[n]; p += 64) *reinterpret_cast<double2 *>(&buf[w][n][p]) = make_double2(0.0, 0.0);
+    // lane l <-> (cell u = l / N of the group, column node j = l % N)
+    const int u = l / N, j = l % N;
+    const bool lane_ok = l < CPI * N;
+    double2 x0[NPW][NI], x1[NPW][NI];  // rows (i, 0) and (i, 1), columns (j, 0..1)
+    int sl[NPW][NI];
+    const uint8_t *sb = reinterpret_cast<const uint8_t *>(slots);
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+#pragma unroll
+        for (int t = 0; t < NI; ++t) {
+            const int e = CPI * t + u;  // incidence entry of this lane
+            const bool live = lane_ok && e < BATCH && e < cnt[n];
+            const int32_t ci = __shfl_sync(0xffffffffu, my, n * LPN + (e < BATCH ? e : 0));
+            const int64_t cell = ci / N;
+            const int i = ci - (int)(cell * N);
+            x0[n][t] = x1[n][t] = make_double2(0.0, 0.0);
+            sl[n][t] = -1;
+            if (live) {
+                const double *b = Jp + cell * (4 * NB);
+                if (j >= i) {
+                    const double4 q = ld_v4_nc(b + 4 * pk_block<N>(i, j));
+                    x0[n][t] = make_double2(q.x, q.y);
+                    x1[n][t] = make_double2(q.z, q.w);
+                } else {  // block (j, i): entries [c][d] = J[(j,c),(i,d)], so J[(i,a),(j,b)] = [b][a]
+                    const double4 q = ld_v4_nc(b + 4 * pk_block<N>(j, i));
+                    x0[n][t] = make_double2(q.x, q.z);
+                    x1[n][t] = make_double2(q.y, q.w);
+                }
+                sl[n][t] = (int)__ldg(sb + 8 * (int64_t)ci + j);
+            }
+        }
+    __syncwarp();
+#pragma unroll
+    for (int n = 0; n < NPW; ++n) {
+        const int half = len[n] >> 1;
+        // the CPI cells of a load group may hit the same entries: add them in turn
+#pragma unroll
+        for (int t = 0; t < NI; ++t)
+#pragma unroll
+            for (int uu = 0; uu < CPI; ++uu) {
+                if (u == uu && sl[n][t] >= 0) {
+                    double2 *p0 = reinterpret_cast<double2 *>(&buf[w][n][2 * sl[n][t]]);
+                    double2 *p1 = reinterpret_cast<double2 *>(&buf[w][n][half + 2 * sl[n][t]]);
+                    double2 b0 = *p0, b1 = *p1;
+                    b0.x += x0[n][t].x;
+                    b0.y += x0[n][t].y;
+                    b1.x += x1[n][t].x;
+                    b1.y += x1[n][t].y;
+                    *p0 = b0;
+                    *p1 = b1;
+                }
+                __syncwarp();
+            }
+        // rare: more than BATCH incident cells (not on extruded hex8 / wedge6 meshes)
+        for (int64_t k = k0[n] + BATCH; k < k0[n] + cnt[n]; ++k) {
+            const int32_t ci = __ldg(inc + k);
+            const int64_t cell = ci / N;
+            const int i = ci - (int)(cell * N);
+            if (l < N) {
+                const int s = (int)__ldg(sb + 8 * (int64_t)ci + j);
+                const double *b = Jp + cell * (4 * NB);
+                const double4 q = ld_v4_nc(b + 4 * (j >= i ? pk_block<N>(i, j) : pk_block<N>(j, i)));
+                const double2 y0 = j >= i ? make_double2(q.x, q.y) : make_double2(q.x, q.z);
+                const double2 y1 = j >= i ? make_double2(q.z, q.w) : make_double2(q.y, q.w);
+                buf[w][n][2 * s] += y0.x;
+                buf[w][n][2 * s + 1] += y0.y;
+                buf[w][n][half + 2 * s] += y1.x;
+                buf[w][n][half + 2 * s + 1] += y1.y;
+            }
+            __syncwarp();
+        }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int n = 0; n < NPW; ++n)
+        for (int p = 2 * l; p < len[n]; p += 64) {
+            double2 *o = reinterpret_cast<double2 *>(vals + r0[n] + p);
+            const double2 b = *reinterpret_cast<const double2 *>(&buf[w][n][p]);
+            if (ACC) {
+                double2 c = *o;
+                c.x += b.x;
+                c.y += b.y;
+                *o = c;
+            } else {
+                __stcs(o, b);
             }
         }
 }

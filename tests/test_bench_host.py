@@ -111,3 +111,21 @@ def test_gpus_n_relaunch_refuses_without_enough_gpus(monkeypatch, capsys):
     monkeypatch.setattr("sys.argv", ["bench.py", "--gpus", "2", "--no-cpu-baseline"])
     assert bench.main() == 2
     assert "WORLD_SIZE = 3" in capsys.readouterr().err
+
+
+def test_global_fill_byte_model_packed(monkeypatch):
+    """--op jac_global byte model (DESIGN §6 NEXT-2): the element matrices are written once and read once by
+    the pull assembly; in the symmetric block-packed form that is N(N+1)/2 blocks of 4 doubles per cell instead
+    of (2N)^2 doubles (hex8 1,152 vs 2,048 B; wedge6 672 vs 1,152 B), everything else unchanged."""
+    for elem, N in (("hex8", 8), ("wedge6", 6)):
+        full = bench.bytes_per_launch(elem, 1000, 900, "stored", "jac_global", 5000)
+        packed = bench.bytes_per_launch(elem, 1000, 900, "stored", "jac_global", 5000, packed=True)
+        assert full - packed == 1000 * 2 * 8 * ((2 * N) ** 2 - 4 * N * (N + 1) // 2)
+    # which kernels a line names: tensor cores for hex8 by default, packed global fill on them too
+    monkeypatch.delenv("STOKESFO_JAC_MMA", raising=False)
+    assert bench.jac_mma("hex8", "stored") and not bench.jac_mma("wedge6", "stored")
+    assert bench.jac_mma("wedge6", "compact", packed=True) and not bench.jac_mma("hex8", "on_the_fly")
+    assert bench.kernel_name("hex8", "compact", "jacobian").startswith("eval_compact_mma_kernel<Hex8>")
+    monkeypatch.setenv("STOKESFO_JAC_MMA", "0")
+    assert not bench.jac_mma("hex8", "stored", packed=True)
+    assert bench.kernel_name("hex8", "stored", "jacobian").startswith("eval_kernel<Hex8,M_JAC>")
