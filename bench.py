@@ -331,7 +331,7 @@ def main():
     ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--geometry", default="stored", choices=["stored", "on_the_fly", "compact"])
-    ap.add_argument("--global-format", default="packed", choices=["packed", "full"],
+    ap.add_argument("--global-format", default="full", choices=["packed", "full"],
                     help="--op jac_global: element matrices in symmetric block-packed form (tensor-core kernels) "
                          "or full [C][2N][2N]")
     ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jvp_y", "jac_csr", "jac_global"],

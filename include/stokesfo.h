@@ -221,10 +221,9 @@ int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_val
 int stokesfo_jacobian_packed(stokesfo_ctx *c, const double *U, double *Jp, double *R_cell, double *R);
 
 /* stokesfo_assemble_csr from the packed form: row (i, a) of cell c is block
- * (i, j) for j >= i and the transpose of block (j, i) for j < i (one 32-B
- * load per block).  Jp dev [C][N(N+1)/2][2][2], 32-B aligned (else EINVAL);
- * otherwise the same requirements, ordering and accumulate semantics as
- * stokesfo_assemble_csr. */
+ * (i, j) for j >= i and the transpose of block (j, i) for j < i.  Jp dev
+ * [C][N(N+1)/2][2][2]; otherwise the same requirements, ordering and
+ * accumulate semantics as stokesfo_assemble_csr. */
 int stokesfo_assemble_csr_packed(stokesfo_ctx *c, const double *Jp, double *csr_vals, int accumulate);
 
 /* CSR pattern over dofs (rows = 2*num_nodes; columns of a row = sorted dofs of
@@ -240,7 +239,10 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
  * csr_vals[rowptr[2 conn[c][i] + a] + 2 slot + b].  Requires an earlier
  * stokesfo_csr_pattern fill (rowptr 16-B aligned); computed on the device once
  * (binary searches in colidx) into caller-owned slots: dev uint64 [C][N]
- * (stokesfo_csr_slots_size bytes, 16-B aligned, must stay valid).  Attaches
+ * followed by the node -> cell incidence and a 128-B record per node for the
+ * pull assembly (row base, lengths, first 8 incident cells and their slot
+ * rows: one coalesced load per node) -- stokesfo_csr_slots_size bytes in all,
+ * 16-B aligned, must stay valid.  Attaches
  * the table to the ctx: stokesfo_scatter_assemble then uses it instead of
  * per-entry searches, and stokesfo_jacobian_csr becomes available.  A node
  * with more than 256 neighbour nodes returns EUNSUPPORTED; a missing entry

@@ -41,6 +41,7 @@ struct stokesfo_ctx {
     const uint64_t *slots = nullptr;   // per-cell CSR slots (set by stokesfo_csr_slots)
     const int64_t *inc_ptr = nullptr;  // node -> (cell N + i) incidence on the device (in the slots buffer)
     const int32_t *inc = nullptr;
+    const uint64_t *nrec = nullptr;    // per-node pull records (in the slots buffer; csr_gather_kernel)
     std::vector<int64_t> inc_ptr_h;    // host incidence from the last csr_pattern fill (until csr_slots)
     std::vector<int32_t> inc_h;
     // lateral pressure term attached for the Newton driver (stokesfo_set_lateral)
@@ -573,11 +574,15 @@ static int64_t slots_off_incptr(const stokesfo_ctx *c) { return round_up(c->d.nu
 static int64_t slots_off_inc(const stokesfo_ctx *c) {
     return slots_off_incptr(c) + round_up((c->d.num_nodes + 1) * 8, 16);
 }
+// + per-node pull records [nodes][NREC_WORDS] uint64 (csr_gather_kernel)
+static int64_t slots_off_nrec(const stokesfo_ctx *c) {
+    return slots_off_inc(c) + round_up(c->d.num_cells * c->N * 4, 128);
+}
 
 int stokesfo_csr_slots_size(stokesfo_ctx *c, size_t *bytes) {
     SFO_RANGE("stokesfo_csr_slots_size");
     if (!c || !bytes) return STOKESFO_EINVAL;
-    *bytes = (size_t)(slots_off_inc(c) + round_up(c->d.num_cells * c->N * 4, 16));
+    *bytes = (size_t)(slots_off_nrec(c) + c->d.num_nodes * NREC_WORDS * 8);
     return STOKESFO_OK;
 }
 
@@ -611,6 +616,16 @@ int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots) {
         c->inc = in;
         std::vector<int64_t>().swap(c->inc_ptr_h);
         std::vector<int32_t>().swap(c->inc_h);
+    }
+    if (c->inc_ptr && c->inc && c->d.num_nodes > 0) {  // per-node pull records
+        uint64_t *nrec = reinterpret_cast<uint64_t *>(base + slots_off_nrec(c));
+        const int bs = 256;
+        const unsigned g = (unsigned)((c->d.num_nodes + bs - 1) / bs);
+        if (c->N == 8)
+            node_rec_kernel<8><<<g, bs, 0, c->stream>>>(c->d.num_nodes, c->rowptr, c->inc_ptr, c->inc, slots, nrec);
+        else
+            node_rec_kernel<6><<<g, bs, 0, c->stream>>>(c->d.num_nodes, c->rowptr, c->inc_ptr, c->inc, slots, nrec);
+        c->nrec = nrec;
     }
     return cuda_status();
 }
@@ -720,16 +735,16 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
         if (!c->rowptr || !c->colidx) return STOKESFO_EINVAL;
         const int64_t work = C * 2 * c->N;
         const unsigned g = (unsigned)((work + bs - 1) / bs);
-        if (c->slots && c->inc && c->csr_maxdeg <= CSR_GATHER_MAXDEG && pull) {  // atomic-free, deterministic
+        if (c->slots && c->nrec && c->csr_maxdeg <= CSR_GATHER_MAXDEG && pull) {  // atomic-free, deterministic
             const int64_t NN = c->d.num_nodes;
             const int64_t per_block = (int64_t)CSR_GATHER_WARPS * CSR_GATHER_NPW;
             const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
             if (c->N == 8)
-                csr_gather_kernel<8><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr,
-                                                                                 c->inc, c->slots, csr_vals);
+                csr_gather_kernel<8><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->nrec, c->inc,
+                                                                                 c->slots, csr_vals);
             else
-                csr_gather_kernel<6><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr,
-                                                                                 c->inc, c->slots, csr_vals);
+                csr_gather_kernel<6><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->nrec, c->inc,
+                                                                                 c->slots, csr_vals);
         } else if (c->slots) {  // slot table attached: no per-entry search
             if (c->N == 8)
                 scatter_csr_slots_kernel<8><<<g, bs, 0, c->stream>>>(C, c->d.conn, J_cell, c->rowptr, c->slots, csr_vals);
@@ -747,29 +762,21 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
 template <bool PACKED>
 static int assemble_csr_impl(stokesfo_ctx *c, const double *J_cell, double *csr_vals, int accumulate) {
     if (!c || !J_cell || !csr_vals || !aligned(J_cell, 16) || !aligned(csr_vals, 16)) return STOKESFO_EINVAL;
-    if (!c->slots || !c->inc || !c->rowptr) return STOKESFO_EINVAL;  // needs stokesfo_csr_slots
+    if (!c->slots || !c->nrec || !c->rowptr) return STOKESFO_EINVAL;  // needs stokesfo_csr_slots
     if (c->csr_maxdeg > CSR_GATHER_MAXDEG) return STOKESFO_EUNSUPPORTED;
     const int64_t NN = c->d.num_nodes;
     if (NN == 0) return STOKESFO_OK;
     const int64_t per_block = (int64_t)CSR_GATHER_WARPS * CSR_GATHER_NPW;
     const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
     const int bt = 32 * CSR_GATHER_WARPS;
-#define PULL(K, NN_, ACC_) K<NN_, ACC_><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->rowptr, c->inc_ptr, c->inc, c->slots, csr_vals)
-    if (PACKED) {
-        if (!aligned(J_cell, 32)) return STOKESFO_EINVAL;
-        if (c->N == 8) {
-            if (accumulate) PULL(csr_gather_packed_kernel, 8, true);
-            else PULL(csr_gather_packed_kernel, 8, false);
-        } else {
-            if (accumulate) PULL(csr_gather_packed_kernel, 6, true);
-            else PULL(csr_gather_packed_kernel, 6, false);
-        }
-    } else if (c->N == 8) {
-        if (accumulate) PULL(csr_gather_kernel, 8, true);
-        else PULL(csr_gather_kernel, 8, false);
+#define PULL(NN_, ACC_)                                                                                       \
+    csr_gather_kernel<NN_, ACC_, PACKED><<<gg, bt, 0, c->stream>>>(NN, J_cell, c->nrec, c->inc, c->slots, csr_vals)
+    if (c->N == 8) {
+        if (accumulate) PULL(8, true);
+        else PULL(8, false);
     } else {
-        if (accumulate) PULL(csr_gather_kernel, 6, true);
-        else PULL(csr_gather_kernel, 6, false);
+        if (accumulate) PULL(6, true);
+        else PULL(6, false);
     }
 #undef PULL
     return cuda_status();
@@ -1284,6 +1291,7 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
     c->slots = nullptr;  // a new pattern invalidates an attached slot table
     c->inc_ptr = nullptr;
     c->inc = nullptr;
+    c->nrec = nullptr;
     c->inc_ptr_h = std::move(nc);
     c->inc_h = std::move(ncell);
     return STOKESFO_OK;

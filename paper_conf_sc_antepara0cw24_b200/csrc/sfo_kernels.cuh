@@ -2280,29 +2280,71 @@ constexpr int CSR_GATHER_MAXDEG = 64;   // neighbour nodes per node (else the at
 constexpr int CSR_GATHER_WARPS = 8;
 constexpr int CSR_GATHER_NPW = 2;       // nodes per warp
 // ACC = false: the rows are overwritten (vals = assembled J; no prior zeroing, no read of vals).
-template <int N, bool ACC = true>
+// row pair (2 i + a, columns 2 j, 2 j + 1) of cell `cell`'s element matrix: full [C][2N][2N] (streamed
+// once) or symmetric block-packed (block (i, j) or the transpose of block (j, i); each off-diagonal
+// block is read by two node warps, so the packed reads keep the default L2 policy)
+template <int N, bool PACKED>
+__device__ __forceinline__ double2 jrow2(const double *__restrict__ Jc, int64_t cell, int i, int a, int j) {
+    if (!PACKED) return __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * 2 * N + 2 * i + a) * 2 * N) + j);
+    const double *b = Jc + cell * (4 * pk_blocks<N>());
+    if (j >= i) return __ldg(reinterpret_cast<const double2 *>(b + 4 * pk_block<N>(i, j) + 2 * a));
+    const double *t = b + 4 * pk_block<N>(j, i);
+    return make_double2(__ldg(t + a), __ldg(t + 2 + a));
+}
+// Per-node pull record (built once by stokesfo_csr_slots, 128 B per node, 16 words): everything the pull
+// assembly needs before it can load element-matrix rows, in one coalesced load per node instead of the dependent
+// chain rowptr / inc_ptr -> inc -> slots (three DRAM round trips per task; ncu r2g: long_sb 43-44%).
+//   w0 CSR row base r0 (rowptr[2v]); w1 = len (both rows) | cnt << 32; w2..w5 the first 8 incidence entries
+//   (cell N + i) as int32 pairs; w6..w13 their slot rows; w14 = incidence start k0 (the rare > 8 path)
+constexpr int NREC_WORDS = 16;
+template <int N>
+__global__ void node_rec_kernel(int64_t nnodes, const int64_t *__restrict__ rowptr, const int64_t *__restrict__ inc_ptr,
+                                const int32_t *__restrict__ inc, const uint64_t *__restrict__ slots,
+                                uint64_t *__restrict__ rec) {
+    const int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (v >= nnodes) return;
+    const int64_t r0 = rowptr[2 * v], k0 = inc_ptr[v];
+    const int len = (int)(rowptr[2 * v + 2] - r0), cnt = (int)(inc_ptr[v + 1] - k0);
+    uint64_t w[NREC_WORDS];
+    w[0] = (uint64_t)r0;
+    w[1] = (uint64_t)(uint32_t)len | ((uint64_t)(uint32_t)cnt << 32);
+    for (int e = 0; e < 8; ++e) {
+        const int32_t ci = e < cnt ? inc[k0 + e] : 0;
+        if (e & 1) w[2 + e / 2] |= (uint64_t)(uint32_t)ci << 32;
+        else w[2 + e / 2] = (uint32_t)ci;
+        w[6 + e] = e < cnt ? slots[ci] : 0;
+    }
+    w[14] = (uint64_t)k0;
+    w[15] = 0;
+    uint4 *o = reinterpret_cast<uint4 *>(rec + v * NREC_WORDS);
+    for (int k = 0; k < NREC_WORDS / 2; ++k) o[k] = make_uint4((uint32_t)w[2 * k], (uint32_t)(w[2 * k] >> 32),
+                                                             (uint32_t)w[2 * k + 1], (uint32_t)(w[2 * k + 1] >> 32));
+}
+
+template <int N, bool ACC = true, bool PACKED = false>
 __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
-    csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const int64_t *__restrict__ rowptr,
-                      const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
-                      const uint64_t *__restrict__ slots, double *__restrict__ vals) {
-    constexpr int ND = 2 * N;
+    csr_gather_kernel(int64_t nnodes, const double *__restrict__ Jc, const uint64_t *__restrict__ nrec,
+                      const int32_t *__restrict__ inc, const uint64_t *__restrict__ slots, double *__restrict__ vals) {
     constexpr int LC = 2 * N;            // lanes per cell: each loads one (j, b = 0..1) pair of one row
     constexpr int CPI = 32 / LC;         // cells per load instruction (2 for hex8 and wedge6)
-    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW, NI = BATCH / CPI;
+    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, NI = BATCH / CPI;
     __shared__ __align__(16) double buf[CSR_GATHER_WARPS][NPW][4 * CSR_GATHER_MAXDEG];
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
     const int64_t v0 = (blockIdx.x * (int64_t)CSR_GATHER_WARPS + w) * NPW;
     if (v0 >= nnodes) return;  // uniform per warp
+    static_assert(NPW * NREC_WORDS == 32, "one record word per lane");
+    // lane l holds word l % 16 of node l / 16's pull record
+    const int64_t vr = v0 + l / NREC_WORDS;
+    const uint64_t rw = vr < nnodes ? __ldg(nrec + vr * NREC_WORDS + (l % NREC_WORDS)) : 0;
     int64_t r0[NPW], k0[NPW];
     int len[NPW], cnt[NPW];
 #pragma unroll
     for (int n = 0; n < NPW; ++n) {
-        const bool ok = v0 + n < nnodes;
-        const int64_t v = ok ? v0 + n : v0;
-        r0[n] = __ldg(rowptr + 2 * v);
-        len[n] = ok ? (int)(__ldg(rowptr + 2 * v + 2) - r0[n]) : 0;  // both rows: 4 deg entries
-        k0[n] = __ldg(inc_ptr + v);
-        cnt[n] = ok ? (int)(__ldg(inc_ptr + v + 1) - k0[n]) : 0;
+        r0[n] = (int64_t)__shfl_sync(0xffffffffu, rw, n * NREC_WORDS);
+        const uint64_t lc = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 1);
+        len[n] = (int)(uint32_t)lc;  // both rows: 4 deg entries
+        cnt[n] = (int)(uint32_t)(lc >> 32);
+        k0[n] = (int64_t)__shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 14);
     }
     // pull the rows' vals lines into L2 now: the final read-modify-write then hits L2
     if (ACC) {
@@ -2311,12 +2353,6 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
             for (int p = 16 * l; p < len[n]; p += 16 * 32)
                 asm volatile("prefetch.global.L2 [%0];" ::"l"(vals + r0[n] + p));
     }
-    // incidence: lane n LPN + t holds entry t (< BATCH) of node n
-    const int ln = l / LPN, lt = l % LPN;
-    int32_t my = 0;
-#pragma unroll
-    for (int n = 0; n < NPW; ++n)
-        if (ln == n && lt < cnt[n] && lt < BATCH) my = __ldg(inc + k0[n] + lt);
 #pragma unroll
     for (int n = 0; n < NPW; ++n)
         for (int p = 2 * l; p < len[n]; p += 64) *reinterpret_cast<double2 *>(&buf[w][n][p]) = make_double2(0.0, 0.0);
@@ -2331,13 +2367,14 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
 #pragma unroll
         for (int t = 0; t < NI; ++t) {
             const int e = CPI * t + (u < CPI ? u : 0);  // incidence entry of this lane
-            const int32_t ci = __shfl_sync(0xffffffffu, my, n * LPN + e);
+            const uint64_t cp = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 2 + (e >> 1));
+            const uint64_t srow = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 6 + e);
+            const int32_t ci = (int32_t)(uint32_t)((e & 1) ? (cp >> 32) : cp);
             const bool live = lane_ok && e < cnt[n];
             const int64_t cell = ci / N;
             const int i = ci - (int)(cell * N);
-            x[n][t] = live ? __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j)
-                           : make_double2(0.0, 0.0);
-            sl[n][t] = live ? (int)__ldg(sb + 8 * (int64_t)ci + j) : -1;
+            x[n][t] = live ? jrow2<N, PACKED>(Jc, cell, i, a, j) : make_double2(0.0, 0.0);
+            sl[n][t] = live ? (int)((srow >> (8 * j)) & 0xffu) : -1;
         }
     __syncwarp();
 #pragma unroll
@@ -2364,7 +2401,7 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
             const int i = ci - (int)(cell * N);
             if (l < LC) {
                 const int s = (int)__ldg(sb + 8 * (int64_t)ci + j);
-                const double2 y = __ldcs(reinterpret_cast<const double2 *>(Jc + (cell * ND + 2 * i + a) * ND) + j);
+                const double2 y = jrow2<N, PACKED>(Jc, cell, i, a, j);
                 buf[w][n][a * half + 2 * s] += y.x;
                 buf[w][n][a * half + 2 * s + 1] += y.y;
             }
@@ -2384,141 +2421,6 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
                 *o = c;
             } else {
                 __stcs(o, b);  // streamed: the assembled matrix is not re-read by this kernel
-            }
-        }
-}
-
-// Pull assembly from the symmetric block-packed element matrices: lane <-> (incident cell u, column node j)
-// loads the whole 2 x 2 block (i, j) -- or block (j, i), transposed in registers -- with one 256-bit load
-// (a full 32-B sector; the row-pair mapping of csr_gather_kernel needs two scalar loads for every transposed
-// block: C4 5.46 vs 5.04 ms, ncu r2g), and adds both of its rows to the node's two CSR rows in shared memory.
-__device__ __forceinline__ double4 ld_v4_nc(const double *p) {
-    double4 v;
-    asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w) : "l"(p));
-    return v;
-}
-template <int N, bool ACC = true>
-__global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
-    csr_gather_packed_kernel(int64_t nnodes, const double *__restrict__ Jp, const int64_t *__restrict__ rowptr,
-                             const int64_t *__restrict__ inc_ptr, const int32_t *__restrict__ inc,
-                             const uint64_t *__restrict__ slots, double *__restrict__ vals) {
-    constexpr int CPI = 32 / N;  // cells per load instruction (hex8 4, wedge6 5)
-    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, LPN = 32 / NPW, NI = (BATCH + CPI - 1) / CPI;
-    constexpr int NB = pk_blocks<N>();
-    __shared__ __align__(16) double buf[CSR_GATHER_WARPS][NPW][4 * CSR_GATHER_MAXDEG];
-    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
-    const int64_t v0 = (blockIdx.x * (int64_t)CSR_GATHER_WARPS + w) * NPW;
-    if (v0 >= nnodes) return;  // uniform per warp
-    int64_t r0[NPW], k0[NPW];
-    int len[NPW], cnt[NPW];
-#pragma unroll
-    for (int n = 0; n < NPW; ++n) {
-        const bool ok = v0 + n < nnodes;
-        const int64_t v = ok ? v0 + n : v0;
-        r0[n] = __ldg(rowptr + 2 * v);
-        len[n] = ok ? (int)(__ldg(rowptr + 2 * v + 2) - r0[n]) : 0;  // both rows: 4 deg entries
-        k0[n] = __ldg(inc_ptr + v);
-        cnt[n] = ok ? (int)(__ldg(inc_ptr + v + 1) - k0[n]) : 0;
-    }
-    if (ACC) {
-#pragma unroll
-        for (int n = 0; n < NPW; ++n)
-            for (int p = 16 * l; p < len[n]; p += 16 * 32)
-                asm volatile("prefetch.global.L2 [%0];" ::"l"(vals + r0[n] + p));
-    }
-    const int ln = l / LPN, lt = l % LPN;
-    int32_t my = 0;
-#pragma unroll
-    for (int n = 0; n < NPW; ++n)
-        if (ln == n && lt < cnt[n] && lt < BATCH) my = __ldg(inc + k0[n] + lt);
-#pragma unroll
-    for (int n = 0; n < NPW; ++n)
-        for (int p = 2 * l; p < len[n]; p += 64) *reinterpret_cast<double2 *>(&buf[w][n][p]) = make_double2(0.0, 0.0);
-    // lane l <-> (cell u = l / N of the group, column node j = l % N)
-    const int u = l / N, j = l % N;
-    const bool lane_ok = l < CPI * N;
-    double2 x0[NPW][NI], x1[NPW][NI];  // rows (i, 0) and (i, 1), columns (j, 0..1)
-    int sl[NPW][NI];
-    const uint8_t *sb = reinterpret_cast<const uint8_t *>(slots);
-#pragma unroll
-    for (int n = 0; n < NPW; ++n)
-#pragma unroll
-        for (int t = 0; t < NI; ++t) {
-            const int e = CPI * t + u;  // incidence entry of this lane
-            const bool live = lane_ok && e < BATCH && e < cnt[n];
-            const int32_t ci = __shfl_sync(0xffffffffu, my, n * LPN + (e < BATCH ? e : 0));
-            const int64_t cell = ci / N;
-            const int i = ci - (int)(cell * N);
-            x0[n][t] = x1[n][t] = make_double2(0.0, 0.0);
-            sl[n][t] = -1;
-            if (live) {
-                const double *b = Jp + cell * (4 * NB);
-                if (j >= i) {
-                    const double4 q = ld_v4_nc(b + 4 * pk_block<N>(i, j));
-                    x0[n][t] = make_double2(q.x, q.y);
-                    x1[n][t] = make_double2(q.z, q.w);
-                } else {  // block (j, i): entries [c][d] = J[(j,c),(i,d)], so J[(i,a),(j,b)] = [b][a]
-                    const double4 q = ld_v4_nc(b + 4 * pk_block<N>(j, i));
-                    x0[n][t] = make_double2(q.x, q.z);
-                    x1[n][t] = make_double2(q.y, q.w);
-                }
-                sl[n][t] = (int)__ldg(sb + 8 * (int64_t)ci + j);
-            }
-        }
-    __syncwarp();
-#pragma unroll
-    for (int n = 0; n < NPW; ++n) {
-        const int half = len[n] >> 1;
-        // the CPI cells of a load group may hit the same entries: add them in turn
-#pragma unroll
-        for (int t = 0; t < NI; ++t)
-#pragma unroll
-            for (int uu = 0; uu < CPI; ++uu) {
-                if (u == uu && sl[n][t] >= 0) {
-                    double2 *p0 = reinterpret_cast<double2 *>(&buf[w][n][2 * sl[n][t]]);
-                    double2 *p1 = reinterpret_cast<double2 *>(&buf[w][n][half + 2 * sl[n][t]]);
-                    double2 b0 = *p0, b1 = *p1;
-                    b0.x += x0[n][t].x;
-                    b0.y += x0[n][t].y;
-                    b1.x += x1[n][t].x;
-                    b1.y += x1[n][t].y;
-                    *p0 = b0;
-                    *p1 = b1;
-                }
-                __syncwarp();
-            }
-        // rare: more than BATCH incident cells (not on extruded hex8 / wedge6 meshes)
-        for (int64_t k = k0[n] + BATCH; k < k0[n] + cnt[n]; ++k) {
-            const int32_t ci = __ldg(inc + k);
-            const int64_t cell = ci / N;
-            const int i = ci - (int)(cell * N);
-            if (l < N) {
-                const int s = (int)__ldg(sb + 8 * (int64_t)ci + j);
-                const double *b = Jp + cell * (4 * NB);
-                const double4 q = ld_v4_nc(b + 4 * (j >= i ? pk_block<N>(i, j) : pk_block<N>(j, i)));
-                const double2 y0 = j >= i ? make_double2(q.x, q.y) : make_double2(q.x, q.z);
-                const double2 y1 = j >= i ? make_double2(q.z, q.w) : make_double2(q.y, q.w);
-                buf[w][n][2 * s] += y0.x;
-                buf[w][n][2 * s + 1] += y0.y;
-                buf[w][n][half + 2 * s] += y1.x;
-                buf[w][n][half + 2 * s + 1] += y1.y;
-            }
-            __syncwarp();
-        }
-    }
-    __syncwarp();
-#pragma unroll
-    for (int n = 0; n < NPW; ++n)
-        for (int p = 2 * l; p < len[n]; p += 64) {
-            double2 *o = reinterpret_cast<double2 *>(vals + r0[n] + p);
-            const double2 b = *reinterpret_cast<const double2 *>(&buf[w][n][p]);
-            if (ACC) {
-                double2 c = *o;
-                c.x += b.x;
-                c.y += b.y;
-                *o = c;
-            } else {
-                __stcs(o, b);
             }
         }
 }

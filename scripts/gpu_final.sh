@@ -14,7 +14,9 @@ timeout 900 python bench.py --impl reference --steps 5 --warmup 3 > $OUT/bench_r
 for A in "--config C3" "--config C5" "--config C4p" "--config C4 --op resid" "--config C5 --op resid" \
          "--config C4 --op jvp" "--config C4 --geometry compact" "--config C4 --op jvp --geometry compact" \
          "--config C5 --geometry compact" "--config C4 --geometry on_the_fly" "--config C4 --op jac_global" \
-         "--config C4 --op jac_csr" "--config C4 --op jvp_y" "--config C4 --op jvp_y --geometry compact" "--config C1"; do
+         "--config C4 --op jac_csr" "--config C4 --op jvp_y" "--config C4 --op jvp_y --geometry compact" "--config C1" \
+         "--config C4 --op jac_global --global-format full" "--config C3 --op jac_global" \
+         "--config C5 --op jac_global --global-format full" "--config C5 --op jvp" "--config C4 --op jvp --geometry compact"; do
   timeout 900 python bench.py $A --no-cpu-baseline >> $OUT/bench_lines.jsonl 2>> $OUT/bench_lines.err
 done
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \

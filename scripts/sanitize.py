@@ -1,6 +1,7 @@
 """Runs of every kernel variant for compute-sanitizer (memcheck / racecheck /
 synccheck / initcheck): hex8 + wedge6, stored + on-the-fly + compact geometry, residual
-(partial-sum exchange), Jacobian, J.v, diagonal, fused CSR, slot table + pull assembly,
+(partial-sum exchange), Jacobian (vector and tensor-core kernels, packed form), J.v, diagonal, fused CSR,
+slot table + pull assembly (full and packed),
 ragged tiles, side sets, the NEXT-1 chain and a short Newton solve.  A second,
 larger mesh (more tiles than resident warps) exercises the persistent tile
 loop: record ring refills, next-tile gathers and the partial-sum overlay of a
@@ -37,6 +38,21 @@ def run(elem, n, L, drop, full):
         vals = torch.zeros(ci.numel(), dtype=torch.float64, device="cuda")
         ctx.jacobian_csr(Ud, vals, R=R)
         ctx.scatter_assemble(R_cell=Rc, R=R, J_cell=J, csr_vals=vals)
+        ctx.assemble_csr(J, vals, accumulate=False)
+        if geo != "on_the_fly":  # tensor-core kernels: packed element matrices + their pull assembly
+            Jp = torch.empty((C, N * (N + 1) // 2, 2, 2), dtype=torch.float64, device="cuda")
+            ctx.jacobian_packed(Ud, Jp, R_cell=Rc, R=R)
+            ctx.assemble_csr_packed(Jp, vals, accumulate=True)
+            Jm = torch.empty((C * 4 * N * N + 2,), dtype=torch.float64, device="cuda")[2:].view(C, 2 * N, 2 * N)
+            ctx.jacobian(Ud, Jm, R=R)  # 16-B aligned only: the vector kernel
+            if elem == "wedge6":  # the wedge6 DMMA kernel (opt-in)
+                os.environ["STOKESFO_JAC_MMA"] = "1"
+                c2 = StokesFO(elem, torch.from_numpy(conn).cuda(), torch.from_numpy(coords).cuda(),
+                              surface=torch.from_numpy(s).cuda(), flow_factor=torch.from_numpy(kc).cuda(),
+                              geometry=geo)
+                del os.environ["STOKESFO_JAC_MMA"]
+                c2.jacobian(Ud, J, R_cell=Rc, R=R)
+                c2.sync()
         ctx.sync()
         if not full:
             continue
