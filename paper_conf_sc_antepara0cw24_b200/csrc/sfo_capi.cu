@@ -616,6 +616,15 @@ int stokesfo_csr_slots(stokesfo_ctx *c, uint64_t *slots) {
         c->inc = in;
         std::vector<int64_t>().swap(c->inc_ptr_h);
         std::vector<int32_t>().swap(c->inc_h);
+    } else if (c->inc_ptr && c->inc && c->inc_ptr != ip) {
+        // a second slot table for the same pattern: carry the incidence over from the previous buffer, so the
+        // new table does not depend on the old buffer staying allocated
+        if (cudaMemcpyAsync(ip, c->inc_ptr, (c->d.num_nodes + 1) * 8, cudaMemcpyDeviceToDevice, c->stream) !=
+                cudaSuccess ||
+            (work > 0 && cudaMemcpyAsync(in, c->inc, work * 4, cudaMemcpyDeviceToDevice, c->stream) != cudaSuccess))
+            return cuda_status();
+        c->inc_ptr = ip;
+        c->inc = in;
     }
     if (c->inc_ptr && c->inc && c->d.num_nodes > 0) {  // per-node pull records
         uint64_t *nrec = reinterpret_cast<uint64_t *>(base + slots_off_nrec(c));

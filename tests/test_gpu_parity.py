@@ -445,6 +445,33 @@ def test_csr_slots_and_fused_assembly(torch, elem, geometry):
     _assembled_check(R.cpu().numpy(), orc, ref["R_cell"])
 
 
+@pytest.mark.parametrize("elem", ["hex8", "wedge6"])
+def test_second_slot_table_is_self_contained(torch, elem):
+    """A second stokesfo_csr_slots call into a new buffer (same pattern) carries the node incidence and
+    rebuilds the per-node pull records in that buffer: overwriting the first buffer afterwards must not change
+    the pull assembly (it matches the oracle's CSR scatter)."""
+    ctx, orc = _setup(torch, elem, n=5, L=3, drop=2)
+    C, N = ctx.num_cells, ctx.N
+    conn = orc["conn"]
+    rowptr, colidx = ctx.csr_pattern()
+    rp2, ci2 = O.csr_pattern(conn, ctx.num_nodes)
+    ctx.csr_slots()
+    first = ctx.slots
+    ctx.csr_slots()
+    assert ctx.slots.data_ptr() != first.data_ptr()
+    first.fill_(-1)  # garbage where the first table, incidence and records were
+    ref = O.evaluate(orc["e"], conn, orc["G"], orc["wm"], orc["U"], surface=orc["s"], kc=orc["kc"], mode="jac")
+    v2, _ = O.scatter_csr(orc["e"], conn, ref["J_cell"], rp2, ci2)
+    cell_scale = np.abs(ref["J_cell"]).reshape(C, -1).max(1)[:, None, None] * np.ones_like(ref["J_cell"])
+    a2, _ = O.scatter_csr(orc["e"], conn, cell_scale, rp2, ci2)
+    J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
+    ctx.jacobian(_t(torch, orc["U"]), J)
+    vals = torch.full((colidx.numel(),), float("nan"), dtype=torch.float64, device="cuda")
+    ctx.assemble_csr(J, vals, accumulate=False)
+    ctx.sync()
+    assert (np.abs(vals.cpu().numpy() - v2) <= TOL * a2).all()
+
+
 def _unpack_blocks(Jp, N):
     """Full [C][2N][2N] element matrices from the symmetric block-packed form (header: block (i, j >= i) at
     index i N - i (i - 1) / 2 + (j - i), entries [a][b] = J[(i,a),(j,b)]; block (j, i) = block (i, j)^T)."""
