@@ -190,7 +190,11 @@ int stokesfo_lateral_pressure(stokesfo_ctx *c, const int32_t *faces, int64_t nfa
 int stokesfo_set_lateral(stokesfo_ctx *c, const int32_t *faces, int64_t nfaces, const double *surface,
                          double rho_i_g, double rho_w_g, double sea_level);
 
-/* Assembly: R[2 conn[c][n] + a] += R_cell[c][n][a] (if R_cell and R are non-NULL)
+/* Assembly: the sum over cells of eq. (3)
+ * into the global residual and into the global Jacobian matrix that the damped
+ * Newton method computes at each nonlinear iteration and hands to GMRES with a
+ * matrix-dependent AMG preconditioner (section III-A).
+ * R[2 conn[c][n] + a] += R_cell[c][n][a] (if R_cell and R are non-NULL)
  * and csr_vals[pos(row, col)] += J_cell[c][k][l] (if J_cell and csr_vals are
  * non-NULL; requires an earlier stokesfo_csr_pattern call with non-NULL rowptr
  * and colidx, which must stay valid). */
@@ -226,7 +230,9 @@ int stokesfo_jacobian_packed(stokesfo_ctx *c, const double *U, double *Jp, doubl
  * accumulate semantics as stokesfo_assemble_csr. */
 int stokesfo_assemble_csr_packed(stokesfo_ctx *c, const double *Jp, double *csr_vals, int accumulate);
 
-/* CSR pattern over dofs (rows = 2*num_nodes; columns of a row = sorted dofs of
+/* CSR pattern of the global Jacobian matrix (NEXT-2; section III-A:
+ * computed at each nonlinear iteration, used by the matrix-dependent AMG) over dofs
+ * (rows = 2*num_nodes; columns of a row = sorted dofs of
  * every node sharing a cell with the row's node).  Size query: pass rowptr =
  * colidx = NULL to get *nnz.  Fill: rowptr dev [2*num_nodes+1] int64, colidx
  * dev [nnz] int32.  Synchronises the stream (host-side construction from a

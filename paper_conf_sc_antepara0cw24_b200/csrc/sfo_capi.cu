@@ -574,7 +574,7 @@ static int64_t slots_off_incptr(const stokesfo_ctx *c) { return round_up(c->d.nu
 static int64_t slots_off_inc(const stokesfo_ctx *c) {
     return slots_off_incptr(c) + round_up((c->d.num_nodes + 1) * 8, 16);
 }
-// + per-node pull records [nodes][NREC_WORDS] uint64 (csr_gather_kernel)
+// + per-node pull records [nodes][PullCfg<N>::WORDS] uint64 (csr_gather_kernel)
 static int64_t slots_off_nrec(const stokesfo_ctx *c) {
     return slots_off_inc(c) + round_up(c->d.num_cells * c->N * 4, 128);
 }
@@ -582,7 +582,7 @@ static int64_t slots_off_nrec(const stokesfo_ctx *c) {
 int stokesfo_csr_slots_size(stokesfo_ctx *c, size_t *bytes) {
     SFO_RANGE("stokesfo_csr_slots_size");
     if (!c || !bytes) return STOKESFO_EINVAL;
-    *bytes = (size_t)(slots_off_nrec(c) + c->d.num_nodes * NREC_WORDS * 8);
+    *bytes = (size_t)(slots_off_nrec(c) + c->d.num_nodes * (c->N == 8 ? pull_words<8>() : pull_words<6>()) * 8);
     return STOKESFO_OK;
 }
 
@@ -746,7 +746,7 @@ int stokesfo_scatter_assemble(stokesfo_ctx *c, const double *R_cell, double *R, 
         const unsigned g = (unsigned)((work + bs - 1) / bs);
         if (c->slots && c->nrec && c->csr_maxdeg <= CSR_GATHER_MAXDEG && pull) {  // atomic-free, deterministic
             const int64_t NN = c->d.num_nodes;
-            const int64_t per_block = (int64_t)CSR_GATHER_WARPS * CSR_GATHER_NPW;
+            const int64_t per_block = (int64_t)CSR_GATHER_WARPS * (c->N == 8 ? pull_npw<8>() : pull_npw<6>());
             const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
             if (c->N == 8)
                 csr_gather_kernel<8><<<gg, 32 * CSR_GATHER_WARPS, 0, c->stream>>>(NN, J_cell, c->nrec, c->inc,
@@ -775,7 +775,7 @@ static int assemble_csr_impl(stokesfo_ctx *c, const double *J_cell, double *csr_
     if (c->csr_maxdeg > CSR_GATHER_MAXDEG) return STOKESFO_EUNSUPPORTED;
     const int64_t NN = c->d.num_nodes;
     if (NN == 0) return STOKESFO_OK;
-    const int64_t per_block = (int64_t)CSR_GATHER_WARPS * CSR_GATHER_NPW;
+    const int64_t per_block = (int64_t)CSR_GATHER_WARPS * (c->N == 8 ? pull_npw<8>() : pull_npw<6>());
     const unsigned gg = (unsigned)((NN + per_block - 1) / per_block);
     const int bt = 32 * CSR_GATHER_WARPS;
 #define PULL(NN_, ACC_)                                                                                       \

@@ -2278,7 +2278,25 @@ __global__ void scatter_csr_slots_kernel(int64_t ncells, const int32_t *__restri
 // what sets its speed.
 constexpr int CSR_GATHER_MAXDEG = 64;   // neighbour nodes per node (else the atomic kernel)
 constexpr int CSR_GATHER_WARPS = 8;
-constexpr int CSR_GATHER_NPW = 2;       // nodes per warp
+// Per element type: nodes per warp, incident cells handled in the batched path (an interior node of an
+// extruded mesh has 2 x (cells around a footprint vertex): hex8 (quads) 8, wedge6 (triangles) 12 on the
+// Voronoi-dual triangulation), and 64-bit words of the per-node pull record.
+template <int N>
+struct PullCfg {
+    static constexpr int NPW = N == 8 ? 2 : 1;
+    static constexpr int BATCH = N == 8 ? 8 : 12;
+    static constexpr int WORDS = 32 / NPW;
+    static constexpr int CI0 = 2, SR0 = CI0 + BATCH / 2, K0W = SR0 + BATCH;  // record word offsets
+    static_assert(K0W < WORDS, "record fits");
+};
+template <int N>
+__host__ __device__ constexpr int pull_npw() {
+    return PullCfg<N>::NPW;
+}
+template <int N>
+__host__ __device__ constexpr int pull_words() {
+    return PullCfg<N>::WORDS;
+}
 // ACC = false: the rows are overwritten (vals = assembled J; no prior zeroing, no read of vals).
 // row pair (2 i + a, columns 2 j, 2 j + 1) of cell `cell`'s element matrix: full [C][2N][2N] (streamed
 // once) or symmetric block-packed (block (i, j) or the transpose of block (j, i); each off-diagonal
@@ -2291,34 +2309,34 @@ __device__ __forceinline__ double2 jrow2(const double *__restrict__ Jc, int64_t 
     const double *t = b + 4 * pk_block<N>(j, i);
     return make_double2(__ldg(t + a), __ldg(t + 2 + a));
 }
-// Per-node pull record (built once by stokesfo_csr_slots, 128 B per node, 16 words): everything the pull
-// assembly needs before it can load element-matrix rows, in one coalesced load per node instead of the dependent
-// chain rowptr / inc_ptr -> inc -> slots (three DRAM round trips per task; ncu r2g: long_sb 43-44%).
-//   w0 CSR row base r0 (rowptr[2v]); w1 = len (both rows) | cnt << 32; w2..w5 the first 8 incidence entries
-//   (cell N + i) as int32 pairs; w6..w13 their slot rows; w14 = incidence start k0 (the rare > 8 path)
-constexpr int NREC_WORDS = 16;
+// Per-node pull record (built once by stokesfo_csr_slots; PullCfg<N>::WORDS 64-bit words per node: 128 B hex8,
+// 256 B wedge6): everything the pull assembly needs before it can load element-matrix rows, in one coalesced
+// load per node instead of the dependent chain rowptr / inc_ptr -> inc -> slots (three DRAM round trips per task;
+// ncu r2g: long_sb 43-44%).
+//   w0 CSR row base r0 (rowptr[2v]); w1 = len (both rows) | cnt << 32; w[CI0..) the first BATCH incidence
+//   entries (cell N + i) as int32 pairs; w[SR0..) their slot rows; w[K0W] = incidence start k0 (> BATCH path)
 template <int N>
 __global__ void node_rec_kernel(int64_t nnodes, const int64_t *__restrict__ rowptr, const int64_t *__restrict__ inc_ptr,
                                 const int32_t *__restrict__ inc, const uint64_t *__restrict__ slots,
                                 uint64_t *__restrict__ rec) {
+    using P = PullCfg<N>;
     const int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (v >= nnodes) return;
     const int64_t r0 = rowptr[2 * v], k0 = inc_ptr[v];
     const int len = (int)(rowptr[2 * v + 2] - r0), cnt = (int)(inc_ptr[v + 1] - k0);
-    uint64_t w[NREC_WORDS];
+    uint64_t w[P::WORDS];
+    for (int k = 0; k < P::WORDS; ++k) w[k] = 0;
     w[0] = (uint64_t)r0;
     w[1] = (uint64_t)(uint32_t)len | ((uint64_t)(uint32_t)cnt << 32);
-    for (int e = 0; e < 8; ++e) {
-        const int32_t ci = e < cnt ? inc[k0 + e] : 0;
-        if (e & 1) w[2 + e / 2] |= (uint64_t)(uint32_t)ci << 32;
-        else w[2 + e / 2] = (uint32_t)ci;
-        w[6 + e] = e < cnt ? slots[ci] : 0;
+    for (int e = 0; e < P::BATCH && e < cnt; ++e) {
+        const int32_t ci = inc[k0 + e];
+        w[P::CI0 + e / 2] |= (uint64_t)(uint32_t)ci << (32 * (e & 1));
+        w[P::SR0 + e] = slots[ci];
     }
-    w[14] = (uint64_t)k0;
-    w[15] = 0;
-    uint4 *o = reinterpret_cast<uint4 *>(rec + v * NREC_WORDS);
-    for (int k = 0; k < NREC_WORDS / 2; ++k) o[k] = make_uint4((uint32_t)w[2 * k], (uint32_t)(w[2 * k] >> 32),
-                                                             (uint32_t)w[2 * k + 1], (uint32_t)(w[2 * k + 1] >> 32));
+    w[P::K0W] = (uint64_t)k0;
+    uint4 *o = reinterpret_cast<uint4 *>(rec + v * P::WORDS);
+    for (int k = 0; k < P::WORDS / 2; ++k) o[k] = make_uint4((uint32_t)w[2 * k], (uint32_t)(w[2 * k] >> 32),
+                                                            (uint32_t)w[2 * k + 1], (uint32_t)(w[2 * k + 1] >> 32));
 }
 
 template <int N, bool ACC = true, bool PACKED = false>
@@ -2327,13 +2345,15 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
                       const int32_t *__restrict__ inc, const uint64_t *__restrict__ slots, double *__restrict__ vals) {
     constexpr int LC = 2 * N;            // lanes per cell: each loads one (j, b = 0..1) pair of one row
     constexpr int CPI = 32 / LC;         // cells per load instruction (2 for hex8 and wedge6)
-    constexpr int NPW = CSR_GATHER_NPW, BATCH = 8, NI = BATCH / CPI;
+    using P = PullCfg<N>;
+    constexpr int NPW = P::NPW, BATCH = P::BATCH, NI = BATCH / CPI, NREC_WORDS = P::WORDS;
     __shared__ __align__(16) double buf[CSR_GATHER_WARPS][NPW][4 * CSR_GATHER_MAXDEG];
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
     const int64_t v0 = (blockIdx.x * (int64_t)CSR_GATHER_WARPS + w) * NPW;
     if (v0 >= nnodes) return;  // uniform per warp
+    static_assert(NI * CPI == BATCH, "whole load groups");
     static_assert(NPW * NREC_WORDS == 32, "one record word per lane");
-    // lane l holds word l % 16 of node l / 16's pull record
+    // lane l holds word l % WORDS of node l / WORDS's pull record
     const int64_t vr = v0 + l / NREC_WORDS;
     const uint64_t rw = vr < nnodes ? __ldg(nrec + vr * NREC_WORDS + (l % NREC_WORDS)) : 0;
     int64_t r0[NPW], k0[NPW];
@@ -2344,7 +2364,7 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
         const uint64_t lc = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 1);
         len[n] = (int)(uint32_t)lc;  // both rows: 4 deg entries
         cnt[n] = (int)(uint32_t)(lc >> 32);
-        k0[n] = (int64_t)__shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 14);
+        k0[n] = (int64_t)__shfl_sync(0xffffffffu, rw, n * NREC_WORDS + P::K0W);
     }
     // pull the rows' vals lines into L2 now: the final read-modify-write then hits L2
     if (ACC) {
@@ -2367,8 +2387,8 @@ __global__ void __launch_bounds__(32 * CSR_GATHER_WARPS, 4)
 #pragma unroll
         for (int t = 0; t < NI; ++t) {
             const int e = CPI * t + (u < CPI ? u : 0);  // incidence entry of this lane
-            const uint64_t cp = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 2 + (e >> 1));
-            const uint64_t srow = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + 6 + e);
+            const uint64_t cp = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + P::CI0 + (e >> 1));
+            const uint64_t srow = __shfl_sync(0xffffffffu, rw, n * NREC_WORDS + P::SR0 + e);
             const int32_t ci = (int32_t)(uint32_t)((e & 1) ? (cp >> 32) : cp);
             const bool live = lane_ok && e < cnt[n];
             const int64_t cell = ci / N;
