@@ -48,10 +48,12 @@ def jac_mma(elem: str, geometry: str, packed: bool = False) -> bool:
 
 def kernel_name(elem: str, geometry: str, op: str, packed: bool = False) -> str:
     E = "Hex8" if elem == "hex8" else "Wedge6"
-    if op in ("jacobian", "jac_global") and (packed or jac_mma(elem, geometry)):
+    if op in ("jacobian", "jac_global", "jac_packed") and (packed or jac_mma(elem, geometry)):
         k = ("eval_compact_mma_kernel<" if geometry == "compact" else "eval_mma_kernel<") + E + ">"
         if op == "jacobian":
             return k + " (stokesfo_jacobian)"
+        if op == "jac_packed":
+            return k + " (stokesfo_jacobian_packed)"
         if packed:
             return k + " (stokesfo_jacobian_packed) + csr_gather_kernel<packed> (stokesfo_assemble_csr_packed " \
                        "overwriting, both timed)"
@@ -74,7 +76,7 @@ def bytes_per_launch(elem: str, cells: int, nodes: int, geometry: str = "stored"
                 per node U 16 + s 8 + R 32 + coordinates 32 (x, y, z, pad)."""
     N = 8 if elem == "hex8" else 6
     Q = N
-    J = 8 * (2 * N) ** 2 if op == "jacobian" else 0
+    J = 8 * (2 * N) ** 2 if op == "jacobian" else (8 * 4 * N * (N + 1) // 2 if op == "jac_packed" else 0)
     xy = (16 + 32) if op in ("jvp", "jvp_y") else 0  # X gather, Y read+write
     rb = 0 if op == "jvp_y" else 32                   # R read + write (jvp_y: the Krylov apply, no residual)
     if op == "jac_csr":
@@ -334,7 +336,8 @@ def main():
     ap.add_argument("--global-format", default="full", choices=["packed", "full"],
                     help="--op jac_global: element matrices in symmetric block-packed form (tensor-core kernels) "
                          "or full [C][2N][2N]")
-    ap.add_argument("--op", default="jacobian", choices=["jacobian", "resid", "jvp", "jvp_y", "jac_csr", "jac_global"],
+    ap.add_argument("--op", default="jacobian", choices=["jacobian", "jac_packed", "resid", "jvp", "jvp_y", "jac_csr",
+                                                         "jac_global"],
                     help="jacobian: residual + element Jacobians (the headline); resid: stokesfo_viscosity_resid "
                          "only; jvp: matrix-free J(U) X + residual (stokesfo_jvp)")
     ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
@@ -392,7 +395,11 @@ def main():
     if world > 1 and args.op in ("jac_csr", "jac_global", "jvp_y"):
         sys.stderr.write("bench.py: --op jac_csr / jac_global / jvp_y are single-GPU lines\n")
         return 2
-    packed = args.op == "jac_global" and args.global_format == "packed" and jac_mma(elem, args.geometry, True)   # NEXT-2 through symmetric block-packed J
+    packed = (args.op == "jac_packed" or
+              (args.op == "jac_global" and args.global_format == "packed")) and jac_mma(elem, args.geometry, True)
+    if args.op == "jac_packed" and not packed:
+        sys.stderr.write("bench.py: --op jac_packed needs the tensor-core kernels (stored / compact geometry)\n")
+        return 2
     J = torch.empty((C, N * (N + 1) // 2, 2, 2) if packed else
                     ((C, 2 * N, 2 * N) if args.op in ("jacobian", "jac_global") else (0,)), dtype=torch.float64,
                     device=dev)
@@ -452,6 +459,8 @@ def main():
     def evaluate(Uc, Rc, Yc):
         if args.op == "jacobian":
             ctx.jacobian(Uc, J, R=Rc)
+        elif args.op == "jac_packed":   # symmetric block-packed element matrices (N(N+1)/2 upper node blocks)
+            ctx.jacobian_packed(Uc, J, R=Rc)
         elif args.op == "jac_csr":
             ctx.jacobian_csr(Uc, vals, R=Rc)
         elif args.op == "jac_global" and packed:   # packed element matrices, then the pull assembly
@@ -679,6 +688,8 @@ def main():
         l2_bytes = 126 * 2 ** 20
         line = {
             "metric": {"jacobian": METRIC,
+                       "jac_packed": "Stokes-FO residual + Jacobian with symmetric block-packed element matrices "
+                                     "(stokesfo_jacobian_packed) cells/s and achieved HBM GB/s",
                        "resid": "Stokes-FO residual-only (stokesfo_viscosity_resid) cells/s and achieved HBM GB/s",
                        "jvp": "Stokes-FO matrix-free J(U)X + residual (stokesfo_jvp) cells/s and achieved HBM GB/s",
                        "jvp_y": "Stokes-FO matrix-free J(U)X only (stokesfo_jvp, the Krylov operator apply) cells/s "

@@ -245,9 +245,10 @@ int stokesfo_csr_pattern(stokesfo_ctx *c, int64_t *nnz, int64_t *rowptr, int32_t
  * csr_vals[rowptr[2 conn[c][i] + a] + 2 slot + b].  Requires an earlier
  * stokesfo_csr_pattern fill (rowptr 16-B aligned); computed on the device once
  * (binary searches in colidx) into caller-owned slots: dev uint64 [C][N]
- * followed by the node -> cell incidence and a 128-B record per node for the
- * pull assembly (row base, lengths, first 8 incident cells and their slot
- * rows: one coalesced load per node) -- stokesfo_csr_slots_size bytes in all,
+ * followed by the node -> cell incidence and a record per node for the pull
+ * assembly (row base, lengths, the first 8 (hex8) / 12 (wedge6) incident
+ * cells and their slot rows: one coalesced load per node; 128 / 256 B) --
+ * stokesfo_csr_slots_size bytes in all,
  * 16-B aligned, must stay valid.  Attaches
  * the table to the ctx: stokesfo_scatter_assemble then uses it instead of
  * per-entry searches, and stokesfo_jacobian_csr becomes available.  A node

@@ -2,7 +2,7 @@
 import json
 import sys
 
-OPS = {"jacobian": "residual + Jacobian", "resid": "residual", "jvp": "J·v + residual", "jvp_y": "J·v only (Krylov apply)",
+OPS = {"jacobian": "residual + Jacobian", "jac_packed": "residual + Jacobian (symmetric block-packed J)", "resid": "residual", "jvp": "J·v + residual", "jvp_y": "J·v only (Krylov apply)",
        "jac_csr": "Jacobian into global CSR (fused, atomics)", "jac_global": "Jacobian into global CSR (element matrices + pull assembly)"}
 print("| config | elem | op | geometry | kernel | cells/s | ms/step | HBM frac | traffic / algorithmic | sustained cells/s | e2e cells/s |")
 print("|---|---|---|---|---|---|---|---|---|---|---|")
