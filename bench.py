@@ -37,11 +37,11 @@ WORKLOADS = {
 
 
 def jac_mma(elem: str, geometry: str, packed: bool = False) -> bool:
-    """The element Jacobians run on the fp64 tensor cores (eval_mma_kernel / eval_compact_mma_kernel): stored
-    or compact geometry; STOKESFO_JAC_MMA (read by stokesfo_create) unset: hex8 only, 1: both elements, 0:
+    """The element Jacobians run on the fp64 tensor cores (eval_mma_kernel / eval_compact_mma_kernel /
+    eval_otf_mma_kernel, one per geometry mode); STOKESFO_JAC_MMA (read by stokesfo_create) unset: hex8 only, 1: both elements, 0:
     neither. The packed form (stokesfo_jacobian_packed) always comes from them unless STOKESFO_JAC_MMA=0."""
     v = os.environ.get("STOKESFO_JAC_MMA")
-    if geometry == "on_the_fly" or v == "0":
+    if v == "0":
         return False
     return packed or v == "1" or elem == "hex8"
 
@@ -49,7 +49,8 @@ def jac_mma(elem: str, geometry: str, packed: bool = False) -> bool:
 def kernel_name(elem: str, geometry: str, op: str, packed: bool = False) -> str:
     E = "Hex8" if elem == "hex8" else "Wedge6"
     if op in ("jacobian", "jac_global", "jac_packed") and (packed or jac_mma(elem, geometry)):
-        k = ("eval_compact_mma_kernel<" if geometry == "compact" else "eval_mma_kernel<") + E + ">"
+        k = {"compact": "eval_compact_mma_kernel<", "on_the_fly": "eval_otf_mma_kernel<"}.get(geometry,
+                                                                                            "eval_mma_kernel<") + E + ">"
         if op == "jacobian":
             return k + " (stokesfo_jacobian)"
         if op == "jac_packed":
@@ -398,7 +399,7 @@ def main():
     packed = (args.op == "jac_packed" or
               (args.op == "jac_global" and args.global_format == "packed")) and jac_mma(elem, args.geometry, True)
     if args.op == "jac_packed" and not packed:
-        sys.stderr.write("bench.py: --op jac_packed needs the tensor-core kernels (stored / compact geometry)\n")
+        sys.stderr.write("bench.py: --op jac_packed needs the tensor-core kernels (STOKESFO_JAC_MMA not 0)\n")
         return 2
     J = torch.empty((C, N * (N + 1) // 2, 2, 2) if packed else
                     ((C, 2 * N, 2 * N) if args.op in ("jacobian", "jac_global") else (0,)), dtype=torch.float64,

@@ -219,9 +219,8 @@ int stokesfo_assemble_csr(stokesfo_ctx *c, const double *J_cell, double *csr_val
  * Jp dev [C][N(N+1)/2][2][2], block (i, j >= i) at index i N - i (i - 1) / 2 +
  * (j - i), entries [a][b] = J[(i,a),(j,b)] (hex8 1,152 B per cell instead of
  * 2,048; wedge6 672 instead of 1,152).  Jp must be 32-B aligned.  R_cell and R
- * as stokesfo_jacobian.  Written by the fp64 tensor-core kernels (stored or
- * compact geometry): on-the-fly geometry or STOKESFO_JAC_MMA=0 at create return
- * EUNSUPPORTED. */
+ * as stokesfo_jacobian.  Written by the fp64 tensor-core kernels (every
+ * geometry mode): STOKESFO_JAC_MMA=0 at create returns EUNSUPPORTED. */
 int stokesfo_jacobian_packed(stokesfo_ctx *c, const double *U, double *Jp, double *R_cell, double *R);
 
 /* stokesfo_assemble_csr from the packed form: row (i, a) of cell c is block

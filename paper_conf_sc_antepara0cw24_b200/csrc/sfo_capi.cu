@@ -199,6 +199,20 @@ int configure_compact_mma(int *grid) {
     return STOKESFO_OK;
 }
 
+template <class E>
+int configure_otf_mma(int *grid) {
+    auto fn = eval_otf_mma_kernel<E>;
+    constexpr int bytes = OtfMmaSmem<E>::BYTES;
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
+        return cuda_status();
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 32, bytes) != cudaSuccess) return cuda_status();
+    *grid = std::max(1, sms * std::max(1, per_sm));
+    return STOKESFO_OK;
+}
+
 // Element Jacobians on the fp64 tensor cores. STOKESFO_JAC_MMA unset: hex8 (the DMMA kernels cost the same per
 // cell for both elements, which beats the vector kernel for hex8's 8 x 8 node blocks but not for wedge6's
 // padded 6 x 6); 1: both elements; 0: neither (and no packed form). The DMMA kernels are configured
@@ -245,6 +259,9 @@ int create_impl(stokesfo_ctx *c) {
         if (st) return st;
         st = configure_otf<E, M_DIAG>(&c->grid_diag);
         if (st) return st;
+        c->jac_mma = want_jac_mma<E>();
+        c->mma_ok = jac_mma_env() != 0;
+        if (c->mma_ok && (st = configure_otf_mma<E>(&c->grid_mma))) return st;
     } else {
         // ring depth: default per element, STOKESFO_STAGES_{RESID,JAC} override (2 or 3)
         c->nstage_resid = default_stages<E, false>();
@@ -372,7 +389,7 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
                 : MODE == M_DIAG ? c->grid_diag : c->grid_resid;
     const bool otf = c->mode == STOKESFO_GEOMETRY_ON_THE_FLY;
     // the DMMA kernels store J with 32-B vector stores (16-B aligned J_cell: the vector kernels)
-    const bool mma = MODE == M_JAC && !otf && c->mma_ok && (c->jac_mma || packed) && aligned(J_cell, 32);
+    const bool mma = MODE == M_JAC && c->mma_ok && (c->jac_mma || packed) && aligned(J_cell, 32);
     if (packed && !mma) return STOKESFO_EUNSUPPORTED;  // the packed form comes from the DMMA kernels only
     a.use_jmap = (!otf && !mma && MODE == M_JAC && wedge_jmap<E>(c, J_cell)) ? 1 : 0;
     const CUtensorMap jm = a.use_jmap ? c->jmap : CUtensorMap{};
@@ -385,6 +402,8 @@ int eval_impl(stokesfo_ctx *c, const double *U, double *mu_qp, double *R_cell, d
     else if (c->mode == STOKESFO_GEOMETRY_COMPACT)
         eval_compact_kernel<E, MODE><<<(int)std::min<int64_t>(g, c->ntiles), 32, CompactSmem<E, MODE>::BYTES,
                                         c->stream>>>(a, jm);
+    else if (mma && otf)
+        eval_otf_mma_kernel<E><<<gm, 32, OtfMmaSmem<E>::BYTES, c->stream>>>(a);
     else if (otf)
         eval_otf_kernel<E, MODE><<<grid, 32, OtfSmem<E, MODE>::BYTES, c->stream>>>(a);
     else if (mma)

@@ -1987,6 +1987,143 @@ __global__ void __launch_bounds__(32, (forms_jac<MODE>() ? SFO_OTF_JAC_WARPS : 1
     (void)live_cur;
 }
 
+// ---- G4 with on-the-fly geometry on the fp64 tensor cores (residual + element Jacobians) ----
+// eval_otf_kernel's input ring (register gather of U, s and cell-local coordinates one tile ahead, conn / k_c two
+// tiles ahead) and per-QP phase (J_q from the coordinates, det J, cofactors, GradBF into the per-warp region in the
+// record slot layout), with the DMMA per-node phase of eval_mma_kernel (mma_node_phase). No J staging: the
+// shared memory per warp is the two input buffers + GradBF + per-QP scalars.
+template <class E>
+struct OtfMmaSmem {
+    using O = OtfSmem<E, M_JAC>;
+    static constexpr int IN_BYTES = O::IN_BYTES;
+    static constexpr int OFF_G = 2 * IN_BYTES;
+    static constexpr int OFF_QS = OFF_G + E::Q * 3 * E::SLAB * 8;
+    static constexpr int BYTES = OFF_QS + qs_mma_bytes<E>();
+    static_assert(OFF_G % 128 == 0 && OFF_QS % 16 == 0, "alignment");
+};
+
+template <class E>
+__global__ void __launch_bounds__(32, SFO_MMA_JAC_WARPS) eval_otf_mma_kernel(EvalArgs a) {
+    constexpr int N = E::N, TC = E::TC;
+    using S = OtfMmaSmem<E>;
+    using O = typename S::O;
+    extern __shared__ __align__(128) char smem[];
+    double *rg = reinterpret_cast<double *>(smem + S::OFF_G);
+    const QsMma<E> qs{reinterpret_cast<double *>(smem + S::OFF_QS)};
+    const int l = threadIdx.x;
+    const bool act = l < TC * N;
+    const int c = act ? E::lane_cell(l) : TC, s = act ? E::lane_sub(l) : 0;  // per-QP phase: (cell, qp)
+    const int ni = l >> 2, qq = l & 3;                                       // DMMA fragments: (node, qp quad)
+    const bool have_s = (a.surface != nullptr) && (a.force_qp == nullptr);
+    const uint64_t pol_stream = policy_evict_first();
+
+    double xq, yq, zq, wq;
+    qp_coords<E>(act ? s : 0, xq, yq, zq, wq);
+    double phi[2];
+    mma_phi<E>(ni, qq, phi);
+
+    auto load_tile = [&](int64_t tile, int32_t &g, double &kcv, bool &live) {
+        const int64_t cell = tile * TC + c;
+        live = act && tile < a.ntiles && cell < a.ncells;
+        g = live ? __ldg(a.conn + cell * N + s) : 0;
+        kcv = live ? (a.kc ? __ldg(a.kc + cell) : a.kscal) : 0.0;
+    };
+    int32_t g_cur, g_nxt;
+    double kc_cur, kc_nxt;
+    bool live_cur, live_nxt;
+    load_tile(blockIdx.x, g_cur, kc_cur, live_cur);
+    load_tile(blockIdx.x + (int64_t)gridDim.x, g_nxt, kc_nxt, live_nxt);
+    if ((int64_t)blockIdx.x < a.ntiles)
+        otf_store<E, M_JAC>(smem, otf_load<M_JAC>(g_cur, live_cur, a.U, a.xyz4, a.surface, have_s, nullptr), c, s,
+                            act);
+
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x, ++it) {
+        const char *in = smem + (it & 1) * S::IN_BYTES;
+        const double2 *Us = reinterpret_cast<const double2 *>(in + O::IN_U);
+        const double2 *XY = reinterpret_cast<const double2 *>(in + O::IN_XY);
+        const double *Zs = reinterpret_cast<const double *>(in + O::IN_Z);
+        const double *ss = reinterpret_cast<const double *>(in + O::IN_S);
+        const int64_t cell0 = tile * TC;
+        const int nvalid = (a.ncells - cell0 < (int64_t)TC) ? (int)(a.ncells - cell0) : TC;
+
+        __syncwarp();  // this tile's gathered inputs are visible; the previous node phase is done with G and qs
+
+        // ---- per-QP phase: geometry, GradBF -> smem, then Ugrad etc. (as eval_otf_kernel) ----
+        const double kc = __shfl_sync(0xffffffffu, kc_cur, act ? E::lane_of(c, 0) : 0);
+        if (act) {
+            const int q = s;
+            double dq[N][3];
+#pragma unroll
+            for (int n = 0; n < N; ++n) {
+                double ph;
+                basis<E>(n, xq, yq, zq, ph, dq[n][0], dq[n][1], dq[n][2]);
+            }
+            double J00 = 0, J01 = 0, J02 = 0, J10 = 0, J11 = 0, J12 = 0, J20 = 0, J21 = 0, J22 = 0;
+#pragma unroll
+            for (int n = 1; n < N; ++n) {  // cell-local: node 0 sits at the origin
+                const double2 xy = XY[c * O::UP + n];
+                const double z = Zs[c * O::UP + n];
+                const double d0 = dq[n][0], d1 = dq[n][1], d2 = dq[n][2];
+                J00 = fma(xy.x, d0, J00); J01 = fma(xy.x, d1, J01); J02 = fma(xy.x, d2, J02);
+                J10 = fma(xy.y, d0, J10); J11 = fma(xy.y, d1, J11); J12 = fma(xy.y, d2, J12);
+                J20 = fma(z, d0, J20); J21 = fma(z, d1, J21); J22 = fma(z, d2, J22);
+            }
+            const double c00 = J11 * J22 - J12 * J21, c01 = J12 * J20 - J10 * J22, c02 = J10 * J21 - J11 * J20;
+            const double c10 = J02 * J21 - J01 * J22, c11 = J00 * J22 - J02 * J20, c12 = J01 * J20 - J00 * J21;
+            const double c20 = J01 * J12 - J02 * J11, c21 = J02 * J10 - J00 * J12, c22 = J00 * J11 - J01 * J10;
+            const double det = J00 * c00 + J01 * c01 + J02 * c02;
+            if (!(det > 0.0) && c < nvalid) atomicOr(a.err, ERR_DETJ);
+            const double id = 1.0 / det;
+            double ux = 0, uy = 0, uz = 0, vx = 0, vy = 0, vz = 0, gs0 = 0, gs1 = 0;
+#pragma unroll
+            for (int n = 0; n < N; ++n) {
+                const double d0 = dq[n][0], d1 = dq[n][1], d2 = dq[n][2];
+                const double g0 = fma(c00, d0, fma(c01, d1, c02 * d2)) * id;
+                const double g1 = fma(c10, d0, fma(c11, d1, c12 * d2)) * id;
+                const double g2 = fma(c20, d0, fma(c21, d1, c22 * d2)) * id;
+                rg[gidx<E>(n, q, 0, c)] = g0;
+                rg[gidx<E>(n, q, 1, c)] = g1;
+                rg[gidx<E>(n, q, 2, c)] = g2;
+                const double2 uv = Us[c * O::UP + n];
+                ux = fma(uv.x, g0, ux); uy = fma(uv.x, g1, uy); uz = fma(uv.x, g2, uz);
+                vx = fma(uv.y, g0, vx); vy = fma(uv.y, g1, vy); vz = fma(uv.y, g2, vz);
+                if (have_s) {
+                    const double sn = ss[c * O::UP + n];
+                    gs0 = fma(sn, g0, gs0); gs1 = fma(sn, g1, gs1);
+                }
+            }
+            qp_tail<E, M_JAC>(a, qs, c, q, nvalid, cell0, have_s, kc, wq * det, ux, uy, uz, vx, vy, vz, gs0, gs1);
+        }
+        __syncwarp();
+
+        // ---- per-node phase on the tensor cores (+ register gather of the next tile, conn of the one after) ----
+        int32_t gnode[2];  // lane (ni, qq) scatters (cell qq, node ni) [and wedge6's (cell 4, node ni)]
+        {
+            const int nn = ni < N ? ni : 0;
+            gnode[0] = __shfl_sync(0xffffffffu, g_cur, E::lane_of(qq < TC ? qq : 0, nn));
+            gnode[1] = __shfl_sync(0xffffffffu, g_cur, E::lane_of(TC > 4 ? 4 : 0, nn));
+        }
+        int32_t g_nn = 0;
+        double kc_nn = 0.0;
+        bool live_nn = false;
+        OtfGathered nxt{make_double2(0.0, 0.0), make_double2(0.0, 0.0), make_double2(0.0, 0.0), 0.0, 0.0};
+        double Rm[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
+        mma_node_phase<E, SFO_MMA_UNROLL_COMPACT>(a.J_cell, rg, qs, phi, cell0, nvalid, ni, qq, pol_stream, Rm,
+                                                  a.packed != 0, [&]() {
+            if (tile + gridDim.x < a.ntiles)
+                nxt = otf_load<M_JAC>(g_nxt, live_nxt, a.U, a.xyz4, a.surface, have_s, nullptr);
+            load_tile(tile + 2 * (int64_t)gridDim.x, g_nn, kc_nn, live_nn);
+        });
+        mma_scatter_r<E>(a, gnode, Rm, cell0, nvalid, ni, qq);
+        // the other input buffer was last read in the previous tile's per-QP phase
+        if (tile + gridDim.x < a.ntiles) otf_store<E, M_JAC>(smem + ((it + 1) & 1) * S::IN_BYTES, nxt, c, s, act);
+        g_cur = g_nxt; kc_cur = kc_nxt; live_cur = live_nxt;
+        g_nxt = g_nn; kc_nxt = kc_nn; live_nxt = live_nn;
+    }
+    (void)live_cur;
+}
+
 // Setup for the on-the-fly mode: node coordinates as double4.
 __global__ void xyz4_kernel(int64_t nnodes, const double *__restrict__ coords, double4 *__restrict__ xyz4) {
     const int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;

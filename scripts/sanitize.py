@@ -39,7 +39,7 @@ def run(elem, n, L, drop, full):
         ctx.jacobian_csr(Ud, vals, R=R)
         ctx.scatter_assemble(R_cell=Rc, R=R, J_cell=J, csr_vals=vals)
         ctx.assemble_csr(J, vals, accumulate=False)
-        if geo != "on_the_fly":  # tensor-core kernels: packed element matrices + their pull assembly
+        if True:  # tensor-core kernels: packed element matrices + their pull assembly
             Jp = torch.empty((C, N * (N + 1) // 2, 2, 2), dtype=torch.float64, device="cuda")
             ctx.jacobian_packed(Ud, Jp, R_cell=Rc, R=R)
             ctx.assemble_csr_packed(Jp, vals, accumulate=True)

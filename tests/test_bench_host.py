@@ -124,7 +124,8 @@ def test_global_fill_byte_model_packed(monkeypatch):
     # which kernels a line names: tensor cores for hex8 by default, packed global fill on them too
     monkeypatch.delenv("STOKESFO_JAC_MMA", raising=False)
     assert bench.jac_mma("hex8", "stored") and not bench.jac_mma("wedge6", "stored")
-    assert bench.jac_mma("wedge6", "compact", packed=True) and not bench.jac_mma("hex8", "on_the_fly")
+    assert bench.jac_mma("wedge6", "compact", packed=True) and bench.jac_mma("hex8", "on_the_fly")
+    assert bench.kernel_name("hex8", "on_the_fly", "jacobian").startswith("eval_otf_mma_kernel<Hex8>")
     assert bench.kernel_name("hex8", "compact", "jacobian").startswith("eval_compact_mma_kernel<Hex8>")
     monkeypatch.setenv("STOKESFO_JAC_MMA", "0")
     assert not bench.jac_mma("hex8", "stored", packed=True)

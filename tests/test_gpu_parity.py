@@ -486,7 +486,7 @@ def _unpack_blocks(Jp, N):
     return J
 
 
-@pytest.mark.parametrize("geometry", ["stored", "compact"])
+@pytest.mark.parametrize("geometry", GEOMS)
 @pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 0), ("wedge6", 11)])
 def test_jacobian_packed_and_assembly(torch, elem, drop, geometry):
     """NEXT-2 symmetric block-packed element matrices (stokesfo_jacobian_packed): unpacked, they match the
@@ -531,10 +531,10 @@ def test_jacobian_packed_and_assembly(torch, elem, drop, geometry):
 
 
 def test_jacobian_packed_unsupported(torch, monkeypatch):
-    """The packed form comes from the tensor-core kernels only: on-the-fly geometry, or STOKESFO_JAC_MMA=0
-    at create, returns EUNSUPPORTED (a loud error, no silent fallback)."""
+    """The packed form comes from the tensor-core kernels only: STOKESFO_JAC_MMA=0 at create returns
+    EUNSUPPORTED in every geometry mode (a loud error, no silent fallback)."""
     from paper_conf_sc_antepara0cw24_b200.stokesfo import StokesFOError
-    for geometry, mma in (("on_the_fly", "1"), ("stored", "0")):
+    for geometry, mma in (("on_the_fly", "0"), ("stored", "0"), ("compact", "0")):
         monkeypatch.setenv("STOKESFO_JAC_MMA", mma)
         ctx, orc = _setup(torch, "hex8", n=4, L=2, geometry=geometry)
         C, N = ctx.num_cells, ctx.N
@@ -569,7 +569,7 @@ def test_wedge_tensor_map_store(torch, drop, monkeypatch):
     assert _cell_rel(a[:C], ref["J_cell"]) <= TOL
 
 
-@pytest.mark.parametrize("geometry", ["stored", "compact"])
+@pytest.mark.parametrize("geometry", GEOMS)
 @pytest.mark.parametrize("elem,drop", [("hex8", 0), ("hex8", 3), ("wedge6", 0), ("wedge6", 11)])
 def test_jacobian_tensor_core_vs_vector(torch, elem, drop, geometry, monkeypatch):
     """The element Jacobians on the fp64 tensor cores (eval_mma_kernel / eval_compact_mma_kernel; default for
