@@ -97,8 +97,8 @@ def test_fullsize_residual_only_sampled(cfg):
 @pytest.mark.parametrize("cfg", ["C3", "C5"])
 def test_fullsize_csr_assembly_sampled_rows(cfg):
     """NEXT-2 at full size: CSR pattern rows (bit-exact vs the incident cells' node sets),
-    pull assembly of stokesfo_jacobian's element matrices and the fused jacobian_csr,
-    on sampled rows recomputed by the oracle."""
+    pull assembly of stokesfo_jacobian's element matrices, the fused jacobian_csr and the
+    packed path (jacobian_packed + assemble_csr_packed), on sampled rows recomputed by the oracle."""
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
@@ -139,19 +139,25 @@ def test_fullsize_csr_assembly_sampled_rows(cfg):
                 # bound consistent with the per-cell element tolerance: sum of max|J_cell| of contributing cells
                 np.add.at(absv, pos, np.full(2 * N, np.abs(out["J_cell"][r]).max()))
     nnz = colidx.numel()
-    for fused in (False, True):
+    for how in ("pull", "fused", "packed"):
         vals = torch.zeros(nnz, dtype=torch.float64, device="cuda")
-        if fused:
+        if how == "fused":
             ctx.jacobian_csr(Ud, vals)
-        else:
+        elif how == "pull":
             J = torch.empty((C, 2 * N, 2 * N), dtype=torch.float64, device="cuda")
             ctx.jacobian(Ud, J)
             ctx.scatter_assemble(J_cell=J, csr_vals=vals)
             del J
+        else:  # symmetric block-packed element matrices (tensor cores) + their pull assembly, overwriting
+            Jp = torch.empty((C, ctx.packed_blocks, 2, 2), dtype=torch.float64, device="cuda")
+            ctx.jacobian_packed(Ud, Jp)
+            vals.fill_(float("nan"))
+            ctx.assemble_csr_packed(Jp, vals, accumulate=False)
+            del Jp
         ctx.sync()
         for (v, a), (cols, val, absv) in want.items():
             got = vals[int(rp[2 * v + a]):int(rp[2 * v + a + 1])].cpu().numpy()
-            assert (np.abs(got - val) <= TOL * absv + 1e-300).all(), (fused, v, a)
+            assert (np.abs(got - val) <= TOL * absv + 1e-300).all(), (how, v, a)
         del vals
         torch.cuda.empty_cache()
 
